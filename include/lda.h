@@ -1,0 +1,187 @@
+/*
+ * include/lda.h — C ABI of the B200-native LDA collapsed-Gibbs sweep
+ * (the hot path of CuLDA_CGS, Xie, Liang, Li, Tan, HPDC'19).
+ *
+ * Citations "L<n>" are lines of the paper transcript /root/reference/PAPER.md;
+ * "X<n>" are the readings of ambiguous passages listed in DESIGN.md.
+ *
+ * What the library computes (§2.1, §6):
+ *   corpus: D documents of tokens, each token an instance of a word in [0,V)
+ *           (L369-383).
+ *   model : θ (n_dk, doc-topic counts, sparse), ϕ (n_wk, word-topic counts,
+ *           dense) and n_k = Σ_w n_wk (L391-397, Eq. 1 denominator L407).
+ *   sweep : every token draws a new topic from
+ *             p(k) ∝ (n_dk + α)(n_wk + β) / (n_k + Vβ)            (Eq. 1)
+ *           against the counts frozen at the start of the sweep (L415-421,
+ *           X3), via the split p = p1 + p2 (Eq. 6-8),
+ *           one Philox4x32-10 uniform per token keyed by (seed; canonical
+ *           token index c, sweep t) (X9); then n_wk, n_k and θ are rebuilt
+ *           (§6.2).  Multi-GPU: documents are partitioned, n_wk/n_k
+ *           are sum-allreduced after every sweep (Eq. 4).
+ *
+ * Conventions for every call:
+ *   - Return 0 (LDA_OK) or a negative lda_status.  No exceptions cross the ABI.
+ *   - Input pointers are HOST pointers, borrowed for the duration of the call
+ *     only (the library copies).  Output buffers are caller-allocated host
+ *     memory; passing NULL skips that output.
+ *   - A context is single-threaded: do not call into one context from two
+ *     threads at once.
+ *   - Sticky failures: a CUDA or NCCL error marks the context failed; every
+ *     later call on it returns the same code until lda_destroy.
+ *     lda_last_error() gives a human-readable detail.
+ *   - Call order: lda_create -> [lda_set_option]* -> [lda_init_dist] ->
+ *     lda_load_corpus -> (lda_iterate | lda_loglik | lda_get_counts |
+ *     lda_get_stats | lda_set_z)* -> lda_destroy.  Calls that need a corpus
+ *     return LDA_ESTATE before a successful lda_load_corpus.
+ */
+#ifndef LDA_H
+#define LDA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct lda_ctx lda_ctx; /* opaque; owned by the library */
+
+typedef enum {
+    LDA_OK = 0,
+    LDA_EINVAL = -1, /* invalid argument or corpus */
+    LDA_ERANGE = -2, /* a size exceeds a representable range / buffer too small */
+    LDA_ENOMEM = -3, /* host or device allocation failed */
+    LDA_ECUDA = -4,  /* CUDA runtime error (including: no device) */
+    LDA_ENCCL = -5,  /* NCCL error */
+    LDA_ESTATE = -6  /* call out of order */
+} lda_status;
+
+/* Per-call statistics of the last lda_iterate (device time from CUDA events
+ * on the library's streams). */
+typedef struct lda_stats {
+    int64_t sweeps_done;    /* global sweep counter t after the last call */
+    int64_t local_tokens;   /* T_g: tokens held by this rank */
+    int64_t local_docs;     /* D_g */
+    int64_t global_tokens;  /* T */
+    int32_t last_n;         /* sweeps in the last lda_iterate call */
+    int32_t world;          /* ranks */
+    double ms_total;        /* compute-stream time of the last call, all sweeps */
+    double ms_sample;       /* prologue + sampling kernel (Alg. 2, K1) */
+    double ms_recount;      /* n_wk / n_k rebuild (K2) */
+    double ms_theta;        /* θ rebuild (K3+K4) */
+    double ms_allreduce;    /* raw NCCL allreduce time on the comm stream (0 if world==1) */
+    double ms_last_sweep;   /* compute-stream time of the last sweep only */
+    double ms_last_sample;  /* sampling kernel time of the last sweep only */
+    int64_t sum_nnz_tok;    /* Σ_t nnz_{d(t)} read by the last sweep's sampler */
+    int64_t sum_nnz_doc;    /* Σ_d nnz_d of θ after the last sweep */
+    int64_t n_launches;     /* library kernels launched by the last call */
+    int64_t n_sample_chunks;/* sampler work items (word chunks) */
+} lda_stats;
+
+/* Create a context.  D = global number of documents, V = vocabulary size,
+ * K = number of topics, α, β = Dirichlet hyper-parameters (Eq. 1; the paper
+ * uses α = 50/K, β = 0.01 at L1339, X1).  No device work is done.
+ * Errors: LDA_EINVAL unless D >= 1, V >= 1, 1 <= K <= 65536 (topic ids are
+ * uint16, L1239-1243), α and β finite and > 0.  *out is set to NULL on error. */
+int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_ctx **out);
+
+/* Set an integer option before lda_load_corpus (LDA_ESTATE after).  Keys:
+ *   "device"        CUDA device ordinal (default 0)
+ *   "exclude_self"  0 (default; Eq. 1 as printed, X2) or 1 (remove the
+ *                   token's own old topic from the counts it draws against)
+ *   "chunk_tokens"  max tokens per sampling work item (default 4096)
+ *   "recount_tokens" max tokens per n_wk recount work item (default 65536)
+ *   "tile_tokens"   split the documents into tiles of about this many tokens
+ *                   and sample tile by tile (0 = one tile, the default)
+ *   "threads"       host threads for corpus preparation (default: all)
+ * Results do not depend on chunk_tokens, recount_tokens, tile_tokens or
+ * threads (the draw of every token is a function of the frozen counts and
+ * its canonical index only).
+ * Unknown key or bad value: LDA_EINVAL. */
+int lda_set_option(lda_ctx *ctx, const char *key, int64_t value);
+
+/* Multi-GPU: join a communicator of `world` ranks as `rank` (one process per
+ * GPU).  nccl_unique_id points to the 128-byte ncclUniqueId that rank 0 made
+ * with lda_nccl_unique_id and the caller broadcast (e.g. through
+ * torch.distributed).  Must precede lda_load_corpus.  world == 1 is allowed
+ * (no communicator is made).  Errors: LDA_EINVAL, LDA_ESTATE, LDA_ENCCL. */
+int lda_init_dist(lda_ctx *ctx, int32_t rank, int32_t world, const void *nccl_unique_id);
+
+/* Write a fresh 128-byte ncclUniqueId to out128 (host-only helper). */
+int lda_nccl_unique_id(void *out128);
+
+/* Token-balanced contiguous document partition (§4 "evenly
+ * partitioned by number of tokens", X21): rank g owns documents
+ * [doc_begin[g], doc_begin[g+1]), where doc_begin[g] is the first d with
+ * doc_ptr[d] >= ceil(g*T/world), doc_begin[0] = 0, doc_begin[world] = D.
+ * doc_ptr: D+1 non-decreasing offsets (doc_ptr[0] == 0, T = doc_ptr[D]);
+ * doc_begin: world+1 outputs.  Host-only.  Errors: LDA_EINVAL. */
+int lda_partition_docs(int64_t D, const int64_t *doc_ptr, int32_t world, int64_t *doc_begin);
+
+/* Load this rank's documents [doc_begin, doc_end) of the global corpus,
+ * randomly initialise every token's topic (L377-379; Philox at t = 0, X10)
+ * and build n_wk, n_k and θ (allreduced across ranks when world > 1).
+ *   doc_ptr : doc_end-doc_begin+1 offsets into `words`, doc_ptr[0] == 0,
+ *             non-decreasing (empty documents are allowed)
+ *   words   : doc-major token word ids, each in [0, V)
+ *   seed    : 64-bit Philox key (X9)
+ * Every rank must pass the same seed.  With world == 1 pass the whole corpus
+ * (doc_begin = 0, doc_end = D).  Errors: LDA_EINVAL (bad ids/offsets/range),
+ * LDA_ERANGE (a document longer than 65535 tokens, or >= 2^32 local tokens),
+ * LDA_ENOMEM, LDA_ECUDA, LDA_ENCCL, LDA_ESTATE (called twice). */
+int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int64_t *doc_ptr,
+                    const int32_t *words, uint64_t seed);
+
+/* Run n_sweeps >= 0 sweeps (iterations, L415-421).  Synchronous: returns after
+ * the last sweep's counts are rebuilt on every rank.  Collective when
+ * world > 1.  Errors: LDA_EINVAL (n < 0), LDA_ESTATE, LDA_ECUDA, LDA_ENCCL. */
+int lda_iterate(lda_ctx *ctx, int32_t n_sweeps);
+
+/* Per-token log-likelihood of the current state (Fig. 8; formula
+ * of reading X11, the collapsed joint log p(w, z | α, β) divided by the global
+ * token count T).  Collective when world > 1. */
+int lda_loglik(lda_ctx *ctx, double *ll_per_token);
+
+/* Copy the model out (Alg. 1 lines 17-20, L829-835).  Any pointer may be NULL.
+ *   n_wk       : V*K int32, row-major by word (X13) — global counts
+ *   n_k        : K int32
+ *   ndk_ptr    : D_g+1 int64 CSR offsets of θ for this rank's documents
+ *   ndk_topic, ndk_count : ndk_capacity entries each; topics ascending per row
+ *   ndk_nnz_out: receives Σ_d nnz_d (the capacity needed).  If ndk_topic or
+ *                ndk_count is non-NULL and ndk_capacity < nnz the call writes
+ *                *ndk_nnz_out and returns LDA_ERANGE.
+ *   z          : T_g uint16 topics in input (doc-major) order */
+int lda_get_counts(lda_ctx *ctx, int32_t *n_wk, int32_t *n_k, int64_t *ndk_ptr,
+                   uint16_t *ndk_topic, int32_t *ndk_count, int64_t ndk_capacity,
+                   int64_t *ndk_nnz_out, uint16_t *z);
+
+/* Statistics of the last lda_iterate call. */
+int lda_get_stats(lda_ctx *ctx, lda_stats *out);
+
+/* Per-sweep log of the last lda_iterate call: up to `cap` entries of each
+ * non-NULL array (device ms per sweep and per phase; Σ_t nnz_{d(t)} of the θ
+ * each sweep sampled against).  *n_out = number of sweeps in that call. */
+int lda_get_sweep_log(lda_ctx *ctx, int32_t cap, double *ms_sweep, double *ms_sample, double *ms_recount,
+                      double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int32_t *n_out);
+
+/* The CUDA stream (cudaStream_t) the sweep kernels run on; valid after
+ * lda_load_corpus until lda_destroy. */
+int lda_get_stream(lda_ctx *ctx, void **stream);
+
+/* Test hook (teacher forcing): replace every local token's topic with z
+ * (T_g uint16, input order, each < K) and rebuild all counts (collective when
+ * world > 1).  Does not advance the sweep counter. */
+int lda_set_z(lda_ctx *ctx, const uint16_t *z);
+
+/* Free everything (NULL is a no-op). */
+void lda_destroy(lda_ctx *ctx);
+
+/* Detail of the last failure on ctx ("" if none; a static string for NULL). */
+const char *lda_last_error(const lda_ctx *ctx);
+
+/* Library version string. */
+const char *lda_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LDA_H */

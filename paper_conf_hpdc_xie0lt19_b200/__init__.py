@@ -1,1 +1,296 @@
-"""B200-native LDA collapsed-Gibbs sweep (CuLDA_CGS hot path)."""
+"""B200-native LDA collapsed-Gibbs sweep (the CuLDA_CGS hot path).
+
+Thin ctypes binding of the C ABI in ``include/lda.h`` (argument marshalling
+only; every step of the sweep runs in the library's CUDA kernels).  The
+functions keep the ABI's names; :class:`LDA` strings them together.
+
+The library ``liblda.so`` is built in-tree by ``_build.build()``
+(``__graft_entry__.build()``).  There is no fallback: if the library is
+missing or the GPU is absent the calls raise ``LDAError``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "liblda.so")
+
+LDA_OK, LDA_EINVAL, LDA_ERANGE, LDA_ENOMEM, LDA_ECUDA, LDA_ENCCL, LDA_ESTATE = 0, -1, -2, -3, -4, -5, -6
+STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4: "LDA_ECUDA",
+          -5: "LDA_ENCCL", -6: "LDA_ESTATE"}
+
+# every symbol include/lda.h declares
+ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_partition_docs",
+               "lda_load_corpus", "lda_iterate", "lda_loglik", "lda_get_counts", "lda_get_stats",
+               "lda_get_sweep_log", "lda_get_stream", "lda_set_z", "lda_destroy", "lda_last_error",
+               "lda_version")
+
+
+class LDAError(RuntimeError):
+    def __init__(self, code, msg=""):
+        self.code = code
+        super().__init__(f"{STATUS.get(code, code)}: {msg}")
+
+
+class lda_stats(ctypes.Structure):
+    _fields_ = [("sweeps_done", ctypes.c_int64), ("local_tokens", ctypes.c_int64),
+                ("local_docs", ctypes.c_int64), ("global_tokens", ctypes.c_int64),
+                ("last_n", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("ms_total", ctypes.c_double), ("ms_sample", ctypes.c_double),
+                ("ms_recount", ctypes.c_double), ("ms_theta", ctypes.c_double),
+                ("ms_allreduce", ctypes.c_double), ("ms_last_sweep", ctypes.c_double),
+                ("ms_last_sample", ctypes.c_double), ("sum_nnz_tok", ctypes.c_int64),
+                ("sum_nnz_doc", ctypes.c_int64), ("n_launches", ctypes.c_int64),
+                ("n_sample_chunks", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+_lib = None
+_vp = ctypes.c_void_p
+_i64, _i32, _u64, _f64 = ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, ctypes.c_double
+
+
+def lib():
+    """Load liblda.so (raises if it has not been built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise LDAError(LDA_ECUDA, f"{LIB_PATH} not built; run __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        sig = {
+            "lda_create": ([_i64, _i32, _i32, _f64, _f64, ctypes.POINTER(_vp)], ctypes.c_int),
+            "lda_set_option": ([_vp, ctypes.c_char_p, _i64], ctypes.c_int),
+            "lda_init_dist": ([_vp, _i32, _i32, _vp], ctypes.c_int),
+            "lda_nccl_unique_id": ([_vp], ctypes.c_int),
+            "lda_partition_docs": ([_i64, _vp, _i32, _vp], ctypes.c_int),
+            "lda_load_corpus": ([_vp, _i64, _i64, _vp, _vp, _u64], ctypes.c_int),
+            "lda_iterate": ([_vp, _i32], ctypes.c_int),
+            "lda_loglik": ([_vp, ctypes.POINTER(_f64)], ctypes.c_int),
+            "lda_get_counts": ([_vp, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp], ctypes.c_int),
+            "lda_get_stats": ([_vp, ctypes.POINTER(lda_stats)], ctypes.c_int),
+            "lda_get_sweep_log": ([_vp, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp], ctypes.c_int),
+            "lda_get_stream": ([_vp, ctypes.POINTER(_vp)], ctypes.c_int),
+            "lda_set_z": ([_vp, _vp], ctypes.c_int),
+            "lda_destroy": ([_vp], None),
+            "lda_last_error": ([_vp], ctypes.c_char_p),
+            "lda_version": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+    return _lib
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(_vp)
+
+
+def _check(rc, ctx=None):
+    if rc != LDA_OK:
+        msg = lib().lda_last_error(ctx).decode() if ctx else ""
+        raise LDAError(rc, msg)
+
+
+# ---------------------------------------------------------------------------
+# same-name wrappers of the C ABI
+# ---------------------------------------------------------------------------
+
+def lda_version() -> str:
+    return lib().lda_version().decode()
+
+
+def lda_create(D, V, K, alpha, beta):
+    h = _vp()
+    _check(lib().lda_create(int(D), int(V), int(K), float(alpha), float(beta), ctypes.byref(h)))
+    return h
+
+
+def lda_set_option(ctx, key, value):
+    _check(lib().lda_set_option(ctx, key.encode(), int(value)), ctx)
+
+
+def lda_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().lda_nccl_unique_id(buf))
+    return buf.raw
+
+
+def lda_init_dist(ctx, rank, world, unique_id: bytes | None):
+    buf = ctypes.create_string_buffer(unique_id, 128) if unique_id is not None else None
+    _check(lib().lda_init_dist(ctx, int(rank), int(world), buf), ctx)
+
+
+def lda_partition_docs(doc_ptr, world):
+    doc_ptr = np.ascontiguousarray(doc_ptr, np.int64)
+    out = np.empty(int(world) + 1, np.int64)
+    _check(lib().lda_partition_docs(len(doc_ptr) - 1, _p(doc_ptr), int(world), _p(out)))
+    return out
+
+
+def lda_load_corpus(ctx, doc_begin, doc_end, doc_ptr, words, seed):
+    doc_ptr = np.ascontiguousarray(doc_ptr, np.int64)
+    words = np.ascontiguousarray(words, np.int32)
+    _check(lib().lda_load_corpus(ctx, int(doc_begin), int(doc_end), _p(doc_ptr), _p(words),
+                                 int(seed) & 0xFFFFFFFFFFFFFFFF), ctx)
+
+
+def lda_iterate(ctx, n):
+    _check(lib().lda_iterate(ctx, int(n)), ctx)
+
+
+def lda_loglik(ctx) -> float:
+    v = _f64()
+    _check(lib().lda_loglik(ctx, ctypes.byref(v)), ctx)
+    return v.value
+
+
+def lda_get_counts(ctx, n_wk=None, n_k=None, ndk_ptr=None, ndk_topic=None, ndk_count=None, z=None):
+    """Fills the given (preallocated, C-contiguous) numpy arrays; returns nnz."""
+    nnz = _i64()
+    cap = 0 if ndk_topic is None else len(ndk_topic)
+    if ndk_count is not None:
+        cap = len(ndk_count) if ndk_topic is None else min(cap, len(ndk_count))
+    _check(lib().lda_get_counts(ctx, _p(n_wk), _p(n_k), _p(ndk_ptr), _p(ndk_topic), _p(ndk_count), cap,
+                                ctypes.byref(nnz), _p(z)), ctx)
+    return nnz.value
+
+
+def lda_get_stats(ctx) -> dict:
+    s = lda_stats()
+    _check(lib().lda_get_stats(ctx, ctypes.byref(s)), ctx)
+    return s.as_dict()
+
+
+def lda_get_sweep_log(ctx) -> dict:
+    n = _i32()
+    _check(lib().lda_get_sweep_log(ctx, 0, None, None, None, None, None, None, ctypes.byref(n)), ctx)
+    m = n.value
+    arr = {k: np.zeros(m, np.float64) for k in ("ms_sweep", "ms_sample", "ms_recount", "ms_theta", "ms_allreduce")}
+    nnz = np.zeros(m, np.int64)
+    _check(lib().lda_get_sweep_log(ctx, m, _p(arr["ms_sweep"]), _p(arr["ms_sample"]), _p(arr["ms_recount"]),
+                                   _p(arr["ms_theta"]), _p(arr["ms_allreduce"]), _p(nnz), ctypes.byref(n)), ctx)
+    arr["sum_nnz_tok"] = nnz
+    return arr
+
+
+def lda_get_stream(ctx) -> int:
+    s = _vp()
+    _check(lib().lda_get_stream(ctx, ctypes.byref(s)), ctx)
+    return int(s.value or 0)
+
+
+def lda_set_z(ctx, z):
+    z = np.ascontiguousarray(z, np.uint16)
+    _check(lib().lda_set_z(ctx, _p(z)), ctx)
+
+
+def lda_destroy(ctx):
+    if ctx:
+        lib().lda_destroy(ctx)
+
+
+def lda_last_error(ctx) -> str:
+    return lib().lda_last_error(ctx).decode()
+
+
+# ---------------------------------------------------------------------------
+# convenience object
+# ---------------------------------------------------------------------------
+
+class LDA:
+    """One rank's sampler: create -> [options] -> [dist] -> load -> iterate."""
+
+    def __init__(self, D, V, K, alpha=None, beta=0.01, **options):
+        self.D, self.V, self.K = int(D), int(V), int(K)
+        self.alpha = 50.0 / K if alpha is None else float(alpha)
+        self.beta = float(beta)
+        self.ctx = lda_create(self.D, self.V, self.K, self.alpha, self.beta)
+        for k, v in options.items():
+            lda_set_option(self.ctx, k, v)
+        self.doc_begin, self.doc_end = 0, self.D
+        self.T = 0
+
+    def init_dist(self, rank, world, unique_id):
+        lda_init_dist(self.ctx, rank, world, unique_id)
+
+    def load(self, doc_ptr, words, seed, doc_begin=0, doc_end=None):
+        self.doc_begin = int(doc_begin)
+        self.doc_end = self.D if doc_end is None else int(doc_end)
+        self.doc_ptr = np.ascontiguousarray(doc_ptr, np.int64)
+        self.T = int(self.doc_ptr[-1])
+        lda_load_corpus(self.ctx, self.doc_begin, self.doc_end, self.doc_ptr, words, seed)
+        return self
+
+    def iterate(self, n=1):
+        lda_iterate(self.ctx, n)
+
+    def loglik(self):
+        return lda_loglik(self.ctx)
+
+    def z(self):
+        z = np.empty(self.T, np.uint16)
+        lda_get_counts(self.ctx, z=z)
+        return z
+
+    def set_z(self, z):
+        lda_set_z(self.ctx, z)
+
+    def nwk(self):
+        a = np.empty(self.V * self.K, np.int32)
+        lda_get_counts(self.ctx, n_wk=a)
+        return a.reshape(self.V, self.K)
+
+    def nk(self):
+        a = np.empty(self.K, np.int32)
+        lda_get_counts(self.ctx, n_k=a)
+        return a
+
+    def theta_csr(self):
+        nnz = lda_get_counts(self.ctx)
+        Dg = self.doc_end - self.doc_begin
+        ptr = np.empty(Dg + 1, np.int64)
+        top = np.empty(nnz, np.uint16)
+        cnt = np.empty(nnz, np.int32)
+        lda_get_counts(self.ctx, ndk_ptr=ptr, ndk_topic=top, ndk_count=cnt)
+        return ptr, top, cnt
+
+    def ndk_dense(self):
+        ptr, top, cnt = self.theta_csr()
+        Dg = len(ptr) - 1
+        out = np.zeros((Dg, self.K), np.int32)
+        rows = np.repeat(np.arange(Dg), np.diff(ptr))
+        out[rows, top.astype(np.int64)] = cnt
+        return out
+
+    def stats(self):
+        return lda_get_stats(self.ctx)
+
+    def sweep_log(self):
+        return lda_get_sweep_log(self.ctx)
+
+    def stream(self):
+        return lda_get_stream(self.ctx)
+
+    def close(self):
+        if self.ctx:
+            lda_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()

@@ -1,0 +1,620 @@
+// C ABI (include/lda.h): context life cycle, corpus loading, the per-sweep
+// orchestration of Alg. 1 WorkSchedule1 (M = 1, L807-835) on one GPU per
+// process, and the n_wk/n_k sum-allreduce of Eq. 4 (L935-937) over NCCL.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <cmath>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/lda.h"
+#include "lda_internal.h"
+
+struct lda_ctx {
+    int64_t D = 0;
+    int32_t V = 0, K = 0;
+    double alpha = 0, beta = 0;
+    // options
+    int device = 0;
+    int exclude_self = 0;
+    int64_t chunk_tokens = 4096;
+    int64_t recount_tokens = 65536;
+    int64_t tile_tokens = 0;
+    int threads = 0;
+    // distribution
+    int32_t rank = 0, world = 1;
+    ncclComm_t comm = nullptr;
+    // state
+    bool loaded = false;
+    int failed = 0;
+    std::string err;
+    uint64_t sweeps = 0;
+    int64_t T_global = 0;
+    lda::HostLayout H;
+    lda::DevState S;
+    cudaStream_t stream = nullptr, comm_stream = nullptr;
+    std::vector<cudaEvent_t> ev;  // 6 per sweep
+    lda_stats stats{};
+    std::vector<void *> allocs;
+    // θ statistics: Σ_d L_d·nnz_d (= Σ_t nnz_{d(t)}) and Σ_d nnz_d of the
+    // current θ, and a per-sweep log of the last lda_iterate call.
+    int64_t cur_lnnz = 0, cur_nnz = 0;
+    unsigned long long *d_stat_log = nullptr;
+    size_t stat_log_cap = 0;
+    std::vector<double> log_ms, log_ms_sample, log_ms_recount, log_ms_theta, log_ms_comm;
+    std::vector<int64_t> log_nnz_tok;
+};
+
+namespace {
+
+// NCCL is opened at run time (only multi-GPU contexts need it), so that
+// loading liblda.so never pins an NCCL build into the process before torch
+// loads its own.  dlopen("libnccl.so.2") returns the copy already loaded by
+// torch when there is one; LDA_NCCL_LIBRARY overrides the path.
+struct NcclApi {
+    ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                              cudaStream_t) = nullptr;
+    ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+    const char *(*GetErrorString)(ncclResult_t) = nullptr;
+    std::string err;
+    bool ok = false;
+};
+
+NcclApi load_nccl() {
+    NcclApi a;
+    const char *env = std::getenv("LDA_NCCL_LIBRARY");
+    const char *cands[] = {env, "libnccl.so.2", "libnccl.so"};
+    void *h = nullptr;
+    for (const char *c : cands) {
+        if (!c) continue;
+        h = dlopen(c, RTLD_NOW | RTLD_GLOBAL);
+        if (h) break;
+    }
+    if (!h) {
+        a.err = std::string("cannot dlopen NCCL: ") + dlerror();
+        return a;
+    }
+#define LDA_SYM(field, name)                                              \
+    a.field = reinterpret_cast<decltype(a.field)>(dlsym(h, name));        \
+    if (!a.field) {                                                       \
+        a.err = std::string("NCCL symbol missing: ") + name;              \
+        return a;                                                         \
+    }
+    LDA_SYM(GetUniqueId, "ncclGetUniqueId")
+    LDA_SYM(CommInitRank, "ncclCommInitRank")
+    LDA_SYM(AllReduce, "ncclAllReduce")
+    LDA_SYM(AllGather, "ncclAllGather")
+    LDA_SYM(CommDestroy, "ncclCommDestroy")
+    LDA_SYM(GetErrorString, "ncclGetErrorString")
+#undef LDA_SYM
+    a.ok = true;
+    return a;
+}
+
+const NcclApi &nccl() {
+    static NcclApi api = load_nccl();
+    return api;
+}
+
+int fail(lda_ctx *c, int code, const std::string &msg) {
+    if (c) {
+        c->err = msg;
+        if (code == LDA_ECUDA || code == LDA_ENCCL) c->failed = code;
+    }
+    return code;
+}
+
+#define CU(call)                                                                             \
+    do {                                                                                     \
+        cudaError_t e_ = (call);                                                             \
+        if (e_ != cudaSuccess)                                                               \
+            return fail(ctx, LDA_ECUDA, std::string(#call) + ": " + cudaGetErrorString(e_)); \
+    } while (0)
+
+#define KL(call)                                                                                   \
+    do {                                                                                           \
+        int e_ = (call);                                                                           \
+        if (e_ != 0)                                                                               \
+            return fail(ctx, LDA_ECUDA,                                                            \
+                        std::string(#call) + ": " + cudaGetErrorString(static_cast<cudaError_t>(e_))); \
+    } while (0)
+
+#define NC(call)                                                                                  \
+    do {                                                                                          \
+        if (!nccl().ok) return fail(ctx, LDA_ENCCL, nccl().err);                                  \
+        ncclResult_t r_ = nccl().call;                                                            \
+        if (r_ != ncclSuccess)                                                                    \
+            return fail(ctx, LDA_ENCCL, std::string(#call) + ": " + nccl().GetErrorString(r_));   \
+    } while (0)
+
+#define PRECHECK(ctx)                                   \
+    do {                                                \
+        if (!(ctx)) return LDA_EINVAL;                  \
+        if ((ctx)->failed) return (ctx)->failed;        \
+    } while (0)
+
+template <class T>
+int dalloc(lda_ctx *ctx, T **p, size_t n) {
+    void *q = nullptr;
+    cudaError_t e = cudaMalloc(&q, std::max<size_t>(n, 1) * sizeof(T));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ctx, e == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
+                    std::string("cudaMalloc(") + std::to_string(n * sizeof(T)) + " B): " + cudaGetErrorString(e));
+    }
+    ctx->allocs.push_back(q);
+    *p = static_cast<T *>(q);
+    return LDA_OK;
+}
+
+#define DA(ptr, n)                               \
+    do {                                         \
+        int r_ = dalloc(ctx, &(ptr), (n));       \
+        if (r_ != LDA_OK) return r_;             \
+    } while (0)
+
+int ensure_events(lda_ctx *ctx, size_t n) {
+    while (ctx->ev.size() < n) {
+        cudaEvent_t e;
+        CU(cudaEventCreate(&e));
+        ctx->ev.push_back(e);
+    }
+    return LDA_OK;
+}
+
+// Rebuild n_wk, n_k (and allreduce them) and θ from tok_z.
+int rebuild_counts(lda_ctx *ctx, int *launches) {
+    lda::DevState &S = ctx->S;
+    KL(lda::launch_recount(S, ctx->stream, launches));
+    if (ctx->world > 1) {
+        NC(AllReduce(S.nwk, S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ncclInt32, ncclSum, ctx->comm,
+                         ctx->stream));
+    }
+    KL(lda::launch_theta(S, S.stat, ctx->stream, launches));
+    unsigned long long hs[2] = {0, 0};
+    CU(cudaMemcpyAsync(hs, S.stat, sizeof(hs), cudaMemcpyDeviceToHost, ctx->stream));
+    CU(cudaStreamSynchronize(ctx->stream));
+    ctx->cur_lnnz = static_cast<int64_t>(hs[0]);
+    ctx->cur_nnz = static_cast<int64_t>(hs[1]);
+    return LDA_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *lda_version(void) { return "lda-b200 0.1 (sm_100a)"; }
+
+const char *lda_last_error(const lda_ctx *ctx) {
+    if (!ctx) return "null context";
+    return ctx->err.c_str();
+}
+
+int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_ctx **out) {
+    if (!out) return LDA_EINVAL;
+    *out = nullptr;
+    if (D < 1 || V < 1 || K < 1 || K > 65536) return LDA_EINVAL;
+    if (!std::isfinite(alpha) || !std::isfinite(beta) || !(alpha > 0) || !(beta > 0)) return LDA_EINVAL;
+    lda_ctx *c = new (std::nothrow) lda_ctx();
+    if (!c) return LDA_ENOMEM;
+    c->D = D;
+    c->V = V;
+    c->K = K;
+    c->alpha = alpha;
+    c->beta = beta;
+    *out = c;
+    return LDA_OK;
+}
+
+int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
+    PRECHECK(ctx);
+    if (!key) return fail(ctx, LDA_EINVAL, "null option key");
+    if (ctx->loaded) return fail(ctx, LDA_ESTATE, "options must be set before lda_load_corpus");
+    std::string k(key);
+    if (k == "device") {
+        if (value < 0 || value > 1024) return fail(ctx, LDA_EINVAL, "bad device");
+        ctx->device = static_cast<int>(value);
+    } else if (k == "exclude_self") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "exclude_self must be 0 or 1");
+        ctx->exclude_self = static_cast<int>(value);
+    } else if (k == "chunk_tokens") {
+        if (value < 32 || value > (int64_t(1) << 30)) return fail(ctx, LDA_EINVAL, "chunk_tokens out of range");
+        ctx->chunk_tokens = value;
+    } else if (k == "recount_tokens") {
+        if (value < 256 || value > (int64_t(1) << 31)) return fail(ctx, LDA_EINVAL, "recount_tokens out of range");
+        ctx->recount_tokens = value;
+    } else if (k == "tile_tokens") {
+        if (value < 0) return fail(ctx, LDA_EINVAL, "tile_tokens must be >= 0");
+        ctx->tile_tokens = value;
+    } else if (k == "threads") {
+        if (value < 0 || value > 1024) return fail(ctx, LDA_EINVAL, "threads out of range");
+        ctx->threads = static_cast<int>(value);
+    } else {
+        return fail(ctx, LDA_EINVAL, "unknown option '" + k + "'");
+    }
+    return LDA_OK;
+}
+
+int lda_nccl_unique_id(void *out128) {
+    if (!out128) return LDA_EINVAL;
+    ncclUniqueId id;
+    if (!nccl().ok || nccl().GetUniqueId(&id) != ncclSuccess) return LDA_ENCCL;
+    std::memcpy(out128, &id, sizeof(id));
+    return LDA_OK;
+}
+
+int lda_init_dist(lda_ctx *ctx, int32_t rank, int32_t world, const void *uid) {
+    PRECHECK(ctx);
+    if (ctx->loaded || ctx->comm) return fail(ctx, LDA_ESTATE, "lda_init_dist must precede lda_load_corpus");
+    if (world < 1 || rank < 0 || rank >= world) return fail(ctx, LDA_EINVAL, "bad rank/world");
+    ctx->rank = rank;
+    ctx->world = world;
+    if (world == 1) return LDA_OK;
+    if (!uid) return fail(ctx, LDA_EINVAL, "null nccl unique id");
+    CU(cudaSetDevice(ctx->device));
+    ncclUniqueId id;
+    std::memcpy(&id, uid, sizeof(id));
+    NC(CommInitRank(&ctx->comm, world, id, rank));
+    return LDA_OK;
+}
+
+int lda_partition_docs(int64_t D, const int64_t *doc_ptr, int32_t world, int64_t *doc_begin) {
+    if (D < 0 || !doc_ptr || world < 1 || !doc_begin) return LDA_EINVAL;
+    if (doc_ptr[0] != 0) return LDA_EINVAL;
+    for (int64_t d = 0; d < D; ++d)
+        if (doc_ptr[d + 1] < doc_ptr[d]) return LDA_EINVAL;
+    const int64_t T = doc_ptr[D];
+    doc_begin[0] = 0;
+    for (int32_t g = 1; g < world; ++g) {
+        // first d with doc_ptr[d] >= ceil(g*T/world)   (X21)
+        const __int128 num = static_cast<__int128>(g) * T;
+        const int64_t target = static_cast<int64_t>((num + world - 1) / world);
+        const int64_t *it = std::lower_bound(doc_ptr, doc_ptr + D + 1, target);
+        int64_t d = it - doc_ptr;
+        doc_begin[g] = std::min(std::max(d, doc_begin[g - 1]), D);
+    }
+    doc_begin[world] = D;
+    return LDA_OK;
+}
+
+int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int64_t *doc_ptr,
+                    const int32_t *words, uint64_t seed) {
+    PRECHECK(ctx);
+    if (ctx->loaded) return fail(ctx, LDA_ESTATE, "corpus already loaded");
+    if (doc_begin < 0 || doc_end < doc_begin || doc_end > ctx->D)
+        return fail(ctx, LDA_EINVAL, "document range outside [0, D]");
+    if (ctx->world == 1 && (doc_begin != 0 || doc_end != ctx->D))
+        return fail(ctx, LDA_EINVAL, "with world == 1 the whole corpus [0, D) must be loaded");
+    const int64_t Dg = doc_end - doc_begin;
+    bool range_err = false;
+    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err);
+    if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
+    if (ctx->K > 16384)
+        return fail(ctx, LDA_ERANGE, "K > 16384 is not supported by this build's shared-memory layout");
+    const int64_t Tg = doc_ptr[Dg];
+    const int32_t V = ctx->V, K = ctx->K;
+
+    CU(cudaSetDevice(ctx->device));
+    CU(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking));
+
+    // Local word histogram -> canonical bases.  c for rank g's tokens of word
+    // w starts at Σ_{w'<w} T(w') + Σ_{g'<g} T_{g'}(w)   (X18, §8(c) step 2).
+    std::vector<int64_t> local(V, 0);
+    for (int64_t i = 0; i < Tg; ++i) local[words[i]]++;
+    std::vector<int64_t> all(static_cast<size_t>(V) * ctx->world, 0);
+    if (ctx->world > 1) {
+        int64_t *d_all = nullptr;
+        DA(d_all, all.size());
+        CU(cudaMemcpyAsync(d_all + static_cast<size_t>(ctx->rank) * V, local.data(), sizeof(int64_t) * V,
+                           cudaMemcpyHostToDevice, ctx->stream));
+        NC(AllGather(d_all + static_cast<size_t>(ctx->rank) * V, d_all, V, ncclInt64, ctx->comm,
+                         ctx->stream));
+        CU(cudaMemcpyAsync(all.data(), d_all, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost, ctx->stream));
+        CU(cudaStreamSynchronize(ctx->stream));
+    } else {
+        std::copy(local.begin(), local.end(), all.begin());
+    }
+    std::vector<int64_t> cbase(V);
+    int64_t run = 0;
+    for (int32_t w = 0; w < V; ++w) {
+        int64_t before_rank = 0, tot = 0;
+        for (int32_t g = 0; g < ctx->world; ++g) {
+            int64_t n = all[static_cast<size_t>(g) * V + w];
+            if (g < ctx->rank) before_rank += n;
+            tot += n;
+        }
+        cbase[w] = run + before_rank;
+        run += tot;
+    }
+    ctx->T_global = run;
+
+    lda::HostLayout &H = ctx->H;
+    std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
+                                      ctx->chunk_tokens, ctx->recount_tokens, ctx->threads, H);
+    if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
+
+    lda::DevState &S = ctx->S;
+    S.V = V;
+    S.K = K;
+    S.D = Dg;
+    S.T = Tg;
+    S.ntiles = H.ntiles;
+    S.alpha = ctx->alpha;
+    S.beta = ctx->beta;
+    S.seed = seed;
+    S.exclude_self = ctx->exclude_self;
+    KL(lda::configure_kernels(S));
+
+    DA(S.tok_row, Tg);
+    DA(S.tok_z, Tg);
+    DA(S.doc_map, Tg);
+    DA(S.doc_ptr32, Dg + 1);
+    DA(S.row_off16, std::max<int64_t>(Dg, 1));
+    DA(S.tseg, H.tseg.size());
+    S.n_chunks = static_cast<int64_t>(H.chunks.size());
+    DA(S.chunks, H.chunks.size());
+    S.n_rchunks = static_cast<int64_t>(H.rchunks.size());
+    DA(S.rchunks, H.rchunks.size());
+    S.n_split = static_cast<int64_t>(H.split_words.size());
+    DA(S.split_words, H.split_words.size());
+    DA(S.rows, H.rows16 * 4);
+    DA(S.nwk, static_cast<size_t>(V) * K + K);
+    DA(S.invk, K);
+    DA(S.counter, 4);
+    DA(S.stat, 4);
+    DA(S.ll_part, 2 * S.ll_blocks + 2);
+    DA(S.ll_out, 2);
+    if (S.sweep_smem == 0) DA(S.sweep_scratch, static_cast<size_t>(S.sweep_grid) * 2 * K);
+
+    auto h2d = [&](void *dst, const void *src, size_t bytes) {
+        return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream) : cudaSuccess;
+    };
+    CU(h2d(S.tok_row, H.tok_row.data(), sizeof(uint32_t) * Tg));
+    CU(h2d(S.doc_map, H.doc_map.data(), sizeof(uint32_t) * Tg));
+    CU(h2d(S.doc_ptr32, H.doc_ptr32.data(), sizeof(uint32_t) * (Dg + 1)));
+    CU(h2d(S.row_off16, H.row_off16.data(), sizeof(uint32_t) * Dg));
+    CU(h2d(S.tseg, H.tseg.data(), sizeof(uint32_t) * H.tseg.size()));
+    CU(h2d(S.chunks, H.chunks.data(), sizeof(lda::SampleChunk) * H.chunks.size()));
+    CU(h2d(S.rchunks, H.rchunks.data(), sizeof(lda::RecountChunk) * H.rchunks.size()));
+    CU(h2d(S.split_words, H.split_words.data(), sizeof(int32_t) * H.split_words.size()));
+    CU(cudaMemsetAsync(S.rows, 0, H.rows16 * 16, ctx->stream));
+    CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
+
+    // a1: random init (t = 0), then the count rebuild.
+    KL(lda::launch_init(S, ctx->stream));
+    int launches = 1;
+    int r = rebuild_counts(ctx, &launches);
+    if (r != LDA_OK) return r;
+    CU(cudaStreamSynchronize(ctx->stream));
+    // host copies no longer needed on the device side (doc_map kept for get_counts)
+    std::vector<uint32_t>().swap(H.tok_row);
+    ctx->loaded = true;
+    ctx->sweeps = 0;
+    ctx->stats.local_tokens = Tg;
+    ctx->stats.local_docs = Dg;
+    ctx->stats.global_tokens = ctx->T_global;
+    ctx->stats.world = ctx->world;
+    ctx->stats.n_sample_chunks = S.n_chunks;
+    ctx->stats.sum_nnz_doc = ctx->cur_nnz;
+    return LDA_OK;
+}
+
+int lda_iterate(lda_ctx *ctx, int32_t n) {
+    PRECHECK(ctx);
+    if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
+    if (n < 0) return fail(ctx, LDA_EINVAL, "negative sweep count");
+    CU(cudaSetDevice(ctx->device));
+    lda::DevState &S = ctx->S;
+    const int per = 6;
+    int r = ensure_events(ctx, static_cast<size_t>(per) * std::max(n, 1));
+    if (r != LDA_OK) return r;
+    if (ctx->stat_log_cap < static_cast<size_t>(n)) {
+        if (ctx->d_stat_log) {
+            CU(cudaFree(ctx->d_stat_log));
+            ctx->allocs.erase(std::find(ctx->allocs.begin(), ctx->allocs.end(),
+                                        static_cast<void *>(ctx->d_stat_log)));
+            ctx->d_stat_log = nullptr;
+        }
+        DA(ctx->d_stat_log, 2 * static_cast<size_t>(n));
+        ctx->stat_log_cap = n;
+    }
+    int launches = 0;
+    for (int32_t s = 0; s < n; ++s) {
+        cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
+        const uint32_t t = static_cast<uint32_t>(++ctx->sweeps);
+        CU(cudaEventRecord(E[0], ctx->stream));
+        KL(lda::launch_sweep(S, t, ctx->stream, &launches));
+        CU(cudaEventRecord(E[1], ctx->stream));
+        KL(lda::launch_recount(S, ctx->stream, &launches));
+        CU(cudaEventRecord(E[2], ctx->stream));
+        if (ctx->world > 1) {
+            // ϕ sync overlapped with the θ update (§6.2)
+            CU(cudaStreamWaitEvent(ctx->comm_stream, E[2], 0));
+            NC(AllReduce(S.nwk, S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ncclInt32, ncclSum,
+                             ctx->comm, ctx->comm_stream));
+            CU(cudaEventRecord(E[4], ctx->comm_stream));
+        }
+        KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches));
+        CU(cudaEventRecord(E[3], ctx->stream));
+        if (ctx->world > 1) CU(cudaStreamWaitEvent(ctx->stream, E[4], 0));
+        CU(cudaEventRecord(E[5], ctx->stream));
+    }
+    CU(cudaStreamSynchronize(ctx->stream));
+    std::vector<unsigned long long> hs(2 * static_cast<size_t>(n));
+    if (n)
+        CU(cudaMemcpy(hs.data(), ctx->d_stat_log, hs.size() * sizeof(unsigned long long),
+                      cudaMemcpyDeviceToHost));
+    lda_stats &st = ctx->stats;
+    st.last_n = n;
+    st.sweeps_done = static_cast<int64_t>(ctx->sweeps);
+    st.ms_total = st.ms_sample = st.ms_recount = st.ms_theta = st.ms_allreduce = 0;
+    st.ms_last_sweep = st.ms_last_sample = 0;
+    ctx->log_ms.assign(n, 0);
+    ctx->log_ms_sample.assign(n, 0);
+    ctx->log_ms_recount.assign(n, 0);
+    ctx->log_ms_theta.assign(n, 0);
+    ctx->log_ms_comm.assign(n, 0);
+    ctx->log_nnz_tok.assign(n, 0);
+    for (int32_t s = 0; s < n; ++s) {
+        cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
+        float a = 0, b = 0, c = 0, d = 0, tot = 0;
+        CU(cudaEventElapsedTime(&a, E[0], E[1]));
+        CU(cudaEventElapsedTime(&b, E[1], E[2]));
+        CU(cudaEventElapsedTime(&c, E[2], E[3]));
+        CU(cudaEventElapsedTime(&tot, E[0], E[5]));
+        if (ctx->world > 1) CU(cudaEventElapsedTime(&d, E[2], E[4]));
+        st.ms_sample += a;
+        st.ms_recount += b;
+        st.ms_theta += c;
+        st.ms_allreduce += d;
+        st.ms_total += tot;
+        ctx->log_ms[s] = tot;
+        ctx->log_ms_sample[s] = a;
+        ctx->log_ms_recount[s] = b;
+        ctx->log_ms_theta[s] = c;
+        ctx->log_ms_comm[s] = d;
+        // sweep s sampled against the θ built before it
+        ctx->log_nnz_tok[s] = ctx->cur_lnnz;
+        ctx->cur_lnnz = static_cast<int64_t>(hs[2 * s]);
+        ctx->cur_nnz = static_cast<int64_t>(hs[2 * s + 1]);
+        if (s == n - 1) {
+            st.ms_last_sweep = tot;
+            st.ms_last_sample = a;
+            st.sum_nnz_tok = ctx->log_nnz_tok[s];
+        }
+    }
+    st.sum_nnz_doc = ctx->cur_nnz;
+    st.n_launches = launches;
+    return LDA_OK;
+}
+
+int lda_get_sweep_log(lda_ctx *ctx, int32_t cap, double *ms_sweep, double *ms_sample, double *ms_recount,
+                      double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int32_t *n_out) {
+    PRECHECK(ctx);
+    const int32_t n = static_cast<int32_t>(ctx->log_ms.size());
+    if (n_out) *n_out = n;
+    const int32_t m = std::min(n, std::max(cap, 0));
+    for (int32_t s = 0; s < m; ++s) {
+        if (ms_sweep) ms_sweep[s] = ctx->log_ms[s];
+        if (ms_sample) ms_sample[s] = ctx->log_ms_sample[s];
+        if (ms_recount) ms_recount[s] = ctx->log_ms_recount[s];
+        if (ms_theta) ms_theta[s] = ctx->log_ms_theta[s];
+        if (ms_allreduce) ms_allreduce[s] = ctx->log_ms_comm[s];
+        if (sum_nnz_tok) sum_nnz_tok[s] = ctx->log_nnz_tok[s];
+    }
+    return LDA_OK;
+}
+
+int lda_loglik(lda_ctx *ctx, double *ll) {
+    PRECHECK(ctx);
+    if (!ll) return fail(ctx, LDA_EINVAL, "null output");
+    if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
+    CU(cudaSetDevice(ctx->device));
+    int launches = 0;
+    KL(lda::launch_loglik(ctx->S, ctx->rank == 0, ctx->stream, &launches));
+    if (ctx->world > 1)
+        NC(AllReduce(ctx->S.ll_out, ctx->S.ll_out, 2, ncclFloat64, ncclSum, ctx->comm, ctx->stream));
+    double h[2];
+    CU(cudaMemcpyAsync(h, ctx->S.ll_out, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
+    CU(cudaStreamSynchronize(ctx->stream));
+    *ll = (h[0] + h[1]) / static_cast<double>(ctx->T_global > 0 ? ctx->T_global : 1);
+    return LDA_OK;
+}
+
+int lda_get_counts(lda_ctx *ctx, int32_t *n_wk, int32_t *n_k, int64_t *ndk_ptr, uint16_t *ndk_topic,
+                   int32_t *ndk_count, int64_t ndk_capacity, int64_t *ndk_nnz_out, uint16_t *z) {
+    PRECHECK(ctx);
+    if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
+    CU(cudaSetDevice(ctx->device));
+    CU(cudaStreamSynchronize(ctx->stream));
+    const lda::DevState &S = ctx->S;
+    const lda::HostLayout &H = ctx->H;
+    if (n_wk) CU(cudaMemcpy(n_wk, S.nwk, sizeof(int32_t) * S.V * S.K, cudaMemcpyDeviceToHost));
+    if (n_k) CU(cudaMemcpy(n_k, S.nwk + static_cast<size_t>(S.V) * S.K, sizeof(int32_t) * S.K,
+                           cudaMemcpyDeviceToHost));
+    if (ndk_ptr || ndk_topic || ndk_count || ndk_nnz_out) {
+        std::vector<uint32_t> rows(H.rows16 * 4);
+        CU(cudaMemcpy(rows.data(), S.rows, rows.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+        int64_t nnz = 0;
+        for (int64_t d = 0; d < S.D; ++d) nnz += rows[static_cast<size_t>(H.row_off16[d]) * 4];
+        if (ndk_nnz_out) *ndk_nnz_out = nnz;
+        if ((ndk_topic || ndk_count) && ndk_capacity < nnz)
+            return fail(ctx, LDA_ERANGE, "ndk_capacity smaller than nnz");
+        int64_t pos = 0;
+        for (int64_t d = 0; d < S.D; ++d) {
+            const uint32_t *row = rows.data() + static_cast<size_t>(H.row_off16[d]) * 4;
+            if (ndk_ptr) ndk_ptr[d] = pos;
+            for (uint32_t j = 0; j < row[0]; ++j, ++pos) {
+                if (ndk_topic) ndk_topic[pos] = static_cast<uint16_t>(row[1 + j] >> 16);
+                if (ndk_count) ndk_count[pos] = static_cast<int32_t>(row[1 + j] & 0xFFFFu);
+            }
+        }
+        if (ndk_ptr) ndk_ptr[S.D] = pos;
+    }
+    if (z) {
+        std::vector<uint16_t> zw(S.T);
+        if (S.T) CU(cudaMemcpy(zw.data(), S.tok_z, sizeof(uint16_t) * S.T, cudaMemcpyDeviceToHost));
+        for (int64_t i = 0; i < S.T; ++i) z[i] = zw[H.doc_map[i]];
+    }
+    return LDA_OK;
+}
+
+int lda_set_z(lda_ctx *ctx, const uint16_t *z) {
+    PRECHECK(ctx);
+    if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
+    const lda::DevState &S = ctx->S;
+    if (!z && S.T) return fail(ctx, LDA_EINVAL, "null z");
+    std::vector<uint16_t> zw(S.T);
+    for (int64_t i = 0; i < S.T; ++i) {
+        if (z[i] >= S.K) return fail(ctx, LDA_EINVAL, "topic id >= K");
+        zw[ctx->H.doc_map[i]] = z[i];
+    }
+    CU(cudaSetDevice(ctx->device));
+    if (S.T) CU(cudaMemcpy(S.tok_z, zw.data(), sizeof(uint16_t) * S.T, cudaMemcpyHostToDevice));
+    int launches = 0;
+    int r = rebuild_counts(ctx, &launches);
+    if (r != LDA_OK) return r;
+    CU(cudaStreamSynchronize(ctx->stream));
+    return LDA_OK;
+}
+
+int lda_get_stats(lda_ctx *ctx, lda_stats *out) {
+    PRECHECK(ctx);
+    if (!out) return fail(ctx, LDA_EINVAL, "null output");
+    *out = ctx->stats;
+    return LDA_OK;
+}
+
+int lda_get_stream(lda_ctx *ctx, void **stream) {
+    PRECHECK(ctx);
+    if (!stream) return fail(ctx, LDA_EINVAL, "null output");
+    if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
+    *stream = ctx->stream;
+    return LDA_OK;
+}
+
+void lda_destroy(lda_ctx *ctx) {
+    if (!ctx) return;
+    if (ctx->stream || !ctx->allocs.empty()) {
+        cudaSetDevice(ctx->device);
+        if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+        for (void *p : ctx->allocs) cudaFree(p);
+        for (cudaEvent_t e : ctx->ev) cudaEventDestroy(e);
+        if (ctx->stream) cudaStreamDestroy(ctx->stream);
+        if (ctx->comm_stream) cudaStreamDestroy(ctx->comm_stream);
+    }
+    if (ctx->comm && nccl().ok) nccl().CommDestroy(ctx->comm);
+    delete ctx;
+}
+
+}  // extern "C"

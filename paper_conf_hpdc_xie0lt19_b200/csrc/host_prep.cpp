@@ -1,0 +1,229 @@
+// Host-side corpus preparation (the paper's CPU preprocessing, L593-597):
+// validation, the word-first token order (L1189-1191), the document-word map
+// (L1297-1303), fixed-capacity θ rows (CSR with short column index,
+// L1235-1243) and the heavy-first work-item tables (L1203-1221).
+#include <algorithm>
+#include <cstring>
+#include <thread>
+
+#include "lda_internal.h"
+
+namespace lda {
+
+int host_threads(int requested) {
+    unsigned hw = std::thread::hardware_concurrency();
+    if (hw == 0) hw = 1;
+    int n = requested > 0 ? requested : static_cast<int>(hw);
+    return std::max(1, std::min(n, 64));
+}
+
+// f(thread_id, begin, end) over [0, n) split into nthreads contiguous parts.
+template <class F>
+static void parallel_for(int nthreads, int64_t n, F f) {
+    if (nthreads <= 1 || n < (1 << 16)) {
+        f(0, int64_t(0), n);
+        return;
+    }
+    std::vector<std::thread> th;
+    th.reserve(nthreads);
+    for (int t = 0; t < nthreads; ++t) {
+        int64_t b = n * t / nthreads, e = n * (t + 1) / nthreads;
+        th.emplace_back([=, &f] { f(t, b, e); });
+    }
+    for (auto &x : th) x.join();
+}
+
+std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
+                            bool *range_error) {
+    *range_error = false;
+    if (D < 0) return "negative document count";
+    if (!doc_ptr) return "doc_ptr is NULL";
+    if (doc_ptr[0] != 0) return "doc_ptr[0] must be 0";
+    for (int64_t d = 0; d < D; ++d) {
+        int64_t len = doc_ptr[d + 1] - doc_ptr[d];
+        if (len < 0) return "doc_ptr must be non-decreasing";
+        if (len > 65535) {
+            *range_error = true;
+            return "document " + std::to_string(d) + " has " + std::to_string(len) +
+                   " tokens (> 65535, the uint16 θ count limit)";
+        }
+    }
+    int64_t T = doc_ptr[D];
+    if (T >= (int64_t(1) << 32)) {
+        *range_error = true;
+        return "more than 2^32-1 tokens on one rank";
+    }
+    if (T > 0 && !words) return "words is NULL";
+    int nth = host_threads(0);
+    std::vector<int64_t> bad(nth, -1);
+    parallel_for(nth, T, [&](int t, int64_t b, int64_t e) {
+        for (int64_t i = b; i < e; ++i)
+            if (words[i] < 0 || words[i] >= V) {
+                bad[t] = i;
+                return;
+            }
+    });
+    for (int64_t i : bad)
+        if (i >= 0)
+            return "word id " + std::to_string(words[i]) + " at token " + std::to_string(i) +
+                   " outside [0, V)";
+    return "";
+}
+
+std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
+                         int32_t K, const int64_t *cbase, int64_t tile_tokens,
+                         int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
+                         HostLayout &L) {
+    const int64_t T = doc_ptr[D];
+    L.D = D;
+    L.T = T;
+    L.V = V;
+    L.K = K;
+    nthreads = host_threads(nthreads);
+
+    // θ rows: capacity min(L_d, K) entries + 1 header word, 16-byte aligned.
+    L.doc_ptr32.resize(D + 1);
+    L.row_off16.resize(D);
+    uint64_t off16 = 0;
+    for (int64_t d = 0; d < D; ++d) {
+        int64_t len = doc_ptr[d + 1] - doc_ptr[d];
+        int64_t cap = std::min<int64_t>(len, K);
+        L.doc_ptr32[d] = static_cast<uint32_t>(doc_ptr[d]);
+        L.row_off16[d] = static_cast<uint32_t>(off16);
+        off16 += static_cast<uint64_t>((cap + 1 + 3) / 4);
+        if (off16 >= (uint64_t(1) << 32) - 64) return "θ row storage exceeds 2^32 x 16 bytes";
+    }
+    L.doc_ptr32[D] = static_cast<uint32_t>(T);
+    L.rows16 = off16 + 64;  // tail pad: the sampler may read up to 32 x 16 B past a row
+
+    // Doc tiles: contiguous document ranges of about tile_tokens tokens.
+    std::vector<int64_t> tile_doc{0};
+    if (tile_tokens > 0) {
+        int64_t acc = 0;
+        for (int64_t d = 0; d < D; ++d) {
+            int64_t len = doc_ptr[d + 1] - doc_ptr[d];
+            if (acc > 0 && acc + len > tile_tokens) {
+                tile_doc.push_back(d);
+                acc = 0;
+            }
+            acc += len;
+        }
+    }
+    tile_doc.push_back(D);
+    const int nt = static_cast<int>(tile_doc.size()) - 1;
+    L.ntiles = nt;
+
+    L.tok_row.assign(T, 0);
+    L.doc_map.assign(T, 0);
+    L.tseg.assign(static_cast<size_t>(nt) * V + 1, 0);
+    L.word_count.assign(V, 0);
+    std::vector<std::vector<uint32_t>> tile_cnt(nt);
+
+    std::vector<std::vector<uint32_t>> hist(nthreads, std::vector<uint32_t>(V));
+    for (int b = 0; b < nt; ++b) {
+        const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
+        const int64_t nd = d1 - d0;
+        const int64_t t0 = doc_ptr[d0];
+        // split the tile's docs across threads (contiguous, by doc count)
+        int nth = (doc_ptr[d1] - t0) < (1 << 16) ? 1 : nthreads;
+        std::vector<int64_t> tdoc(nth + 1);
+        for (int t = 0; t <= nth; ++t) tdoc[t] = d0 + nd * t / nth;
+        auto count_part = [&](int t) {
+            auto &h = hist[t];
+            std::fill(h.begin(), h.end(), 0u);
+            for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) h[words[i]]++;
+        };
+        {
+            std::vector<std::thread> th;
+            for (int t = 1; t < nth; ++t) th.emplace_back(count_part, t);
+            count_part(0);
+            for (auto &x : th) x.join();
+        }
+        // segment starts and per-thread scatter bases
+        auto &cnt = tile_cnt[b];
+        cnt.assign(V, 0);
+        uint64_t pos = static_cast<uint64_t>(t0);
+        for (int32_t w = 0; w < V; ++w) {
+            L.tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
+            uint64_t run = pos;
+            for (int t = 0; t < nth; ++t) {
+                uint32_t h = hist[t][w];
+                hist[t][w] = static_cast<uint32_t>(run);  // becomes the thread's next position
+                run += h;
+            }
+            cnt[w] = static_cast<uint32_t>(run - pos);
+            L.word_count[w] += cnt[w];
+            pos = run;
+        }
+        auto scatter_part = [&](int t) {
+            auto &next = hist[t];
+            for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
+                uint32_t row = L.row_off16[d];
+                for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
+                    uint32_t p = next[words[i]]++;
+                    L.doc_map[i] = p;
+                    L.tok_row[p] = row;
+                }
+            }
+        };
+        {
+            std::vector<std::thread> th;
+            for (int t = 1; t < nth; ++t) th.emplace_back(scatter_part, t);
+            scatter_part(0);
+            for (auto &x : th) x.join();
+        }
+    }
+    L.tseg[static_cast<size_t>(nt) * V] = static_cast<uint32_t>(T);
+
+    // Sampling work items: per (tile, word) segment, split into near-equal
+    // pieces of <= chunk_tokens; c_base continues word w's canonical run
+    // across tiles (tiles are increasing doc ranges, so (tile, d, j) order
+    // restricted to word w is its (d, j) order).
+    L.chunks.clear();
+    std::vector<int64_t> woff(V, 0);
+    for (int b = 0; b < nt; ++b) {
+        for (int32_t w = 0; w < V; ++w) {
+            int64_t n = tile_cnt[b][w];
+            if (n == 0) continue;
+            int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
+            uint32_t seg = L.tseg[static_cast<size_t>(b) * V + w];
+            int64_t done = 0;
+            for (int64_t p = 0; p < pieces; ++p) {
+                int64_t sz = n * (p + 1) / pieces - n * p / pieces;
+                SampleChunk c;
+                c.begin = static_cast<uint32_t>(seg + done);
+                c.count = static_cast<uint32_t>(sz);
+                c.word = static_cast<uint32_t>(w);
+                c.pad = 0;
+                c.c_base = static_cast<uint64_t>(cbase[w] + woff[w] + done);
+                L.chunks.push_back(c);
+                done += sz;
+            }
+            woff[w] += n;
+        }
+    }
+    std::stable_sort(L.chunks.begin(), L.chunks.end(),
+                     [](const SampleChunk &a, const SampleChunk &b) { return a.count > b.count; });
+
+    // Recount work items: per word over its tile segments.
+    L.rchunks.clear();
+    L.split_words.clear();
+    for (int32_t w = 0; w < V; ++w) {
+        int64_t n = L.word_count[w];
+        int64_t pieces = std::max<int64_t>(1, (n + recount_tokens - 1) / recount_tokens);
+        if (pieces > 1) L.split_words.push_back(w);
+        for (int64_t p = 0; p < pieces; ++p) {
+            RecountChunk c;
+            c.word = static_cast<uint32_t>(w);
+            c.vbegin = static_cast<uint32_t>(n * p / pieces);
+            c.vcount = static_cast<uint32_t>(n * (p + 1) / pieces - n * p / pieces);
+            c.split = pieces > 1 ? 1u : 0u;
+            L.rchunks.push_back(c);
+        }
+    }
+    std::stable_sort(L.rchunks.begin(), L.rchunks.end(),
+                     [](const RecountChunk &a, const RecountChunk &b) { return a.vcount > b.vcount; });
+    return "";
+}
+
+}  // namespace lda

@@ -1,0 +1,123 @@
+"""The C-ABI library on a CPU-only host (-m "not gpu"): it loads, exports every
+symbol include/lda.h declares, validates its arguments before touching the
+device, partitions documents by tokens (X21), and fails loudly (LDA_ECUDA)
+rather than falling back when there is no GPU."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_hpdc_xie0lt19_b200 as L
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _header_symbols():
+    src = open(os.path.join(ROOT, "include", "lda.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return set(re.findall(r"\b(lda_[a-z_]+)\s*\(", src))
+
+
+def test_library_exports_every_declared_symbol():
+    lib = L.lib()
+    declared = _header_symbols()
+    assert declared == set(L.ABI_SYMBOLS)
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert "sm_100a" in L.lda_version()
+
+
+def test_create_validation():
+    ok = L.lda_create(10, 5, 16, 0.1, 0.01)
+    L.lda_destroy(ok)
+    for args in [(0, 5, 16, 0.1, 0.01), (10, 0, 16, 0.1, 0.01), (10, 5, 0, 0.1, 0.01),
+                 (10, 5, 65537, 0.1, 0.01), (10, 5, 16, 0.0, 0.01), (10, 5, 16, 0.1, -1.0),
+                 (10, 5, 16, float("nan"), 0.01), (10, 5, 16, 0.1, float("inf"))]:
+        with pytest.raises(L.LDAError) as e:
+            L.lda_create(*args)
+        assert e.value.code == L.LDA_EINVAL
+    L.lda_destroy(L.lda_create(1, 1, 65536, 1.0, 1.0))
+
+
+def test_options_validation():
+    ctx = L.lda_create(10, 5, 16, 0.1, 0.01)
+    try:
+        L.lda_set_option(ctx, "exclude_self", 1)
+        L.lda_set_option(ctx, "chunk_tokens", 64)
+        L.lda_set_option(ctx, "tile_tokens", 0)
+        for key, val in [("exclude_self", 2), ("chunk_tokens", 1), ("nonsense", 1), ("device", -1)]:
+            with pytest.raises(L.LDAError) as e:
+                L.lda_set_option(ctx, key, val)
+            assert e.value.code == L.LDA_EINVAL
+        # calls that need a corpus
+        for f in (lambda: L.lda_iterate(ctx, 1), lambda: L.lda_loglik(ctx),
+                  lambda: L.lda_get_stream(ctx)):
+            with pytest.raises(L.LDAError) as e:
+                f()
+            assert e.value.code == L.LDA_ESTATE
+    finally:
+        L.lda_destroy(ctx)
+
+
+def test_partition_docs_token_balanced():
+    rng = np.random.default_rng(1)
+    for D, world in [(1, 1), (5, 8), (100, 3), (1000, 8), (7, 2)]:
+        L_d = rng.integers(0, 50, size=D)
+        doc_ptr = np.concatenate([[0], np.cumsum(L_d)]).astype(np.int64)
+        T = int(doc_ptr[-1])
+        b = L.lda_partition_docs(doc_ptr, world)
+        assert b[0] == 0 and b[-1] == D and np.all(np.diff(b) >= 0)
+        for g in range(1, world):
+            target = -(-g * T // world)   # ceil(g T / world)
+            expect = int(np.argmax(doc_ptr >= target)) if (doc_ptr >= target).any() else D
+            assert b[g] == max(expect, b[g - 1])
+    with pytest.raises(L.LDAError):
+        L.lda_partition_docs(np.array([0, 3, 2], np.int64), 2)
+
+
+def test_load_validation_before_device():
+    doc_ptr = np.array([0, 3, 5], np.int64)
+    words = np.array([0, 1, 2, 3, 4], np.int32)
+    cases = [
+        (dict(doc_ptr=np.array([1, 3, 5], np.int64)), L.LDA_EINVAL),            # doc_ptr[0] != 0
+        (dict(doc_ptr=np.array([0, 3, 2], np.int64)), L.LDA_EINVAL),            # decreasing
+        (dict(words=np.array([0, 1, 2, 3, 5], np.int32)), L.LDA_EINVAL),        # id >= V
+        (dict(words=np.array([0, -1, 2, 3, 4], np.int32)), L.LDA_EINVAL),       # id < 0
+        (dict(doc_end=3), L.LDA_EINVAL),                                         # range > D
+    ]
+    for over, code in cases:
+        ctx = L.lda_create(2, 5, 8, 0.1, 0.01)
+        try:
+            kw = dict(doc_begin=0, doc_end=2, doc_ptr=doc_ptr, words=words, seed=1)
+            kw.update(over)
+            with pytest.raises(L.LDAError) as e:
+                L.lda_load_corpus(ctx, **kw)
+            assert e.value.code == code, (over, e.value)
+        finally:
+            L.lda_destroy(ctx)
+    # a document longer than 65535 tokens (uint16 θ counts) -> LDA_ERANGE
+    ctx = L.lda_create(1, 2, 8, 0.1, 0.01)
+    try:
+        with pytest.raises(L.LDAError) as e:
+            L.lda_load_corpus(ctx, 0, 1, np.array([0, 65536], np.int64), np.zeros(65536, np.int32), 1)
+        assert e.value.code == L.LDA_ERANGE
+    finally:
+        L.lda_destroy(ctx)
+
+
+def test_no_gpu_fails_loudly():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    ctx = L.lda_create(2, 5, 8, 0.1, 0.01)
+    try:
+        with pytest.raises(L.LDAError) as e:
+            L.lda_load_corpus(ctx, 0, 2, np.array([0, 3, 5], np.int64), np.arange(5, dtype=np.int32), 1)
+        assert e.value.code == L.LDA_ECUDA
+        # sticky: the context stays failed
+        with pytest.raises(L.LDAError) as e2:
+            L.lda_iterate(ctx, 1)
+        assert e2.value.code == L.LDA_ECUDA
+    finally:
+        L.lda_destroy(ctx)

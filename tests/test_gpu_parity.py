@@ -1,0 +1,165 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle (-m gpu).
+
+Every case feeds both sides the same seeded synthetic corpus.  Tolerances are
+the north_star's (BASELINE.json): integer counts bit-exact; per-token z exact
+except tokens whose oracle uniform is within 1e-6 of a CDF boundary (< 1e-4
+of all tokens); LL/token within 1e-3 relative.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import lda_testutil as U
+from oracle import oracle as O
+from paper_conf_hpdc_xie0lt19_b200 import synth
+
+pytestmark = pytest.mark.gpu
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+
+
+def _corpus(D, V, T, sigma, K_gen, seed):
+    return synth.to_numpy(*synth.generate(D, V, T, sigma, K_gen, seed, "cpu"))[:2]
+
+
+def test_appendix_a_micro_bit_exact():
+    g = json.load(open(os.path.join(GOLDEN, "appendix_a_micro.json")))
+    words = np.array(sum(g["docs"], []), np.int32)
+    doc_ptr = np.cumsum([0] + [len(d) for d in g["docs"]]).astype(np.int64)
+    m = U.gpu_model(g["D"], g["V"], g["K"], g["alpha"], g["beta"], doc_ptr, words, g["seed"])
+    canon = O.canonical_order(doc_ptr, words, g["V"])
+    inv = np.argsort(canon)
+    assert m.z()[inv].tolist() == g["init"]["z_canonical"]
+    assert m.nwk().tolist() == g["init"]["n_wk"]
+    assert m.ndk_dense().tolist() == g["init"]["n_dk"]
+    assert m.nk().tolist() == g["init"]["n_k"]
+    assert m.loglik() == pytest.approx(g["init"]["ll_per_token"], rel=1e-10)
+    for sw in g["sweeps"]:
+        m.iterate(1)
+        assert m.z()[inv].tolist() == sw["z_canonical"]
+        assert m.nwk().tolist() == sw["n_wk"]
+        assert m.ndk_dense().tolist() == sw["n_dk"]
+        assert m.nk().tolist() == sw["n_k"]
+        assert m.loglik() == pytest.approx(sw["ll_per_token"], rel=1e-10)
+
+
+def test_tiny_config_lockstep_and_ll():
+    """BASELINE configs[0]: D=1000, V=500, K=16, 50k tokens, 20 sweeps."""
+    c = synth.CONFIGS["tiny"]
+    doc_ptr, words = synth.tiny_numpy()[:2]
+    o = U.oracle_for(c.D, c.V, c.K, c.alpha, c.beta, doc_ptr, words, c.seed)
+    g = U.gpu_model(c.D, c.V, c.K, c.alpha, c.beta, doc_ptr, words, c.seed)
+    assert np.array_equal(g.z(), o.z)          # init is integer: bit-exact
+    U.check_counts_equal(g, o)
+    assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
+    bad, unexc = U.lockstep(g, o, c.sweeps, teacher_force=True)
+    assert unexc == 0
+    assert bad <= U.MAX_EXCUSED_FRAC * c.T * c.sweeps
+    assert g.loglik() == pytest.approx(o.loglik(), rel=U.LL_RTOL)
+
+
+def test_tiny_config_free_running_ll_after_100():
+    """north_star: per-token LL after 100 iterations within 1e-3 relative."""
+    c = synth.CONFIGS["tiny"]
+    doc_ptr, words = synth.tiny_numpy()[:2]
+    o = U.oracle_for(c.D, c.V, c.K, c.alpha, c.beta, doc_ptr, words, c.seed)
+    g = U.gpu_model(c.D, c.V, c.K, c.alpha, c.beta, doc_ptr, words, c.seed)
+    o.iterate(100)
+    g.iterate(100)
+    llo, llg = o.loglik(), g.loglik()
+    assert llg == pytest.approx(llo, rel=U.LL_RTOL)
+    U.check_invariants_gpu(g, doc_ptr, words)
+    # the chains stayed identical (fp64 probabilities; SURVEY §7 "LL@100")
+    assert np.mean(g.z() != o.z) < 1e-3
+
+
+@pytest.mark.parametrize("K", [1, 2, 37, 128, 1024])
+def test_k_variants_lockstep(K):
+    doc_ptr, words = _corpus(600, 700, 60_000, 0.7, 16, 11)
+    a, b = 50.0 / K, 0.01
+    o = U.oracle_for(600, 700, K, a, b, doc_ptr, words, 5)
+    g = U.gpu_model(600, 700, K, a, b, doc_ptr, words, 5)
+    assert np.array_equal(g.z(), o.z)
+    U.check_counts_equal(g, o)
+    bad, unexc = U.lockstep(g, o, 3)
+    assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 60_000 * 3
+    assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
+
+
+def test_k8192_small():
+    doc_ptr, words = _corpus(300, 400, 40_000, 0.7, 64, 12)
+    K = 8192
+    o = U.oracle_for(300, 400, K, 50.0 / K, 0.01, doc_ptr, words, 9)
+    g = U.gpu_model(300, 400, K, 50.0 / K, 0.01, doc_ptr, words, 9)
+    bad, unexc = U.lockstep(g, o, 2)
+    assert unexc == 0
+
+
+def test_nytimes_shaped_midsize_many_chunks():
+    """A downscaled NYTimes-shaped corpus at K=1024 that spans many sampler
+    chunks, split words and ragged tails; options that only change the work
+    decomposition must give bit-identical results."""
+    cfg = synth.scaled(synth.CONFIGS["nytimes"], 0.002)       # ~200k tokens, V=101636
+    doc_ptr, words = synth.to_numpy(*synth.generate_config(cfg, "cpu"))[:2]
+    o = U.oracle_for(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed)
+    g = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed)
+    bad, unexc = U.lockstep(g, o, 3)
+    assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * cfg.T * 3
+    z_ref = g.z()
+    for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
+                 dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3)]:
+        h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
+        h.iterate(3)
+        assert np.array_equal(h.z(), z_ref), opts
+        assert np.array_equal(h.nwk(), g.nwk())
+
+
+def test_exclude_self_lockstep():
+    doc_ptr, words = _corpus(500, 300, 30_000, 0.5, 16, 13)
+    K = 24
+    o = U.oracle_for(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3)
+    g = U.gpu_model(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3, exclude_self=1)
+    bad, unexc = U.lockstep(g, o, 3, exclude_self=1)
+    assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
+
+
+def test_edge_cases():
+    rng = np.random.default_rng(4)
+    # empty docs, single-token docs, a 65535-token doc, absent words, D=1
+    L_d = np.array([0, 1, 0, 5, 65535, 1, 0, 3] + list(rng.integers(0, 20, 50)), np.int64)
+    doc_ptr = np.concatenate([[0], np.cumsum(L_d)]).astype(np.int64)
+    V = 300
+    words = rng.integers(0, V // 2, size=doc_ptr[-1]).astype(np.int32)   # words >= 150 absent
+    D, K = len(L_d), 40
+    o = U.oracle_for(D, V, K, 0.3, 0.02, doc_ptr, words, 77)
+    g = U.gpu_model(D, V, K, 0.3, 0.02, doc_ptr, words, 77, chunk_tokens=64)
+    assert np.array_equal(g.z(), o.z)
+    U.check_counts_equal(g, o)
+    bad, unexc = U.lockstep(g, o, 3)
+    assert unexc == 0
+    U.check_invariants_gpu(g, doc_ptr, words)
+    assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
+    # D = 1, a single token
+    o1 = U.oracle_for(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
+    g1 = U.gpu_model(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
+    U.lockstep(g1, o1, 5)
+
+
+def test_set_z_and_determinism():
+    doc_ptr, words = _corpus(400, 500, 40_000, 0.5, 16, 21)
+    K = 64
+    g1 = U.gpu_model(400, 500, K, 50.0 / K, 0.01, doc_ptr, words, 8)
+    g2 = U.gpu_model(400, 500, K, 50.0 / K, 0.01, doc_ptr, words, 8)
+    g1.iterate(4)
+    g2.iterate(4)
+    assert np.array_equal(g1.z(), g2.z())            # two runs, identical z
+    # checkpoint/resume: z + sweep counter + seed are the whole state
+    z = g1.z()
+    g3 = U.gpu_model(400, 500, K, 50.0 / K, 0.01, doc_ptr, words, 8)
+    g3.iterate(4)            # advance the counter to the same t ...
+    g3.set_z(z)              # ... and overwrite the state
+    g1.iterate(2)
+    g3.iterate(2)
+    assert np.array_equal(g1.z(), g3.z())
+    assert np.array_equal(g1.nwk(), g3.nwk())
