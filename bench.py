@@ -200,8 +200,13 @@ def run_b200(args):
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
 
+    opts = dict(C.BENCH_OPTIONS)
+    for kv in args.opt:
+        k, v = kv.split("=")
+        opts[k] = int(v)
+
     def make_model():
-        m = L.LDA(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, device=local, **C.BENCH_OPTIONS)
+        m = L.LDA(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, device=local, **opts)
         if world > 1:
             m.init_dist(rank, world, uid)
         return m
@@ -291,7 +296,7 @@ def run_b200(args):
                        "alpha": cfg.alpha, "beta": cfg.beta, "seed": cfg.seed,
                        "timed_sweeps": [int(st["sweeps_done"]) - args.steps + 1, int(st["sweeps_done"])],
                        "l2": "inputs (GBs) larger than the 126 MB L2; no flush",
-                       "parallelism": f"doc-partitioned dp{world}", "options": C.BENCH_OPTIONS},
+                       "parallelism": f"doc-partitioned dp{world}", "options": opts},
             "roofline": {"bound": "hbm", "kernel": "sweep_kernel", "achieved": achieved, "peak": peak,
                          "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
                          "peak_source": peak_src,
@@ -327,6 +332,7 @@ def main():
     ap.add_argument("--config", default="pubmed")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--opt", action="append", default=[], help="extra lda_set_option key=value")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "b200":
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

@@ -93,6 +93,8 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tile_tokens"   split the documents into tiles of about this many tokens
  *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
+ *   "theta_mode"    θ rebuild: 0 = fused gather+histogram (default),
+ *                   1 = two-phase (z gathered into document order first)
  * Results do not depend on chunk_tokens, recount_tokens, tile_tokens or
  * threads (the draw of every token is a function of the frozen counts and
  * its canonical index only).

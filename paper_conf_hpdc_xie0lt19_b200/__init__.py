@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "liblda.so")
+LIB_PATH = os.environ.get("LDA_LIBRARY") or os.path.join(_PKG, "liblda.so")
 
 LDA_OK, LDA_EINVAL, LDA_ERANGE, LDA_ENOMEM, LDA_ECUDA, LDA_ENCCL, LDA_ESTATE = 0, -1, -2, -3, -4, -5, -6
 STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4: "LDA_ECUDA",

@@ -31,13 +31,16 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Compile liblda.so (or a variant at `out` with extra -D defines)."""
+    lib_path = out or LIB
+    if out is None and not force and not _stale():
         return LIB
     objs = []
-    build_dir = os.path.join(PKG, "build")
+    build_dir = os.path.join(PKG, "build", os.path.basename(lib_path))
     os.makedirs(build_dir, exist_ok=True)
     common = ["-std=c++17", "-O3", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-I", os.path.join(ROOT, "include")]
+    common += [f"-D{d}" for d in defines]
     for src in SOURCES:
         obj = os.path.join(build_dir, src + ".o")
         cmd = [NVCC, *ARCH, *common, "-c", os.path.join(CSRC, src), "-o", obj]
@@ -47,13 +50,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
             print(" ".join(cmd), flush=True)
         subprocess.check_call(cmd)
         objs.append(obj)
-    tmp = LIB + ".tmp"
+    tmp = lib_path + ".tmp"
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-ldl", "-lpthread"]
     if verbose:
         print(" ".join(cmd), flush=True)
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib_path)
+    return lib_path
 
 
 if __name__ == "__main__":

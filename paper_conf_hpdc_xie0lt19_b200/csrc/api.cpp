@@ -26,6 +26,8 @@ struct lda_ctx {
     int64_t chunk_tokens = 4096;
     int64_t recount_tokens = 65536;
     int64_t tile_tokens = 0;
+    int theta_mode = 0;
+    int sampler = 1;
     int threads = 0;
     // distribution
     int32_t rank = 0, world = 1;
@@ -235,6 +237,12 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "tile_tokens") {
         if (value < 0) return fail(ctx, LDA_EINVAL, "tile_tokens must be >= 0");
         ctx->tile_tokens = value;
+    } else if (k == "sampler") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "sampler must be 0 or 1");
+        ctx->sampler = static_cast<int>(value);
+    } else if (k == "theta_mode") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_mode must be 0 or 1");
+        ctx->theta_mode = static_cast<int>(value);
     } else if (k == "threads") {
         if (value < 0 || value > 1024) return fail(ctx, LDA_EINVAL, "threads out of range");
         ctx->threads = static_cast<int>(value);
@@ -353,28 +361,30 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.beta = ctx->beta;
     S.seed = seed;
     S.exclude_self = ctx->exclude_self;
+    S.sampler = ctx->sampler;
     KL(lda::configure_kernels(S));
 
     DA(S.tok_row, Tg);
     DA(S.tok_z, Tg);
     DA(S.doc_map, Tg);
+    if (ctx->theta_mode == 1) DA(S.z_doc, Tg + 4);
     DA(S.doc_ptr32, Dg + 1);
-    DA(S.row_off16, std::max<int64_t>(Dg, 1));
-    DA(S.tseg, H.tseg.size());
+    DA(S.row_off32, std::max<int64_t>(Dg, 1));
+    DA(S.segs, H.segs.size());
     S.n_chunks = static_cast<int64_t>(H.chunks.size());
     DA(S.chunks, H.chunks.size());
     S.n_rchunks = static_cast<int64_t>(H.rchunks.size());
     DA(S.rchunks, H.rchunks.size());
     S.n_split = static_cast<int64_t>(H.split_words.size());
     DA(S.split_words, H.split_words.size());
-    DA(S.rows, H.rows16 * 4);
+    DA(S.rows, H.rows32 * 8);
     DA(S.nwk, static_cast<size_t>(V) * K + K);
-    DA(S.invk, K);
+    DA(S.denom, K);
     DA(S.counter, 4);
     DA(S.stat, 4);
     DA(S.ll_part, 2 * S.ll_blocks + 2);
     DA(S.ll_out, 2);
-    if (S.sweep_smem == 0) DA(S.sweep_scratch, static_cast<size_t>(S.sweep_grid) * 2 * K);
+    if (S.sweep_smem < static_cast<size_t>(16) * K + 4096) DA(S.sweep_scratch, static_cast<size_t>(S.sweep_grid) * 2 * K);
 
     auto h2d = [&](void *dst, const void *src, size_t bytes) {
         return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream) : cudaSuccess;
@@ -382,12 +392,12 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(h2d(S.tok_row, H.tok_row.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.doc_map, H.doc_map.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.doc_ptr32, H.doc_ptr32.data(), sizeof(uint32_t) * (Dg + 1)));
-    CU(h2d(S.row_off16, H.row_off16.data(), sizeof(uint32_t) * Dg));
-    CU(h2d(S.tseg, H.tseg.data(), sizeof(uint32_t) * H.tseg.size()));
+    CU(h2d(S.row_off32, H.row_off32.data(), sizeof(uint32_t) * Dg));
+    CU(h2d(S.segs, H.segs.data(), sizeof(lda::Seg) * H.segs.size()));
     CU(h2d(S.chunks, H.chunks.data(), sizeof(lda::SampleChunk) * H.chunks.size()));
     CU(h2d(S.rchunks, H.rchunks.data(), sizeof(lda::RecountChunk) * H.rchunks.size()));
     CU(h2d(S.split_words, H.split_words.data(), sizeof(int32_t) * H.split_words.size()));
-    CU(cudaMemsetAsync(S.rows, 0, H.rows16 * 16, ctx->stream));
+    CU(cudaMemsetAsync(S.rows, 0, H.rows32 * 32, ctx->stream));
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
     // a1: random init (t = 0), then the count rebuild.
@@ -543,16 +553,16 @@ int lda_get_counts(lda_ctx *ctx, int32_t *n_wk, int32_t *n_k, int64_t *ndk_ptr, 
     if (n_k) CU(cudaMemcpy(n_k, S.nwk + static_cast<size_t>(S.V) * S.K, sizeof(int32_t) * S.K,
                            cudaMemcpyDeviceToHost));
     if (ndk_ptr || ndk_topic || ndk_count || ndk_nnz_out) {
-        std::vector<uint32_t> rows(H.rows16 * 4);
+        std::vector<uint32_t> rows(H.rows32 * 8);
         CU(cudaMemcpy(rows.data(), S.rows, rows.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
         int64_t nnz = 0;
-        for (int64_t d = 0; d < S.D; ++d) nnz += rows[static_cast<size_t>(H.row_off16[d]) * 4];
+        for (int64_t d = 0; d < S.D; ++d) nnz += rows[static_cast<size_t>(H.row_off32[d]) * 8];
         if (ndk_nnz_out) *ndk_nnz_out = nnz;
         if ((ndk_topic || ndk_count) && ndk_capacity < nnz)
             return fail(ctx, LDA_ERANGE, "ndk_capacity smaller than nnz");
         int64_t pos = 0;
         for (int64_t d = 0; d < S.D; ++d) {
-            const uint32_t *row = rows.data() + static_cast<size_t>(H.row_off16[d]) * 4;
+            const uint32_t *row = rows.data() + static_cast<size_t>(H.row_off32[d]) * 8;
             if (ndk_ptr) ndk_ptr[d] = pos;
             for (uint32_t j = 0; j < row[0]; ++j, ++pos) {
                 if (ndk_topic) ndk_topic[pos] = static_cast<uint16_t>(row[1 + j] >> 16);

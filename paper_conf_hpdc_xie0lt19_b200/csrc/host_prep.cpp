@@ -81,20 +81,22 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     L.K = K;
     nthreads = host_threads(nthreads);
 
-    // θ rows: capacity min(L_d, K) entries + 1 header word, 16-byte aligned.
+    // θ rows: 1 header word (nnz) + capacity min(L_d, K) entries, rounded up
+    // to whole 32-byte sectors; words past nnz are kept zero (zero-mass
+    // padding the sampler may read without a bounds check).
     L.doc_ptr32.resize(D + 1);
-    L.row_off16.resize(D);
-    uint64_t off16 = 0;
+    L.row_off32.resize(D);
+    uint64_t off32 = 0;
     for (int64_t d = 0; d < D; ++d) {
         int64_t len = doc_ptr[d + 1] - doc_ptr[d];
         int64_t cap = std::min<int64_t>(len, K);
         L.doc_ptr32[d] = static_cast<uint32_t>(doc_ptr[d]);
-        L.row_off16[d] = static_cast<uint32_t>(off16);
-        off16 += static_cast<uint64_t>((cap + 1 + 3) / 4);
-        if (off16 >= (uint64_t(1) << 32) - 64) return "θ row storage exceeds 2^32 x 16 bytes";
+        L.row_off32[d] = static_cast<uint32_t>(off32);
+        off32 += static_cast<uint64_t>((cap + 1 + 7) / 8);
+        if (off32 >= (uint64_t(1) << 32) - 64) return "θ row storage exceeds 2^32 x 32 bytes";
     }
     L.doc_ptr32[D] = static_cast<uint32_t>(T);
-    L.rows16 = off16 + 64;  // tail pad: the sampler may read up to 32 x 16 B past a row
+    L.rows32 = off32 + 4;  // tail pad
 
     // Doc tiles: contiguous document ranges of about tile_tokens tokens.
     std::vector<int64_t> tile_doc{0};
@@ -115,7 +117,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 
     L.tok_row.assign(T, 0);
     L.doc_map.assign(T, 0);
-    L.tseg.assign(static_cast<size_t>(nt) * V + 1, 0);
+    std::vector<uint32_t> tseg(static_cast<size_t>(nt) * V, 0);  // run start of (tile, word)
     L.word_count.assign(V, 0);
     std::vector<std::vector<uint32_t>> tile_cnt(nt);
 
@@ -144,7 +146,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         cnt.assign(V, 0);
         uint64_t pos = static_cast<uint64_t>(t0);
         for (int32_t w = 0; w < V; ++w) {
-            L.tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
+            tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
             uint64_t run = pos;
             for (int t = 0; t < nth; ++t) {
                 uint32_t h = hist[t][w];
@@ -158,7 +160,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         auto scatter_part = [&](int t) {
             auto &next = hist[t];
             for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
-                uint32_t row = L.row_off16[d];
+                uint32_t row = L.row_off32[d];
                 for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
                     uint32_t p = next[words[i]]++;
                     L.doc_map[i] = p;
@@ -173,51 +175,65 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             for (auto &x : th) x.join();
         }
     }
-    L.tseg[static_cast<size_t>(nt) * V] = static_cast<uint32_t>(T);
 
-    // Sampling work items: per (tile, word) segment, split into near-equal
-    // pieces of <= chunk_tokens; c_base continues word w's canonical run
-    // across tiles (tiles are increasing doc ranges, so (tile, d, j) order
-    // restricted to word w is its (d, j) order).
-    L.chunks.clear();
-    std::vector<int64_t> woff(V, 0);
-    for (int b = 0; b < nt; ++b) {
-        for (int32_t w = 0; w < V; ++w) {
-            int64_t n = tile_cnt[b][w];
+    // Per-word runs (tile order) + sentinel; segment index of each word's first run.
+    L.segs.clear();
+    std::vector<uint64_t> wseg0(V);
+    for (int32_t w = 0; w < V; ++w) {
+        wseg0[w] = L.segs.size();
+        uint32_t acc = 0;
+        for (int b = 0; b < nt; ++b) {
+            uint32_t n = tile_cnt[b][w];
             if (n == 0) continue;
-            int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
-            uint32_t seg = L.tseg[static_cast<size_t>(b) * V + w];
-            int64_t done = 0;
-            for (int64_t p = 0; p < pieces; ++p) {
-                int64_t sz = n * (p + 1) / pieces - n * p / pieces;
-                SampleChunk c;
-                c.begin = static_cast<uint32_t>(seg + done);
-                c.count = static_cast<uint32_t>(sz);
-                c.word = static_cast<uint32_t>(w);
-                c.pad = 0;
-                c.c_base = static_cast<uint64_t>(cbase[w] + woff[w] + done);
-                L.chunks.push_back(c);
-                done += sz;
-            }
-            woff[w] += n;
+            L.segs.push_back(Seg{tseg[static_cast<size_t>(b) * V + w], acc});
+            acc += n;
+        }
+        L.segs.push_back(Seg{0u, acc});
+    }
+    if (L.segs.size() >= (uint64_t(1) << 32)) return "too many word runs";
+    std::vector<uint32_t>().swap(tseg);
+    auto seg_of = [&](int32_t w, uint32_t v) {
+        uint64_t s = wseg0[w];
+        while (L.segs[s + 1].vstart <= v && L.segs[s + 1].vstart < L.word_count[w]) ++s;
+        return static_cast<uint32_t>(s);
+    };
+
+    // Sampling work items: word w's tokens in near-equal pieces of at most
+    // chunk_tokens, each a virtual range spanning the word's runs; the
+    // canonical index continues word w's run on this rank (cbase[w] + v).
+    L.chunks.clear();
+    for (int32_t w = 0; w < V; ++w) {
+        const int64_t n = L.word_count[w];
+        if (n == 0) continue;
+        const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
+        for (int64_t q = 0; q < pieces; ++q) {
+            const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
+            SampleChunk c;
+            c.word = static_cast<uint32_t>(w);
+            c.vbegin = static_cast<uint32_t>(vb);
+            c.count = static_cast<uint32_t>(ve - vb);
+            c.seg0 = seg_of(w, static_cast<uint32_t>(vb));
+            c.c_base = static_cast<uint64_t>(cbase[w] + vb);
+            L.chunks.push_back(c);
         }
     }
     std::stable_sort(L.chunks.begin(), L.chunks.end(),
                      [](const SampleChunk &a, const SampleChunk &b) { return a.count > b.count; });
 
-    // Recount work items: per word over its tile segments.
+    // Recount work items: per word, pieces of at most recount_tokens.
     L.rchunks.clear();
     L.split_words.clear();
     for (int32_t w = 0; w < V; ++w) {
-        int64_t n = L.word_count[w];
-        int64_t pieces = std::max<int64_t>(1, (n + recount_tokens - 1) / recount_tokens);
+        const int64_t n = L.word_count[w];
+        const int64_t pieces = std::max<int64_t>(1, (n + recount_tokens - 1) / recount_tokens);
         if (pieces > 1) L.split_words.push_back(w);
-        for (int64_t p = 0; p < pieces; ++p) {
+        for (int64_t q = 0; q < pieces; ++q) {
+            const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
             RecountChunk c;
-            c.word = static_cast<uint32_t>(w);
-            c.vbegin = static_cast<uint32_t>(n * p / pieces);
-            c.vcount = static_cast<uint32_t>(n * (p + 1) / pieces - n * p / pieces);
-            c.split = pieces > 1 ? 1u : 0u;
+            c.word = static_cast<uint32_t>(w) | (pieces > 1 ? 0x80000000u : 0u);
+            c.vbegin = static_cast<uint32_t>(vb);
+            c.vcount = static_cast<uint32_t>(ve - vb);
+            c.seg0 = n ? seg_of(w, static_cast<uint32_t>(vb)) : static_cast<uint32_t>(wseg0[w]);
             L.rchunks.push_back(c);
         }
     }

@@ -1,12 +1,12 @@
 // CUDA kernels of the LDA collapsed-Gibbs sweep, written for sm_100a (B200).
 //
 // Path per sweep t (§6):
-//   prologue_kernel   invk[k] = 1/(n_k + Vβ)                (Eq. 1/8 denominator)
-//   sweep_kernel      per word chunk: p*(k) = (n_wk+β)·invk[k] and the dense
+//   prologue_kernel   denom[k] = n_k + Vβ                    (Eq. 1/8 denominator)
+//   sweep_kernel      per word chunk: p*(k) = (n_wk+β)/denom[k] and the dense
 //                     prefix of α·p* in shared memory (Eq. 8);
-//                     per token: sparse doc row walk, S, one Philox uniform,
-//                     x = U·(S+Q), group ballot search in the sparse prefix or a
-//                     32-ary ballot search in the dense prefix (Eq. 6-7,
+//                     per token (one sampler per lane): sparse doc row walk,
+//                     S, one Philox uniform, x = U·(S+Q), rescan of the sparse
+//                     prefix or binary search of the dense prefix (Eq. 6-7,
 //                     Fig. 5, Alg. 2; L1019-1133)
 //   recount_kernel    n_wk, n_k rebuilt from z by per-word segmented histograms
 //                     (ϕ update, L1273-1285)
@@ -26,6 +26,14 @@ namespace lda {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kSweepThreads = 256;
+constexpr int kMaxBlk = 16;  // block-end prefixes kept per token for the sparse rescan
+#ifndef LDA_RING
+#define LDA_RING 6
+#endif
+#ifndef LDA_SWEEP_MINB
+#define LDA_SWEEP_MINB 3
+#endif
+constexpr int kRing = LDA_RING;  // 16-byte row quads in flight per sampler lane
 
 // ---------------------------------------------------------------------------
 // Philox4x32-10 (Salmon et al. SC'11), output word 0 only.  Counter
@@ -55,199 +63,122 @@ __device__ __forceinline__ uint4 ld_nc_v4(const uint4 *p) {
     return v;
 }
 
+// Bring [p, p + bytes) into L2 without a register or scoreboard slot (one
+// bulk-prefetch instruction per θ row; bytes a multiple of 16).
+__device__ __forceinline__ void prefetch_l2_bulk(const void *p, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+
+// Word-major position of virtual index v of a word, walking the word's runs
+// forward from run s (v must not decrease between calls with the same s).
+__device__ __forceinline__ uint32_t run_position(const Seg *__restrict__ segs, uint32_t &s, uint32_t v) {
+    while (segs[s + 1].vstart <= v) ++s;
+    return segs[s].pos + (v - segs[s].vstart);
+}
+
 // ---------------------------------------------------------------------------
 // a1: random initial assignment (L377-379; X10): z = (x0·K) >> 32, t = 0.
 // ---------------------------------------------------------------------------
 __global__ void init_kernel(const SampleChunk *__restrict__ chunks, int64_t n_chunks,
-                            uint16_t *__restrict__ z, uint32_t K, uint32_t k0, uint32_t k1) {
+                            const Seg *__restrict__ segs, uint16_t *__restrict__ z, uint32_t K, uint32_t k0,
+                            uint32_t k1) {
     for (int64_t ci = blockIdx.x; ci < n_chunks; ci += gridDim.x) {
         const SampleChunk ch = chunks[ci];
+        uint32_t sg = ch.seg0;
         for (uint32_t j = threadIdx.x; j < ch.count; j += blockDim.x) {
             const uint32_t x0 = philox_x0(ch.c_base + j, 0u, k0, k1);
-            z[ch.begin + j] = static_cast<uint16_t>((static_cast<uint64_t>(x0) * K) >> 32);
+            z[run_position(segs, sg, ch.vbegin + j)] =
+                static_cast<uint16_t>((static_cast<uint64_t>(x0) * K) >> 32);
         }
     }
 }
 
 // ---------------------------------------------------------------------------
-// a2: sweep prologue, invk[k] = 1 / (n_k + Vβ)  (fp64).
+// a2: sweep prologue, denom[k] = n_k + Vβ  (fp64, Eq. 1 / Eq. 8 denominator).
 // ---------------------------------------------------------------------------
 __global__ void prologue_kernel(const int32_t *__restrict__ nk, int K, double Vbeta,
-                                double *__restrict__ invk) {
+                                double *__restrict__ denom) {
     for (int k = blockIdx.x * blockDim.x + threadIdx.x; k < K; k += gridDim.x * blockDim.x)
-        invk[k] = 1.0 / (static_cast<double>(nk[k]) + Vbeta);
+        denom[k] = static_cast<double>(nk[k]) + Vbeta;
 }
 
 // ---------------------------------------------------------------------------
 // a3 + a4: the sampling kernel.
+//
+// Persistent CTAs pull word chunks from a queue (heavy-first, L1203-1221).
+// Per chunk the CTA builds, in shared memory, p*(k) = (n_wk + β)/(n_k + Vβ)
+// (Eq. 8, one division per topic, the oracle's exact expression) and the
+// inclusive prefix P of α·p*(k) (the dense bucket p2 of Eq. 6, shared by all
+// tokens of the word: Fig. 6).  Then every thread draws its own
+// tokens (one sampler per lane):
+//   pass 1   S = Σ_j c_j·p*(t_j) over the doc's θ row (p1 of Eq. 6, Eq. 7),
+//            32-byte row blocks, zero-mass padding, no per-entry bounds check
+//   draw     x = U·(S+Q), U = x0·2^-32 from Philox(seed; c, t) (X4, X8, X9)
+//   sparse   x < S: rescan the row, first entry with prefix > x (X5, X6)
+//   dense    else: binary search of the first k with S + P[k] > x (Fig. 5)
+// θ rows: word 0 = nnz, words 1..nnz = topic << 16 | count (ascending topics,
+// X7), zero words up to the next 32-byte boundary.
 // ---------------------------------------------------------------------------
 struct SweepArgs {
     const SampleChunk *chunks;
     int64_t n_chunks;
+    const Seg *segs;
     const uint32_t *tok_row;
     uint16_t *z;
     const uint4 *rows;
     const int32_t *nwk;
     const int32_t *nk;
-    const double *invk;
+    const double *denom;
     uint32_t *counter;
     double *gscratch;  // non-null when the K-length arrays do not fit in smem
     int K;
-    int top_step;
     double alpha, beta, Vbeta;
-    uint32_t t, k0, k1;
+    uint32_t t;
+    uint32_t key0[10], key1[10];  // Philox key schedule (seed + r·W)
 };
 
-// One token, drawn by a group of GS lanes (GS | 32).  Returns the new topic
-// on every lane of the group.
-//   row layout: word 0 = nnz, words 1..nnz = (topic << 16 | count), topics
-//   ascending (X7).  Lane q of the group owns words 4q..4q+3 of each 4·GS-word
-//   slice; its masses are count·p*(topic) (p1 of Eq. 6 via Eq. 8).
-// Bins: [sparse entries in row order] ++ [dense α·p*(k), k = 0..K-1] (X4-X6).
-template <int GS, bool EXCL>
-__device__ __forceinline__ int draw_token(const SweepArgs &a, const double *__restrict__ pstar,
-                                          const double *__restrict__ P, double Q,
-                                          const int32_t *__restrict__ nwk_row, uint32_t trow,
-                                          uint32_t x0, int zo, unsigned gmask, int q, int gbase) {
-    const uint4 *r = a.rows + trow;
-    uint4 v = ld_nc_v4(r + q);
-    const uint32_t len = __shfl_sync(gmask, v.x, gbase);
-    const uint32_t nwords = len + 1;
-    const int iters = static_cast<int>((nwords + 4 * GS - 1) / (4 * GS));
-
-    // exclude_self (X2 optional variant): the token's own topic zo loses one
-    // count in n_dk, n_wk and n_k.
-    double po_new = 0.0, delta = 0.0;
-    if (EXCL) {
-        po_new = (static_cast<double>(nwk_row[zo] - 1) + a.beta) /
-                 (static_cast<double>(a.nk[zo] - 1) + a.Vbeta);
-        delta = a.alpha * po_new - a.alpha * pstar[zo];
-    }
-
-    double c0 = 0, c1 = 0, c2 = 0, c3 = 0;
-    uint32_t e0 = 0, e1 = 0, e2 = 0, e3 = 0;
-    uint32_t wb = 0;  // word index of this lane's first word in the slice
-
-    // computes c0..c3 for slice `it` from v; returns the slice's group total
-    auto slice = [&](int it, double carry) -> double {
-        wb = static_cast<uint32_t>(it * 4 * GS + 4 * q);
-        e0 = v.x; e1 = v.y; e2 = v.z; e3 = v.w;
-        double m0 = 0, m1 = 0, m2 = 0, m3 = 0;
-#define LDA_MASS(mi, ei, off)                                                              \
-    if (wb + off >= 1 && wb + off <= len) {                                                \
-        const uint32_t tp = ei >> 16, cn = ei & 0xFFFFu;                                   \
-        mi = (EXCL && static_cast<int>(tp) == zo) ? static_cast<double>(cn - 1) * po_new   \
-                                                  : static_cast<double>(cn) * pstar[tp];   \
-    }
-        LDA_MASS(m0, e0, 0)
-        LDA_MASS(m1, e1, 1)
-        LDA_MASS(m2, e2, 2)
-        LDA_MASS(m3, e3, 3)
-#undef LDA_MASS
-        const double l0 = m0, l1 = l0 + m1, l2 = l1 + m2, l3 = l2 + m3;
-        double incl = l3;
+__device__ __forceinline__ uint32_t philox_x0_sched(uint64_t c, uint32_t t, const uint32_t *k0,
+                                                    const uint32_t *k1) {
+    uint32_t c0 = static_cast<uint32_t>(c), c1 = static_cast<uint32_t>(c >> 32), c2 = t, c3 = 0u;
 #pragma unroll
-        for (int o = 1; o < GS; o <<= 1) {
-            const double y = __shfl_up_sync(gmask, incl, o, GS);
-            if (q >= o) incl += y;
-        }
-        double ex = __shfl_up_sync(gmask, incl, 1, GS);
-        if (q == 0) ex = 0.0;
-        const double base = carry + ex;
-        c0 = base + l0;
-        c1 = base + l1;
-        c2 = base + l2;
-        c3 = base + l3;
-        return __shfl_sync(gmask, incl, GS - 1, GS);
-    };
-
-    // pass 1: S = inclusive prefix at the last sparse entry (word `len`)
-    double carry = 0.0, S = 0.0;
-    for (int it = 0; it < iters; ++it) {
-        if (it > 0) {
-            const uint32_t w0 = static_cast<uint32_t>(it * 4 * GS + 4 * q);
-            v = (w0 < nwords) ? ld_nc_v4(r + it * GS + q) : make_uint4(0u, 0u, 0u, 0u);
-        }
-        const double tot = slice(it, carry);
-        if (it == iters - 1 && len > 0) {
-            const uint32_t rel = len - static_cast<uint32_t>(it * 4 * GS);
-            const int src = gbase + static_cast<int>(rel >> 2);
-            const uint32_t i = rel & 3u;
-            const double mine = i == 0 ? c0 : (i == 1 ? c1 : (i == 2 ? c2 : c3));
-            S = __shfl_sync(gmask, mine, src);
-        }
-        carry = carry + tot;
+    for (int r = 0; r < 10; ++r) {
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
+        c0 = hi1 ^ c1 ^ k0[r];
+        c1 = lo1;
+        c2 = hi0 ^ c3 ^ k1[r];
+        c3 = lo0;
     }
-
-    const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;  // x0 · 2^-32
-    const double x = U * (S + (EXCL ? Q + delta : Q));
-
-    if (x < S) {
-        // sparse bucket (p1): first entry with C > x.  For rows longer than
-        // one slice, recompute each slice bit-identically to pass 1.
-        double carry2 = 0.0;
-        for (int it = 0; it < iters; ++it) {
-            double tot = 0.0;
-            if (iters > 1) {
-                const uint32_t w0 = static_cast<uint32_t>(it * 4 * GS + 4 * q);
-                v = (w0 < nwords) ? ld_nc_v4(r + it * GS + q) : make_uint4(0u, 0u, 0u, 0u);
-                tot = slice(it, carry2);
-            }
-            const bool f0 = wb + 0 >= 1 && wb + 0 <= len && c0 > x;
-            const bool f1 = wb + 1 >= 1 && wb + 1 <= len && c1 > x;
-            const bool f2 = wb + 2 >= 1 && wb + 2 <= len && c2 > x;
-            const bool f3 = wb + 3 >= 1 && wb + 3 <= len && c3 > x;
-            const unsigned bal = __ballot_sync(gmask, f0 || f1 || f2 || f3) & gmask;
-            if (bal) {
-                const uint32_t e = f0 ? e0 : (f1 ? e1 : (f2 ? e2 : e3));
-                return static_cast<int>(__shfl_sync(gmask, e, __ffs(bal) - 1) >> 16);
-            }
-            carry2 = carry2 + tot;
-        }
-        return a.K - 1;  // unreachable: the entry at word `len` has C == S > x
-    }
-
-    // dense bucket (p2): first k with S + P[k] (+Δ for k >= zo) > x, by a
-    // 32-ary search whose candidates are split over the group's lanes
-    // (the index tree of Fig. 5 / Fig. 6).
-    constexpr int PER = 32 / GS;
-    int base = 0, step = a.top_step;
-    for (;;) {
-        int first = 32;
-#pragma unroll
-        for (int i = 0; i < PER; ++i) {
-            const int j = q * PER + i;
-            int idx = base + (j + 1) * step - 1;
-            if (idx > a.K - 1) idx = a.K - 1;
-            double pk = P[idx];
-            if (EXCL && idx >= zo) pk += delta;
-            if (first == 32 && S + pk > x) first = j;
-        }
-        const unsigned bal = __ballot_sync(gmask, first < 32) & gmask;
-        int js;
-        if (bal) {
-            js = __shfl_sync(gmask, first, __ffs(bal) - 1);
-        } else {
-            if (step == a.top_step) return a.K - 1;  // x >= total (rounding), X6 fallback
-            js = 31;
-        }
-        if (step == 1) return min(base + js, a.K - 1);
-        base += js * step;
-        step >>= 5;
-    }
+    return c0;
 }
 
-template <int GS, bool EXCL>
-__global__ void __launch_bounds__(kSweepThreads) sweep_kernel(SweepArgs a) {
+template <bool EXCL>
+struct Mass {
+    // mass of one θ entry e = topic << 16 | count under the word's p*
+    __device__ __forceinline__ static double fma_into(uint32_t e, const double *__restrict__ pstar, int zo,
+                                                      double po_new, double acc) {
+        const uint32_t tp = e >> 16;
+        uint32_t cn = e & 0xFFFFu;
+        double p = pstar[tp];
+        if (EXCL && static_cast<int>(tp) == zo && cn != 0u) {
+            cn -= 1u;
+            p = po_new;
+        }
+        return fma(static_cast<double>(cn), p, acc);
+    }
+};
+
+template <bool EXCL>
+__global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(SweepArgs a) {
     extern __shared__ double smem_d[];
     __shared__ int s_ci;
     __shared__ double s_wtot[kSweepThreads / 32];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    constexpr int NG = 32 / GS;
-    const int g = lane / GS, q = lane % GS, gbase = g * GS;
-    const unsigned gmask = (GS == 32) ? kFull : (((1u << GS) - 1u) << gbase);
     const int K = a.K;
-    double *pstar = a.gscratch ? a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K : smem_d;
+    // smem: [blkC: kMaxBlk x 256 fp64][p*: K][P: K] (p*/P in global scratch for large K)
+    double *blkC = smem_d;
+    double *pstar = a.gscratch ? a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K
+                               : smem_d + kMaxBlk * kSweepThreads;
     double *P = pstar + K;
     const int E = (K + kSweepThreads - 1) / kSweepThreads;
     int cur_word = -1;
@@ -267,7 +198,7 @@ __global__ void __launch_bounds__(kSweepThreads) sweep_kernel(SweepArgs a) {
             for (int e = 0; e < E; ++e) {
                 const int k = kb + e;
                 if (k < K) {
-                    const double ps = (static_cast<double>(__ldg(nwk_row + k)) + a.beta) * __ldg(a.invk + k);
+                    const double ps = (static_cast<double>(__ldg(nwk_row + k)) + a.beta) / __ldg(a.denom + k);
                     pstar[k] = ps;
                     run = run + a.alpha * ps;
                     P[k] = run;
@@ -295,27 +226,368 @@ __global__ void __launch_bounds__(kSweepThreads) sweep_kernel(SweepArgs a) {
         }
         const double Q = P[K - 1];
 
-        for (uint32_t b0 = static_cast<uint32_t>(warp) * 32; b0 < ch.count; b0 += kSweepThreads) {
-            const uint32_t jj = b0 + lane;
-            const bool valid = jj < ch.count;
-            const uint32_t p = ch.begin + jj;
-            const uint32_t row = valid ? __ldg(a.tok_row + p) : 0u;
-            const uint32_t x0 = philox_x0(ch.c_base + jj, a.t, a.k0, a.k1);
-            const int zo = (EXCL && valid) ? static_cast<int>(a.z[p]) : 0;
-            int myz = 0;
-#pragma unroll 1
-            for (int r = 0; r < GS; ++r) {
-                const int j = r * NG + g;
-                const uint32_t trow = __shfl_sync(kFull, row, j);
-                const uint32_t tx0 = __shfl_sync(kFull, x0, j);
-                const int tzo = __shfl_sync(kFull, zo, j);
-                int zn = 0;
-                if (b0 + static_cast<uint32_t>(j) < ch.count)
-                    zn = draw_token<GS, EXCL>(a, pstar, P, Q, nwk_row, trow, tx0, tzo, gmask, q, gbase);
-                const int got = __shfl_sync(kFull, zn, (lane % NG) * GS);
-                if (r == lane / NG) myz = got;
+        // One sampler per lane; each thread draws tokens j, j+256, ...  The
+        // row is streamed in 16-byte quads through a ring of kRing quads held
+        // in registers, so ~kRing·16 B per thread are in flight (a 32-byte
+        // block = 2 quads; words past nnz in the last block are zero).
+        uint32_t sg = ch.seg0;
+        for (uint32_t j = tid; j < ch.count; j += kSweepThreads) {
+            const uint32_t p = run_position(a.segs, sg, ch.vbegin + j);
+            const uint32_t row = __ldg(a.tok_row + p);
+            const uint4 *r = a.rows + static_cast<size_t>(row) * 2;
+            uint4 q[kRing];
+            q[0] = ld_nc_v4(r);            // header quad: nnz + 3 entries
+#pragma unroll
+            for (int i = 1; i < kRing; ++i) q[i] = make_uint4(0u, 0u, 0u, 0u);
+            q[1] = ld_nc_v4(r + 1);        // every row has >= 1 block = 2 quads
+            const uint32_t x0 = philox_x0_sched(ch.c_base + j, a.t, a.key0, a.key1);
+            int zo = 0;
+            double po_new = 0.0, delta = 0.0;
+            if (EXCL) {
+                zo = static_cast<int>(a.z[p]);
+                po_new = (static_cast<double>(nwk_row[zo] - 1) + a.beta) /
+                         (static_cast<double>(a.nk[zo] - 1) + a.Vbeta);
+                delta = a.alpha * po_new - a.alpha * pstar[zo];
             }
-            if (valid) a.z[p] = static_cast<uint16_t>(myz);
+            const uint32_t len = q[0].x;
+            const uint32_t nblk = (len + 8u) >> 3;   // 32-byte blocks holding words 0..len
+            const uint32_t nq = 2u * nblk;           // quads to stream (zero-padded tail)
+#pragma unroll
+            for (int i = 2; i < kRing; ++i)
+                if (static_cast<uint32_t>(i) < nq) q[i] = ld_nc_v4(r + i);
+            // pass 1: S over the row, block-end prefixes to smem
+            double S = 0.0;
+            S = Mass<EXCL>::fma_into(q[0].y, pstar, zo, po_new, S);
+            S = Mass<EXCL>::fma_into(q[0].z, pstar, zo, po_new, S);
+            S = Mass<EXCL>::fma_into(q[0].w, pstar, zo, po_new, S);
+            q[0] = (static_cast<uint32_t>(kRing) < nq) ? ld_nc_v4(r + kRing) : make_uint4(0u, 0u, 0u, 0u);
+            // quads 1 .. nq-1, ring slot (qi % kRing); qi odd ends a block
+            for (uint32_t base = 0; base < nq; base += kRing) {
+#pragma unroll
+                for (int i = 0; i < kRing; ++i) {
+                    const uint32_t qi = base + i;
+                    if (qi == 0) continue;
+                    if (qi >= nq) break;
+                    const uint4 u = q[i];
+                    const uint32_t nx = qi + kRing;
+                    q[i] = (nx < nq) ? ld_nc_v4(r + nx) : make_uint4(0u, 0u, 0u, 0u);
+                    S = Mass<EXCL>::fma_into(u.x, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u.y, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u.z, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u.w, pstar, zo, po_new, S);
+                    if (qi & 1u) {
+                        const uint32_t b = qi >> 1;
+                        if (b < kMaxBlk) blkC[b * kSweepThreads + tid] = S;
+                    }
+                }
+            }
+            const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;  // x0 · 2^-32
+            const double x = U * (S + (EXCL ? Q + delta : Q));
+            int z;
+            if (x < S) {
+                // sparse bucket (p1): the first block whose end prefix exceeds x,
+                // then the identical recomputation inside it: first C > x
+                const uint32_t nb = nblk < kMaxBlk ? nblk : kMaxBlk;
+                uint32_t b = 0;
+                while (b < nb && !(blkC[b * kSweepThreads + tid] > x)) ++b;
+                double C = b == 0 ? 0.0 : blkC[(b - 1) * kSweepThreads + tid];
+                z = -1;
+#define LDA_STEP(e)                                                   \
+    {                                                                 \
+        C = Mass<EXCL>::fma_into((e), pstar, zo, po_new, C);          \
+        if (z < 0 && C > x) z = static_cast<int>((e) >> 16);          \
+    }
+                for (; z < 0 && b < nblk; ++b) {  // one block, or a linear tail past kMaxBlk
+                    const uint4 u0 = ld_nc_v4(r + 2 * b), u1 = ld_nc_v4(r + 2 * b + 1);
+                    if (b > 0) LDA_STEP(u0.x)
+                    LDA_STEP(u0.y) LDA_STEP(u0.z) LDA_STEP(u0.w)
+                    LDA_STEP(u1.x) LDA_STEP(u1.y) LDA_STEP(u1.z) LDA_STEP(u1.w)
+                }
+#undef LDA_STEP
+                if (z < 0) z = K - 1;  // unreachable: the last entry's prefix is S > x
+            } else {
+                // dense bucket (p2): first k with S + P[k] (+Δ for k >= zo) > x
+                int lo = 0, hi = K - 1;
+                while (lo < hi) {
+                    const int mid = (lo + hi) >> 1;
+                    double pk = P[mid];
+                    if (EXCL && mid >= zo) pk += delta;
+                    if (S + pk > x) hi = mid;
+                    else lo = mid + 1;
+                }
+                z = lo;  // K-1 also when x >= S + Q by rounding (X6 fallback)
+            }
+            a.z[p] = static_cast<uint16_t>(z);
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a3 + a4, TMA-staged variant (the default sampler).
+//
+// Same arithmetic as sweep_kernel, but the θ rows are moved by the Tensor
+// Memory Accelerator instead of per-thread loads: each warp draws 32 tokens
+// at a time (one sampler per lane); a lane first loads its row's 32-byte
+// header block (nnz + 7 entries), then issues ONE cp.async.bulk copy of the
+// rest of its row into the warp's shared-memory stage, completing on an
+// mbarrier.  Two stages per warp: the bulk copies of batch i+1 and the header
+// loads of batch i+2 are in flight while batch i is drawn from shared memory,
+// so the memory system sees ~2 x 32 whole rows in flight per warp with no
+// registers tied up (the direct-load sampler above keeps ~1 block per thread
+// in flight and is latency-bound).
+// ---------------------------------------------------------------------------
+constexpr int kTW = 4;                // warps per CTA
+constexpr int kTThreads = 32 * kTW;   // 128
+constexpr int kTCap = 288;            // staged 32-byte blocks per warp per stage (~9 per lane)
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    }
+}
+__device__ __forceinline__ void tma_row_to_smem(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+struct TBatch {
+    uint32_t p;     // word-major position of the lane's token
+    uint32_t row;   // θ row of its document, 32-byte units
+    uint4 h0, h1;   // row block 0: nnz + 7 entries
+    uint32_t off;   // first staged block in the warp's stage
+    uint32_t nst;   // staged blocks (row blocks 1..nst)
+    bool valid;
+};
+
+template <bool EXCL>
+__global__ void __launch_bounds__(kTThreads) sweep_tma_kernel(SweepArgs a) {
+    extern __shared__ __align__(128) unsigned char smem_t[];
+    __shared__ uint64_t mbar[2][kTW];
+    __shared__ int s_ci;
+    __shared__ double s_wtot[kTW];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int K = a.K;
+    // smem: [stage 0: kTW x kTCap x 32 B][stage 1][blkC: kMaxBlk x 128 fp64][p*: K][P: K]
+    uint4 *stage0 = reinterpret_cast<uint4 *>(smem_t);
+    double *blkC = reinterpret_cast<double *>(smem_t + 2 * kTW * kTCap * 32);
+    double *pstar = a.gscratch ? a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K : blkC + kMaxBlk * kTThreads;
+    double *P = pstar + K;
+    const int E = (K + kTThreads - 1) / kTThreads;
+    if (lane == 0) {
+        mbar_init(&mbar[0][warp], 1);
+        mbar_init(&mbar[1][warp], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    __syncthreads();
+    uint32_t parity[2] = {0u, 0u};
+    int cur_word = -1;
+
+    for (;;) {
+        if (tid == 0) s_ci = static_cast<int>(atomicAdd(a.counter, 1u));
+        __syncthreads();
+        const int ci = s_ci;
+        if (ci >= a.n_chunks) break;
+        const SampleChunk ch = a.chunks[ci];
+        const int32_t *nwk_row = a.nwk + static_cast<size_t>(ch.word) * K;
+
+        if (static_cast<int>(ch.word) != cur_word) {
+            // p*(k) = (n_wk + β)/(n_k + Vβ) and the inclusive prefix of α·p*(k) (Eq. 8)
+            const int kb = tid * E;
+            double run = 0.0;
+            for (int e = 0; e < E; ++e) {
+                const int k = kb + e;
+                if (k < K) {
+                    const double ps = (static_cast<double>(__ldg(nwk_row + k)) + a.beta) / __ldg(a.denom + k);
+                    pstar[k] = ps;
+                    run = run + a.alpha * ps;
+                    P[k] = run;
+                }
+            }
+            double incl = run;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const double y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            double lex = __shfl_up_sync(kFull, incl, 1);
+            if (lane == 0) lex = 0.0;
+            if (lane == 31) s_wtot[warp] = incl;
+            __syncthreads();
+            double off = 0.0;
+            for (int i = 0; i < warp; ++i) off += s_wtot[i];
+            off = off + lex;
+            for (int e = 0; e < E; ++e) {
+                const int k = kb + e;
+                if (k < K) P[k] = off + P[k];
+            }
+            __syncthreads();
+            cur_word = static_cast<int>(ch.word);
+        }
+        const double Q = P[K - 1];
+
+        // this warp's batches: tokens j = (i*kTW + warp)*32 + lane
+        uint32_t sg = ch.seg0;
+        auto load_header = [&](uint32_t i, TBatch &B) {
+            const uint32_t j = (i * kTW + warp) * 32u + lane;
+            B.valid = j < ch.count;
+            B.h0 = make_uint4(0u, 0u, 0u, 0u);
+            B.h1 = B.h0;
+            if (B.valid) {
+                B.p = run_position(a.segs, sg, ch.vbegin + j);
+                B.row = __ldg(a.tok_row + B.p);
+                const uint4 *r = a.rows + static_cast<size_t>(B.row) * 2;
+                B.h0 = ld_nc_v4(r);
+                B.h1 = ld_nc_v4(r + 1);
+            }
+        };
+        auto issue_body = [&](int s, TBatch &B) {
+            const uint32_t nblk = B.valid ? ((B.h0.x + 8u) >> 3) : 0u;
+            const uint32_t need = nblk ? nblk - 1u : 0u;
+            uint32_t incl = need;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            const uint32_t total = __shfl_sync(kFull, incl, 31);
+            B.off = incl - need;
+            B.nst = B.off >= static_cast<uint32_t>(kTCap) ? 0u : min(need, kTCap - B.off);
+            const uint32_t staged = min(total, static_cast<uint32_t>(kTCap));
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) mbar_arrive_expect_tx(&mbar[s][warp], staged * 32u);
+            __syncwarp();
+            if (B.nst) {
+                uint4 *dst = stage0 + (static_cast<size_t>(s) * kTW + warp) * kTCap * 2 + B.off * 2;
+                tma_row_to_smem(dst, a.rows + static_cast<size_t>(B.row) * 2 + 2, B.nst * 32u, &mbar[s][warp]);
+            }
+        };
+
+        const uint32_t nb = ch.count > static_cast<uint32_t>(warp) * 32u
+                                ? (ch.count - warp * 32u + kTW * 32u - 1u) / (kTW * 32u)
+                                : 0u;
+        TBatch Bc, Bn, Bnn;
+        if (nb > 0) {
+            load_header(0, Bc);
+            issue_body(0, Bc);
+            if (nb > 1) load_header(1, Bn);
+        }
+        for (uint32_t i = 0; i < nb; ++i) {
+            const int s = static_cast<int>(i & 1u);
+            if (i + 1 < nb) issue_body(s ^ 1, Bn);
+            if (i + 2 < nb) load_header(i + 2, Bnn);
+            mbar_wait(&mbar[s][warp], parity[s]);
+            parity[s] ^= 1u;
+
+            if (Bc.valid) {
+                const uint4 *stg = stage0 + (static_cast<size_t>(s) * kTW + warp) * kTCap * 2 + Bc.off * 2;
+                const uint4 *gr = a.rows + static_cast<size_t>(Bc.row) * 2;
+                const uint32_t j = (i * kTW + warp) * 32u + lane;
+                const uint32_t x0 = philox_x0_sched(ch.c_base + j, a.t, a.key0, a.key1);
+                int zo = 0;
+                double po_new = 0.0, delta = 0.0;
+                if (EXCL) {
+                    zo = static_cast<int>(a.z[Bc.p]);
+                    po_new = (static_cast<double>(nwk_row[zo] - 1) + a.beta) /
+                             (static_cast<double>(a.nk[zo] - 1) + a.Vbeta);
+                    delta = a.alpha * po_new - a.alpha * pstar[zo];
+                }
+                const uint32_t len = Bc.h0.x;
+                const uint32_t nblk = (len + 8u) >> 3;
+                // block b >= 1 of the row: staged copy, or global memory past the stage
+#define LDA_BLOCK(b, u0, u1)                                                     \
+    if ((b) <= Bc.nst) {                                                         \
+        u0 = stg[2 * ((b) - 1)];                                                 \
+        u1 = stg[2 * ((b) - 1) + 1];                                             \
+    } else {                                                                     \
+        u0 = ld_nc_v4(gr + 2 * (b));                                             \
+        u1 = ld_nc_v4(gr + 2 * (b) + 1);                                         \
+    }
+                double S = 0.0;
+                S = Mass<EXCL>::fma_into(Bc.h0.y, pstar, zo, po_new, S);
+                S = Mass<EXCL>::fma_into(Bc.h0.z, pstar, zo, po_new, S);
+                S = Mass<EXCL>::fma_into(Bc.h0.w, pstar, zo, po_new, S);
+                S = Mass<EXCL>::fma_into(Bc.h1.x, pstar, zo, po_new, S);
+                S = Mass<EXCL>::fma_into(Bc.h1.y, pstar, zo, po_new, S);
+                S = Mass<EXCL>::fma_into(Bc.h1.z, pstar, zo, po_new, S);
+                S = Mass<EXCL>::fma_into(Bc.h1.w, pstar, zo, po_new, S);
+                blkC[tid] = S;
+                for (uint32_t b = 1; b < nblk; ++b) {
+                    uint4 u0, u1;
+                    LDA_BLOCK(b, u0, u1)
+                    S = Mass<EXCL>::fma_into(u0.x, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u0.y, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u0.z, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u0.w, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u1.x, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u1.y, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u1.z, pstar, zo, po_new, S);
+                    S = Mass<EXCL>::fma_into(u1.w, pstar, zo, po_new, S);
+                    if (b < kMaxBlk) blkC[b * kTThreads + tid] = S;
+                }
+                const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;  // x0 · 2^-32
+                const double x = U * (S + (EXCL ? Q + delta : Q));
+                int z;
+                if (x < S) {
+                    const uint32_t nbk = nblk < kMaxBlk ? nblk : kMaxBlk;
+                    uint32_t b = 0;
+                    while (b < nbk && !(blkC[b * kTThreads + tid] > x)) ++b;
+                    double C = b == 0 ? 0.0 : blkC[(b - 1) * kTThreads + tid];
+                    z = -1;
+#define LDA_STEP(e)                                                   \
+    {                                                                 \
+        C = Mass<EXCL>::fma_into((e), pstar, zo, po_new, C);          \
+        if (z < 0 && C > x) z = static_cast<int>((e) >> 16);          \
+    }
+                    if (b == 0) {
+                        LDA_STEP(Bc.h0.y) LDA_STEP(Bc.h0.z) LDA_STEP(Bc.h0.w)
+                        LDA_STEP(Bc.h1.x) LDA_STEP(Bc.h1.y) LDA_STEP(Bc.h1.z) LDA_STEP(Bc.h1.w)
+                        b = 1;
+                    }
+                    for (; z < 0 && b < nblk; ++b) {
+                        uint4 u0, u1;
+                        LDA_BLOCK(b, u0, u1)
+                        LDA_STEP(u0.x) LDA_STEP(u0.y) LDA_STEP(u0.z) LDA_STEP(u0.w)
+                        LDA_STEP(u1.x) LDA_STEP(u1.y) LDA_STEP(u1.z) LDA_STEP(u1.w)
+                    }
+#undef LDA_STEP
+                    if (z < 0) z = K - 1;  // unreachable: the last entry's prefix is S > x
+                } else {
+                    int lo = 0, hi = K - 1;
+                    while (lo < hi) {
+                        const int mid = (lo + hi) >> 1;
+                        double pk = P[mid];
+                        if (EXCL && mid >= zo) pk += delta;
+                        if (S + pk > x) hi = mid;
+                        else lo = mid + 1;
+                    }
+                    z = lo;
+                }
+#undef LDA_BLOCK
+                a.z[Bc.p] = static_cast<uint16_t>(z);
+            }
+            __syncwarp();
+            Bc = Bn;
+            Bn = Bnn;
         }
         __syncthreads();
     }
@@ -333,9 +605,9 @@ __global__ void zero_rows_kernel(const int32_t *__restrict__ words, int64_t n, i
 }
 
 __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc,
-                               const uint32_t *__restrict__ tseg, int ntiles, int V, int K,
-                               const uint16_t *__restrict__ z, int32_t *__restrict__ nwk,
-                               int32_t *__restrict__ nk, uint32_t *__restrict__ counter) {
+                               const Seg *__restrict__ segs, int K, const uint16_t *__restrict__ z,
+                               int32_t *__restrict__ nwk, int32_t *__restrict__ nk,
+                               uint32_t *__restrict__ counter) {
     extern __shared__ int smem_i[];
     int *hist = smem_i, *nkp = smem_i + K;
     __shared__ int s_ci;
@@ -347,21 +619,16 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
         const int ci = s_ci;
         if (ci >= n_rc) break;
         const RecountChunk c = rc[ci];
-        const uint32_t vb = c.vbegin, ve = c.vbegin + c.vcount;
-        uint32_t acc = 0;
-        for (int b = 0; b < ntiles && acc < ve; ++b) {
-            const size_t key = static_cast<size_t>(b) * V + c.word;
-            const uint32_t s = tseg[key], n = tseg[key + 1] - s;
-            const uint32_t lo = max(vb, acc), hi = min(ve, acc + n);
-            for (uint32_t vv = lo + threadIdx.x; vv < hi; vv += blockDim.x)
-                atomicAdd(&hist[z[s + (vv - acc)]], 1);
-            acc += n;
-        }
+        const uint32_t w = c.word & 0x7FFFFFFFu;
+        const bool split = (c.word >> 31) != 0u;
+        uint32_t sg = c.seg0;
+        for (uint32_t j = threadIdx.x; j < c.vcount; j += blockDim.x)
+            atomicAdd(&hist[z[run_position(segs, sg, c.vbegin + j)]], 1);
         __syncthreads();
-        int32_t *row = nwk + static_cast<size_t>(c.word) * K;
+        int32_t *row = nwk + static_cast<size_t>(w) * K;
         for (int k = threadIdx.x; k < K; k += blockDim.x) {
             const int h = hist[k];
-            if (c.split) {
+            if (split) {
                 if (h) atomicAdd(row + k, h);
             } else {
                 row[k] = h;
@@ -381,7 +648,26 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
 // as ascending (topic << 16 | count) entries with a popc scan over the bitmap.
 // O(L_d + K/32) per document instead of the paper's dense O(K) row.
 // ---------------------------------------------------------------------------
-__global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off16,
+// Two-phase variant, phase A: z in document order, zd[i] = z[doc_map[i]]
+// (independent gathers with high memory-level parallelism, in doc order).
+__global__ void gather_z_kernel(const uint32_t *__restrict__ doc_map, const uint16_t *__restrict__ z,
+                                uint16_t *__restrict__ zd, int64_t T) {
+    const int64_t i0 = (static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x) * 4;
+    if (i0 + 3 < T) {
+        const uint4 m = __ldcs(reinterpret_cast<const uint4 *>(doc_map + i0));
+        const uint16_t a = z[m.x], b = z[m.y], c = z[m.z], d = z[m.w];
+        ushort4 o;
+        o.x = a; o.y = b; o.z = c; o.w = d;
+        *reinterpret_cast<ushort4 *>(zd + i0) = o;
+    } else {
+        for (int64_t i = i0; i < T; ++i) zd[i] = z[doc_map[i]];
+    }
+}
+
+// GATHERED = false: z through the doc-word map (fused); true: zd is z in
+// document order (phase B of the two-phase variant).
+template <bool GATHERED>
+__global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
                              const uint32_t *__restrict__ doc_map, const uint16_t *__restrict__ z,
                              uint32_t *__restrict__ rows, int64_t D, int K,
                              unsigned long long *__restrict__ stat) {
@@ -397,12 +683,12 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
     for (int64_t d = static_cast<int64_t>(blockIdx.x) * wpb + warp; d < D; d += nw) {
         const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1];
         for (uint32_t i = s + lane; i < e; i += 32) {
-            const uint32_t k = z[doc_map[i]];
+            const uint32_t k = GATHERED ? z[i] : z[doc_map[i]];
             atomicAdd(&cnt[k], 1u);
             atomicOr(&bits[k >> 5], 1u << (k & 31));
         }
         __syncwarp();
-        uint32_t *row = rows + static_cast<size_t>(row_off16[d]) * 4;
+        uint32_t *row = rows + static_cast<size_t>(row_off32[d]) * 8;
         uint32_t base = 0;
         for (int qb = 0; qb < Kw; qb += 32) {
             const int qq = qb + lane;
@@ -425,6 +711,9 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
             if (qq < Kw) bits[qq] = 0u;
             base += __shfl_sync(kFull, incl, 31);
         }
+        // zero the words after the last entry up to the 32-byte boundary
+        const uint32_t pad = (8u - ((1u + base) & 7u)) & 7u;
+        if (static_cast<uint32_t>(lane) < pad) row[1 + base + lane] = 0u;
         if (lane == 0) {
             row[0] = base;
             s_nnz += base;
@@ -467,7 +756,7 @@ __global__ void ll_word_kernel(const int32_t *__restrict__ nwk, int64_t n, doubl
     if (threadIdx.x == 0) part[blockIdx.x] = t;
 }
 
-__global__ void ll_doc_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off16,
+__global__ void ll_doc_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
                               const uint32_t *__restrict__ rows, int64_t D, double alpha, double lga,
                               double Kalpha, double lgKa, double *__restrict__ part) {
     __shared__ double sh[32];
@@ -475,7 +764,7 @@ __global__ void ll_doc_kernel(const uint32_t *__restrict__ doc_ptr32, const uint
     double s = 0.0;
     const int64_t nw = static_cast<int64_t>(gridDim.x) * wpb;
     for (int64_t d = static_cast<int64_t>(blockIdx.x) * wpb + warp; d < D; d += nw) {
-        const uint32_t *row = rows + static_cast<size_t>(row_off16[d]) * 4;
+        const uint32_t *row = rows + static_cast<size_t>(row_off32[d]) * 8;
         const uint32_t nnz = row[0];
         if (lane == 0) s += lgKa - lgamma(static_cast<double>(doc_ptr32[d + 1] - doc_ptr32[d]) + Kalpha);
         for (uint32_t j = lane; j < nnz; j += 32)
@@ -507,14 +796,6 @@ __global__ void ll_final_kernel(const double *__restrict__ part_w, int nw, const
 // ---------------------------------------------------------------------------
 // Launchers
 // ---------------------------------------------------------------------------
-static constexpr int kGS = 8;  // lanes per token in the sampler
-
-static int top_step_for(int K) {
-    int step = 1;
-    while (static_cast<int64_t>(step) * 32 < K) step *= 32;
-    return step;
-}
-
 int configure_kernels(DevState &s) {
     cudaError_t e;
     int dev = 0;
@@ -524,20 +805,40 @@ int configure_kernels(DevState &s) {
     if ((e = cudaDeviceGetAttribute(&max_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev)) != cudaSuccess)
         return e;
     // sampler
-    size_t want = static_cast<size_t>(16) * s.K;
-    s.sweep_smem = (want + 2048 <= static_cast<size_t>(max_optin)) ? want : 0;
-    const void *fns[2] = {reinterpret_cast<const void *>(&sweep_kernel<kGS, false>),
-                          reinterpret_cast<const void *>(&sweep_kernel<kGS, true>)};
-    int bps = 1;
-    for (int i = 0; i < 2; ++i) {
-        if ((e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      static_cast<int>(s.sweep_smem))) != cudaSuccess)
+    if (s.sampler == 1) {
+        const size_t fixed = 2 * kTW * kTCap * 32 + sizeof(double) * kMaxBlk * kTThreads;
+        const size_t want = fixed + static_cast<size_t>(16) * s.K;
+        s.sweep_smem = (want + 2048 <= static_cast<size_t>(max_optin)) ? want : fixed;
+        s.sweep_block = kTThreads;
+        const void *fns[2] = {reinterpret_cast<const void *>(&sweep_tma_kernel<false>),
+                              reinterpret_cast<const void *>(&sweep_tma_kernel<true>)};
+        for (int i = 0; i < 2; ++i)
+            if ((e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          static_cast<int>(s.sweep_smem))) != cudaSuccess)
+                return e;
+        int bps = 1;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fns[s.exclude_self ? 1 : 0], kTThreads,
+                                                               s.sweep_smem)) != cudaSuccess)
             return e;
+        s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
+    } else {
+        const size_t blk = sizeof(double) * kMaxBlk * kSweepThreads;
+        size_t want = blk + static_cast<size_t>(16) * s.K;
+        s.sweep_smem = (want + 2048 <= static_cast<size_t>(max_optin)) ? want : blk;
+        s.sweep_block = kSweepThreads;
+        const void *fns[2] = {reinterpret_cast<const void *>(&sweep_kernel<false>),
+                              reinterpret_cast<const void *>(&sweep_kernel<true>)};
+        int bps = 1;
+        for (int i = 0; i < 2; ++i) {
+            if ((e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          static_cast<int>(s.sweep_smem))) != cudaSuccess)
+                return e;
+        }
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fns[s.exclude_self ? 1 : 0], kSweepThreads,
+                                                               s.sweep_smem)) != cudaSuccess)
+            return e;
+        s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
     }
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fns[s.exclude_self ? 1 : 0], kSweepThreads,
-                                                           s.sweep_smem)) != cudaSuccess)
-        return e;
-    s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
     // recount
     if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&recount_kernel),
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) != cudaSuccess)
@@ -548,12 +849,16 @@ int configure_kernels(DevState &s) {
     if (wpb < 1) return cudaErrorInvalidValue;
     s.theta_block = 32 * wpb;
     s.theta_smem = per_warp * wpb;
-    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel),
+    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel<true>),
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  static_cast<int>(s.theta_smem))) != cudaSuccess)
+        return e;
+    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel<false>),
                                   cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   static_cast<int>(s.theta_smem))) != cudaSuccess)
         return e;
     int tb = 1;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, reinterpret_cast<const void *>(&theta_kernel),
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, reinterpret_cast<const void *>(&theta_kernel<false>),
                                                            s.theta_block, s.theta_smem)) != cudaSuccess)
         return e;
     s.theta_grid = s.num_sms * (tb > 0 ? tb : 1);
@@ -564,7 +869,7 @@ int configure_kernels(DevState &s) {
 int launch_init(const DevState &s, void *stream) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const int grid = static_cast<int>(std::min<int64_t>(s.n_chunks > 0 ? s.n_chunks : 1, 65535));
-    init_kernel<<<grid, 256, 0, st>>>(s.chunks, s.n_chunks, s.tok_z, static_cast<uint32_t>(s.K),
+    init_kernel<<<grid, 256, 0, st>>>(s.chunks, s.n_chunks, s.segs, s.tok_z, static_cast<uint32_t>(s.K),
                                       static_cast<uint32_t>(s.seed), static_cast<uint32_t>(s.seed >> 32));
     return cudaGetLastError();
 }
@@ -581,7 +886,7 @@ int launch_recount(const DevState &s, void *stream, int *launches) {
         ++*launches;
     }
     recount_kernel<<<s.sweep_grid > 0 ? s.num_sms * 4 : 1, 256, 8 * s.K, st>>>(
-        s.rchunks, s.n_rchunks, s.tseg, s.ntiles, s.V, s.K, s.tok_z, s.nwk, nk, s.counter + 1);
+        s.rchunks, s.n_rchunks, s.segs, s.K, s.tok_z, s.nwk, nk, s.counter + 1);
     ++*launches;
     return cudaGetLastError();
 }
@@ -590,8 +895,16 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     if ((e = cudaMemsetAsync(stat_out, 0, 2 * sizeof(unsigned long long), st)) != cudaSuccess) return e;
-    theta_kernel<<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off16, s.doc_map,
-                                                                     s.tok_z, s.rows, s.D, s.K, stat_out);
+    if (s.z_doc) {
+        const int64_t thr = (s.T + 3) / 4;
+        gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, st>>>(s.doc_map, s.tok_z, s.z_doc, s.T);
+        ++*launches;
+        theta_kernel<true><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.doc_map,
+                                                                           s.z_doc, s.rows, s.D, s.K, stat_out);
+    } else {
+        theta_kernel<false><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.doc_map,
+                                                                            s.tok_z, s.rows, s.D, s.K, stat_out);
+    }
     ++*launches;
     return cudaGetLastError();
 }
@@ -601,32 +914,44 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
     cudaError_t e;
     const double Vbeta = static_cast<double>(s.V) * s.beta;
     const int32_t *nk = s.nwk + static_cast<size_t>(s.V) * s.K;
-    prologue_kernel<<<(s.K + 255) / 256, 256, 0, st>>>(nk, s.K, Vbeta, s.invk);
+    prologue_kernel<<<(s.K + 255) / 256, 256, 0, st>>>(nk, s.K, Vbeta, s.denom);
     ++*launches;
     if ((e = cudaMemsetAsync(s.counter, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
     SweepArgs a;
     a.chunks = s.chunks;
     a.n_chunks = s.n_chunks;
+    a.segs = s.segs;
     a.tok_row = s.tok_row;
     a.z = s.tok_z;
     a.rows = reinterpret_cast<const uint4 *>(s.rows);
     a.nwk = s.nwk;
     a.nk = nk;
-    a.invk = s.invk;
+    a.denom = s.denom;
     a.counter = s.counter;
-    a.gscratch = s.sweep_smem ? nullptr : s.sweep_scratch;  // large-K fallback
+    a.gscratch = s.sweep_scratch;  // non-null only when p*/P do not fit in smem
     a.K = s.K;
-    a.top_step = top_step_for(s.K);
     a.alpha = s.alpha;
     a.beta = s.beta;
     a.Vbeta = Vbeta;
     a.t = t;
-    a.k0 = static_cast<uint32_t>(s.seed);
-    a.k1 = static_cast<uint32_t>(s.seed >> 32);
-    if (s.exclude_self)
-        sweep_kernel<kGS, true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
-    else
-        sweep_kernel<kGS, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+    uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
+    for (int r = 0; r < 10; ++r) {
+        a.key0[r] = k0;
+        a.key1[r] = k1;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+    if (s.sampler == 1) {
+        if (s.exclude_self)
+            sweep_tma_kernel<true><<<s.sweep_grid, kTThreads, s.sweep_smem, st>>>(a);
+        else
+            sweep_tma_kernel<false><<<s.sweep_grid, kTThreads, s.sweep_smem, st>>>(a);
+    } else {
+        if (s.exclude_self)
+            sweep_kernel<true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        else
+            sweep_kernel<false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+    }
     ++*launches;
     return cudaGetLastError();
 }
@@ -642,7 +967,7 @@ int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches
         nw = s.ll_blocks;
         ++*launches;
     }
-    ll_doc_kernel<<<s.ll_blocks, 256, 0, st>>>(s.doc_ptr32, s.row_off16, s.rows, s.D, s.alpha, lgamma(s.alpha),
+    ll_doc_kernel<<<s.ll_blocks, 256, 0, st>>>(s.doc_ptr32, s.row_off32, s.rows, s.D, s.alpha, lgamma(s.alpha),
                                                Kalpha, lgamma(Kalpha), pd);
     ++*launches;
     ll_final_kernel<<<1, 256, 0, st>>>(pw, nw, pd, s.ll_blocks, s.nwk + static_cast<size_t>(s.V) * s.K, s.K,

@@ -8,25 +8,36 @@
 
 namespace lda {
 
-// One sampling work item: a run of tokens of one word inside one doc tile
-// (word-first order, L1189-1191; heavy words split over several items,
-// L1203-1221).  c_base = canonical index (X18) of the item's first token.
+// A run of word w's tokens inside one document tile.  Word w's local tokens
+// have "virtual" indices 0..n_w-1 in (doc, position) order, i.e. canonical
+// order (X18) restricted to this rank; the run stores virtual indices
+// [vstart, next.vstart) at word-major positions pos, pos+1, ...  Each word's
+// runs are followed by a sentinel {0, n_w}.
+struct Seg {
+    uint32_t pos;
+    uint32_t vstart;
+};
+
+// One sampling work item: tokens [vbegin, vbegin+count) of one word (the
+// word-first order of L1189-1191; heavy words split over several items,
+// L1203-1221).  seg0 = index of the run holding vbegin; c_base = canonical
+// index of virtual index vbegin.
 struct SampleChunk {
-    uint32_t begin;   // first word-major position
-    uint32_t count;   // tokens
     uint32_t word;
-    uint32_t pad;
+    uint32_t vbegin;
+    uint32_t count;
+    uint32_t seg0;
     uint64_t c_base;
 };
 
-// One n_wk-recount work item: tokens [vbegin, vbegin+vcount) of word `word`
-// counted across its per-tile segments.  split != 0 when the word has more
-// than one item (its row is zeroed first and accumulated atomically).
+// One n_wk-recount work item: virtual indices [vbegin, vbegin+vcount) of word
+// (word & 0x7fffffff); bit 31 set when the word has more than one item (its
+// row is then zeroed first and accumulated atomically).
 struct RecountChunk {
     uint32_t word;
     uint32_t vbegin;
     uint32_t vcount;
-    uint32_t split;
+    uint32_t seg0;
 };
 
 // Host-side layout of one rank's shard (built by build_layout).
@@ -35,11 +46,11 @@ struct HostLayout {
     int32_t V = 0, K = 0;
     int32_t ntiles = 1;
     std::vector<uint32_t> doc_ptr32;   // D+1 doc-major token offsets
-    std::vector<uint32_t> row_off16;   // D   θ row start, in 16-byte units
-    uint64_t rows16 = 0;               // θ row buffer size in 16-byte units (incl. tail pad)
-    std::vector<uint32_t> tok_row;     // T   word-major: θ row (16 B units) of the token's doc
+    std::vector<uint32_t> row_off32;   // D   θ row start, in 32-byte units
+    uint64_t rows32 = 0;               // θ row buffer size in 32-byte units (incl. tail pad)
+    std::vector<uint32_t> tok_row;     // T   word-major: θ row (32 B units) of the token's doc
     std::vector<uint32_t> doc_map;     // T   doc-major token i -> word-major position (S7, L1297-1303)
-    std::vector<uint32_t> tseg;        // ntiles*V+1 segment starts, key = tile*V + word
+    std::vector<Seg> segs;             // per word: its runs, then a sentinel
     std::vector<SampleChunk> chunks;   // heavy-first
     std::vector<RecountChunk> rchunks; // heavy-first
     std::vector<int32_t> split_words;  // words whose row is accumulated atomically
@@ -70,13 +81,15 @@ struct DevState {
     double alpha = 0, beta = 0;
     uint64_t seed = 0;
     int exclude_self = 0;
+    int sampler = 1;                // 1 = TMA-staged rows (default), 0 = direct loads
     // corpus
     uint32_t *tok_row = nullptr;    // T
     uint16_t *tok_z = nullptr;      // T (word-major)
     uint32_t *doc_map = nullptr;    // T
+    uint16_t *z_doc = nullptr;      // T, z in document order (two-phase θ rebuild only)
     uint32_t *doc_ptr32 = nullptr;  // D+1
-    uint32_t *row_off16 = nullptr;  // D
-    uint32_t *tseg = nullptr;       // ntiles*V+1
+    uint32_t *row_off32 = nullptr;  // D
+    Seg *segs = nullptr;
     SampleChunk *chunks = nullptr;
     int64_t n_chunks = 0;
     RecountChunk *rchunks = nullptr;
@@ -84,9 +97,9 @@ struct DevState {
     int32_t *split_words = nullptr;
     int64_t n_split = 0;
     // model
-    uint32_t *rows = nullptr;       // θ rows, rows16*4 words
+    uint32_t *rows = nullptr;       // θ rows, rows32*8 words
     int32_t *nwk = nullptr;         // V*K + K (n_k at offset V*K)
-    double *invk = nullptr;         // K
+    double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch
     uint32_t *counter = nullptr;    // work counters [4]
     unsigned long long *stat = nullptr;  // [4]: Σ L_d nnz_d, Σ nnz_d
@@ -94,7 +107,7 @@ struct DevState {
     double *ll_out = nullptr;       // [2]
     double *sweep_scratch = nullptr;  // sweep_grid*2*K when K does not fit in smem
     int num_sms = 148;
-    int sweep_grid = 0;
+    int sweep_grid = 0, sweep_block = 0;
     int theta_grid = 0, theta_block = 0;
     size_t sweep_smem = 0, theta_smem = 0;
     int ll_blocks = 0;

@@ -108,7 +108,8 @@ def test_nytimes_shaped_midsize_many_chunks():
     assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * cfg.T * 3
     z_ref = g.z()
     for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
-                 dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3)]:
+                 dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3),
+                 dict(theta_mode=1), dict(sampler=0), dict(sampler=0, tile_tokens=20_000)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
@@ -119,9 +120,11 @@ def test_exclude_self_lockstep():
     doc_ptr, words = _corpus(500, 300, 30_000, 0.5, 16, 13)
     K = 24
     o = U.oracle_for(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3)
-    g = U.gpu_model(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3, exclude_self=1)
-    bad, unexc = U.lockstep(g, o, 3, exclude_self=1)
-    assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
+    for sampler in (1, 0):
+        o = U.oracle_for(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3)
+        g = U.gpu_model(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3, exclude_self=1, sampler=sampler)
+        bad, unexc = U.lockstep(g, o, 3, exclude_self=1)
+        assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
 def test_edge_cases():
