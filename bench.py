@@ -263,9 +263,8 @@ def run_b200(args):
     b_sample = sum(C.bytes_sample(T_g, cfg.V, cfg.K, int(n)) for n in log["sum_nnz_tok"])
     t_sample = float(np.sum(log["ms_sample"])) / 1e3
     achieved = b_sample / t_sample / 1e9
-    nnz_next = list(log["sum_nnz_tok"][1:]) + [int(st["sum_nnz_tok"])]
     b_sweep = sum(C.bytes_sweep(T_g, D_g, cfg.V, cfg.K, int(a), int(b)) for a, b in
-                  zip(log["sum_nnz_tok"], nnz_next))
+                  zip(log["sum_nnz_tok"], log["sum_nnz_doc"]))
     sweep_gbs = b_sweep / (float(np.sum(log["ms_sweep"])) / 1e3) / 1e9
     traffic = None
     try:

@@ -93,6 +93,9 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tile_tokens"   split the documents into tiles of about this many tokens
  *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
+ *   "filter32"      1: draw each token in fp32 first and redo it in fp64 when
+ *                   its uniform lies within the fp32 error bound of a CDF
+ *                   boundary — results identical to 0 (always fp64, default)
  *   "theta_mode"    θ rebuild: 0 = fused gather+histogram (default),
  *                   1 = two-phase (z gathered into document order first)
  * Results do not depend on chunk_tokens, recount_tokens, tile_tokens or
@@ -118,6 +121,17 @@ int lda_nccl_unique_id(void *out128);
  * doc_ptr: D+1 non-decreasing offsets (doc_ptr[0] == 0, T = doc_ptr[D]);
  * doc_begin: world+1 outputs.  Host-only.  Errors: LDA_EINVAL. */
 int lda_partition_docs(int64_t D, const int64_t *doc_ptr, int32_t world, int64_t *doc_begin);
+
+/* Canonical-index bases for a rank (host-only; lda_load_corpus uses it).
+ * The canonical index of a token is its position in the stable sort of the
+ * whole corpus by (word, document, position) (X18; the paper's word-first
+ * order, L1189-1191).  With documents partitioned into contiguous rank
+ * ranges, rank g's tokens of word w are one contiguous run of that order,
+ * starting at cbase[w] = Σ_{w'<w} T(w') + Σ_{g'<g} T_{g'}(w).
+ *   word_counts: world*V per-rank word histograms, rank-major
+ *   cbase: V outputs; total (may be NULL): T = Σ of all counts. */
+int lda_canonical_bases(int32_t V, int32_t world, int32_t rank, const int64_t *word_counts, int64_t *cbase,
+                        int64_t *total);
 
 /* Load this rank's documents [doc_begin, doc_end) of the global corpus,
  * randomly initialise every token's topic (L377-379; Philox at t = 0, X10)
@@ -161,9 +175,11 @@ int lda_get_stats(lda_ctx *ctx, lda_stats *out);
 
 /* Per-sweep log of the last lda_iterate call: up to `cap` entries of each
  * non-NULL array (device ms per sweep and per phase; Σ_t nnz_{d(t)} of the θ
- * each sweep sampled against).  *n_out = number of sweeps in that call. */
+ * each sweep sampled against; Σ_d nnz_d of the θ each sweep rebuilt).
+ * *n_out = number of sweeps in that call. */
 int lda_get_sweep_log(lda_ctx *ctx, int32_t cap, double *ms_sweep, double *ms_sample, double *ms_recount,
-                      double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int32_t *n_out);
+                      double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int64_t *sum_nnz_doc,
+                      int32_t *n_out);
 
 /* The CUDA stream (cudaStream_t) the sweep kernels run on; valid after
  * lda_load_corpus until lda_destroy. */

@@ -299,6 +299,30 @@ int32_t orc_draw(int32_t K, int32_t V, double alpha, double beta,
  * start of the sweep, then all counts are rebuilt from the new z.
  * z (input order) and the counts are updated in place; t >= 1 is the global
  * sweep number (Philox counter word 2). */
+/* The draws of one sweep for the tokens of documents [d_begin, d_end) only,
+ * against the given (frozen, global) counts; z_new receives their new topics
+ * (input order, indexed like z).  A partition of the documents across ranks
+ * draws exactly what one process draws (the multi-GPU decomposition, Eq. 4
+ * L935-937: each rank samples its documents against the same replicated ϕ). */
+void orc_draw_docs(int64_t d_begin, int64_t d_end, int32_t V, int32_t K, double alpha,
+                   double beta, const int64_t *doc_ptr, const int32_t *words,
+                   const int64_t *canon, uint64_t seed, uint32_t t, int exclude_self,
+                   const uint16_t *z, const int32_t *n_wk, const int32_t *n_k,
+                   const int32_t *n_dk /* dense D*K, global doc index */,
+                   uint16_t *z_new, double *margin)
+{
+    for (int64_t d = d_begin; d < d_end; d++) {
+        for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; i++) {
+            int32_t w = words[i];
+            uint32_t x0 = orc_token_x0(seed, (uint64_t)canon[i], t);
+            double m;
+            z_new[i] = (uint16_t)orc_draw(K, V, alpha, beta, n_wk + (int64_t)w * K,
+                                          n_k, n_dk + d * K, exclude_self, z[i], x0, &m);
+            if (margin) margin[i] = m;
+        }
+    }
+}
+
 void orc_sweep(int64_t D, int32_t V, int32_t K, double alpha, double beta,
                const int64_t *doc_ptr, const int32_t *words, const int64_t *canon,
                uint64_t seed, uint32_t t, int exclude_self, uint16_t *z,
@@ -306,17 +330,8 @@ void orc_sweep(int64_t D, int32_t V, int32_t K, double alpha, double beta,
 {
     int64_t T = doc_ptr[D];
     uint16_t *z_new = (uint16_t *)malloc(sizeof(uint16_t) * (size_t)(T > 0 ? T : 1));
-    for (int64_t d = 0; d < D; d++) {
-        for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; i++) {
-            int32_t w = words[i];
-            uint32_t x0 = orc_token_x0(seed, (uint64_t)canon[i], t);
-            double m;
-            z_new[i] = (uint16_t)orc_draw(K, V, alpha, beta, n_wk + (int64_t)w * K,
-                                          n_k, n_dk + d * K, exclude_self, z[i],
-                                          x0, &m);
-            if (margin) margin[i] = m;
-        }
-    }
+    orc_draw_docs(0, D, V, K, alpha, beta, doc_ptr, words, canon, seed, t, exclude_self, z,
+                  n_wk, n_k, n_dk, z_new, margin);
     memcpy(z, z_new, sizeof(uint16_t) * (size_t)T);
     free(z_new);
     orc_counts(D, V, K, doc_ptr, words, z, n_wk, n_k, n_dk);

@@ -73,6 +73,10 @@ def lib():
                                 _i64p, _i32p, _i64p, c.c_uint64, c.c_uint32, c.c_int,
                                 _u16p, _i32p, _i32p, _i32p, c.c_void_p]
         L.orc_sweep.restype = None
+        L.orc_draw_docs.argtypes = [c.c_int64, c.c_int64, c.c_int32, c.c_int32, c.c_double,
+                                    c.c_double, _i64p, _i32p, _i64p, c.c_uint64, c.c_uint32,
+                                    c.c_int, _u16p, _i32p, _i32p, _i32p, _u16p, c.c_void_p]
+        L.orc_draw_docs.restype = None
         L.orc_sweep_sequential.argtypes = [c.c_int64, c.c_int32, c.c_int32, c.c_double,
                                            c.c_double, _i64p, _i32p, _i64p, c.c_uint64,
                                            c.c_uint32, _u16p, _i32p, _i32p, _i32p]
@@ -152,6 +156,20 @@ def draw(K, V, alpha, beta, nwk_row, n_k, ndk_row, x0, exclude_self=0, z_old=-1)
                        np.ascontiguousarray(ndk_row, np.int32), exclude_self, z_old,
                        x0, ctypes.byref(m))
     return int(z), m.value
+
+
+def draw_docs(d_begin, d_end, doc_ptr, words, canon, V, K, alpha, beta, seed, t, z, n_wk, n_k,
+              n_dk, exclude_self=0):
+    """New topics of the tokens of documents [d_begin, d_end) against the given
+    global counts (input order; other entries of the result are 0)."""
+    z = np.ascontiguousarray(z, np.uint16)
+    out = np.zeros_like(z)
+    lib().orc_draw_docs(d_begin, d_end, V, K, alpha, beta, np.ascontiguousarray(doc_ptr, np.int64),
+                        np.ascontiguousarray(words, np.int32), np.ascontiguousarray(canon, np.int64),
+                        seed, t, exclude_self, z, np.ascontiguousarray(n_wk, np.int32).reshape(-1),
+                        np.ascontiguousarray(n_k, np.int32), np.ascontiguousarray(n_dk, np.int32).reshape(-1),
+                        out, None)
+    return out
 
 
 def loglik(doc_ptr, V, K, alpha, beta, n_wk, n_k, n_dk):

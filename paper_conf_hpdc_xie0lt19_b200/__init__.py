@@ -24,6 +24,7 @@ STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4:
 
 # every symbol include/lda.h declares
 ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_partition_docs",
+               "lda_canonical_bases",
                "lda_load_corpus", "lda_iterate", "lda_loglik", "lda_get_counts", "lda_get_stats",
                "lda_get_sweep_log", "lda_get_stream", "lda_set_z", "lda_destroy", "lda_last_error",
                "lda_version")
@@ -68,12 +69,13 @@ def lib():
             "lda_init_dist": ([_vp, _i32, _i32, _vp], ctypes.c_int),
             "lda_nccl_unique_id": ([_vp], ctypes.c_int),
             "lda_partition_docs": ([_i64, _vp, _i32, _vp], ctypes.c_int),
+            "lda_canonical_bases": ([_i32, _i32, _i32, _vp, _vp, ctypes.POINTER(_i64)], ctypes.c_int),
             "lda_load_corpus": ([_vp, _i64, _i64, _vp, _vp, _u64], ctypes.c_int),
             "lda_iterate": ([_vp, _i32], ctypes.c_int),
             "lda_loglik": ([_vp, ctypes.POINTER(_f64)], ctypes.c_int),
             "lda_get_counts": ([_vp, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp], ctypes.c_int),
             "lda_get_stats": ([_vp, ctypes.POINTER(lda_stats)], ctypes.c_int),
-            "lda_get_sweep_log": ([_vp, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp], ctypes.c_int),
+            "lda_get_sweep_log": ([_vp, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp], ctypes.c_int),
             "lda_get_stream": ([_vp, ctypes.POINTER(_vp)], ctypes.c_int),
             "lda_set_z": ([_vp, _vp], ctypes.c_int),
             "lda_destroy": ([_vp], None),
@@ -134,6 +136,16 @@ def lda_partition_docs(doc_ptr, world):
     return out
 
 
+def lda_canonical_bases(word_counts, rank):
+    """word_counts: (world, V) int64 per-rank word histograms -> (cbase[V], T)."""
+    wc = np.ascontiguousarray(word_counts, np.int64)
+    world, V = wc.shape
+    out = np.empty(V, np.int64)
+    tot = _i64()
+    _check(lib().lda_canonical_bases(V, world, int(rank), _p(wc), _p(out), ctypes.byref(tot)))
+    return out, tot.value
+
+
 def lda_load_corpus(ctx, doc_begin, doc_end, doc_ptr, words, seed):
     doc_ptr = np.ascontiguousarray(doc_ptr, np.int64)
     words = np.ascontiguousarray(words, np.int32)
@@ -170,13 +182,16 @@ def lda_get_stats(ctx) -> dict:
 
 def lda_get_sweep_log(ctx) -> dict:
     n = _i32()
-    _check(lib().lda_get_sweep_log(ctx, 0, None, None, None, None, None, None, ctypes.byref(n)), ctx)
+    _check(lib().lda_get_sweep_log(ctx, 0, None, None, None, None, None, None, None, ctypes.byref(n)), ctx)
     m = n.value
     arr = {k: np.zeros(m, np.float64) for k in ("ms_sweep", "ms_sample", "ms_recount", "ms_theta", "ms_allreduce")}
     nnz = np.zeros(m, np.int64)
+    nnzd = np.zeros(m, np.int64)
     _check(lib().lda_get_sweep_log(ctx, m, _p(arr["ms_sweep"]), _p(arr["ms_sample"]), _p(arr["ms_recount"]),
-                                   _p(arr["ms_theta"]), _p(arr["ms_allreduce"]), _p(nnz), ctypes.byref(n)), ctx)
+                                   _p(arr["ms_theta"]), _p(arr["ms_allreduce"]), _p(nnz), _p(nnzd),
+                                   ctypes.byref(n)), ctx)
     arr["sum_nnz_tok"] = nnz
+    arr["sum_nnz_doc"] = nnzd
     return arr
 
 

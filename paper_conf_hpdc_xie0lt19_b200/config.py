@@ -3,10 +3,9 @@ the parity test checks exactly the configuration the bench times."""
 
 # Options passed to lda_set_option for the timed runs.
 BENCH_OPTIONS = {
-    "sampler": 0,
     "chunk_tokens": 4096,
     "recount_tokens": 65536,
-    "tile_tokens": 8_000_000,
+    "tile_tokens": 16_000_000,
     "theta_mode": 1,
 }
 

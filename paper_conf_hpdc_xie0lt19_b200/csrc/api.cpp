@@ -27,7 +27,7 @@ struct lda_ctx {
     int64_t recount_tokens = 65536;
     int64_t tile_tokens = 0;
     int theta_mode = 0;
-    int sampler = 1;
+    int filter32 = 0;
     int threads = 0;
     // distribution
     int32_t rank = 0, world = 1;
@@ -50,7 +50,7 @@ struct lda_ctx {
     unsigned long long *d_stat_log = nullptr;
     size_t stat_log_cap = 0;
     std::vector<double> log_ms, log_ms_sample, log_ms_recount, log_ms_theta, log_ms_comm;
-    std::vector<int64_t> log_nnz_tok;
+    std::vector<int64_t> log_nnz_tok, log_nnz_doc;
 };
 
 namespace {
@@ -237,9 +237,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "tile_tokens") {
         if (value < 0) return fail(ctx, LDA_EINVAL, "tile_tokens must be >= 0");
         ctx->tile_tokens = value;
-    } else if (k == "sampler") {
-        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "sampler must be 0 or 1");
-        ctx->sampler = static_cast<int>(value);
+    } else if (k == "filter32") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "filter32 must be 0 or 1");
+        ctx->filter32 = static_cast<int>(value);
     } else if (k == "theta_mode") {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_mode must be 0 or 1");
         ctx->theta_mode = static_cast<int>(value);
@@ -272,6 +272,25 @@ int lda_init_dist(lda_ctx *ctx, int32_t rank, int32_t world, const void *uid) {
     ncclUniqueId id;
     std::memcpy(&id, uid, sizeof(id));
     NC(CommInitRank(&ctx->comm, world, id, rank));
+    return LDA_OK;
+}
+
+int lda_canonical_bases(int32_t V, int32_t world, int32_t rank, const int64_t *word_counts, int64_t *cbase,
+                        int64_t *total) {
+    if (V < 1 || world < 1 || rank < 0 || rank >= world || !word_counts || !cbase) return LDA_EINVAL;
+    int64_t run = 0;
+    for (int32_t w = 0; w < V; ++w) {
+        int64_t before_rank = 0, tot = 0;
+        for (int32_t g = 0; g < world; ++g) {
+            const int64_t n = word_counts[static_cast<size_t>(g) * V + w];
+            if (n < 0) return LDA_EINVAL;
+            if (g < rank) before_rank += n;
+            tot += n;
+        }
+        cbase[w] = run + before_rank;
+        run += tot;
+    }
+    if (total) *total = run;
     return LDA_OK;
 }
 
@@ -334,16 +353,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     }
     std::vector<int64_t> cbase(V);
     int64_t run = 0;
-    for (int32_t w = 0; w < V; ++w) {
-        int64_t before_rank = 0, tot = 0;
-        for (int32_t g = 0; g < ctx->world; ++g) {
-            int64_t n = all[static_cast<size_t>(g) * V + w];
-            if (g < ctx->rank) before_rank += n;
-            tot += n;
-        }
-        cbase[w] = run + before_rank;
-        run += tot;
-    }
+    lda_canonical_bases(V, ctx->world, ctx->rank, all.data(), cbase.data(), &run);
     ctx->T_global = run;
 
     lda::HostLayout &H = ctx->H;
@@ -361,12 +371,13 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.beta = ctx->beta;
     S.seed = seed;
     S.exclude_self = ctx->exclude_self;
-    S.sampler = ctx->sampler;
+    S.filter32 = ctx->filter32;
     KL(lda::configure_kernels(S));
 
     DA(S.tok_row, Tg);
     DA(S.tok_z, Tg);
     DA(S.doc_map, Tg);
+    DA(S.tok_crank, Tg);
     if (ctx->theta_mode == 1) DA(S.z_doc, Tg + 4);
     DA(S.doc_ptr32, Dg + 1);
     DA(S.row_off32, std::max<int64_t>(Dg, 1));
@@ -379,24 +390,29 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     DA(S.split_words, H.split_words.size());
     DA(S.rows, H.rows32 * 8);
     DA(S.nwk, static_cast<size_t>(V) * K + K);
+    if (S.sweep_fused) DA(S.nwk_alt, static_cast<size_t>(V) * K + K);
+    S.n_zero_words = static_cast<int64_t>(H.zero_words.size());
+    DA(S.zero_words, H.zero_words.size());
     DA(S.denom, K);
     DA(S.counter, 4);
     DA(S.stat, 4);
     DA(S.ll_part, 2 * S.ll_blocks + 2);
     DA(S.ll_out, 2);
-    if (S.sweep_smem < static_cast<size_t>(16) * K + 4096) DA(S.sweep_scratch, static_cast<size_t>(S.sweep_grid) * 2 * K);
+    if (!S.sweep_fused) DA(S.sweep_scratch, static_cast<size_t>(S.sweep_grid) * 2 * K);
 
     auto h2d = [&](void *dst, const void *src, size_t bytes) {
         return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream) : cudaSuccess;
     };
     CU(h2d(S.tok_row, H.tok_row.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.doc_map, H.doc_map.data(), sizeof(uint32_t) * Tg));
+    CU(h2d(S.tok_crank, H.tok_crank.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.doc_ptr32, H.doc_ptr32.data(), sizeof(uint32_t) * (Dg + 1)));
     CU(h2d(S.row_off32, H.row_off32.data(), sizeof(uint32_t) * Dg));
     CU(h2d(S.segs, H.segs.data(), sizeof(lda::Seg) * H.segs.size()));
     CU(h2d(S.chunks, H.chunks.data(), sizeof(lda::SampleChunk) * H.chunks.size()));
     CU(h2d(S.rchunks, H.rchunks.data(), sizeof(lda::RecountChunk) * H.rchunks.size()));
     CU(h2d(S.split_words, H.split_words.data(), sizeof(int32_t) * H.split_words.size()));
+    CU(h2d(S.zero_words, H.zero_words.data(), sizeof(int32_t) * H.zero_words.size()));
     CU(cudaMemsetAsync(S.rows, 0, H.rows32 * 32, ctx->stream));
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
@@ -408,6 +424,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(cudaStreamSynchronize(ctx->stream));
     // host copies no longer needed on the device side (doc_map kept for get_counts)
     std::vector<uint32_t>().swap(H.tok_row);
+    std::vector<uint32_t>().swap(H.tok_crank);
     ctx->loaded = true;
     ctx->sweeps = 0;
     ctx->stats.local_tokens = Tg;
@@ -445,7 +462,8 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventRecord(E[0], ctx->stream));
         KL(lda::launch_sweep(S, t, ctx->stream, &launches));
         CU(cudaEventRecord(E[1], ctx->stream));
-        KL(lda::launch_recount(S, ctx->stream, &launches));
+        if (S.sweep_fused) std::swap(S.nwk, S.nwk_alt);  // the sampler wrote the next counts
+        else KL(lda::launch_recount(S, ctx->stream, &launches));
         CU(cudaEventRecord(E[2], ctx->stream));
         if (ctx->world > 1) {
             // ϕ sync overlapped with the θ update (§6.2)
@@ -475,6 +493,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     ctx->log_ms_theta.assign(n, 0);
     ctx->log_ms_comm.assign(n, 0);
     ctx->log_nnz_tok.assign(n, 0);
+    ctx->log_nnz_doc.assign(n, 0);
     for (int32_t s = 0; s < n; ++s) {
         cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
         float a = 0, b = 0, c = 0, d = 0, tot = 0;
@@ -497,6 +516,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         ctx->log_nnz_tok[s] = ctx->cur_lnnz;
         ctx->cur_lnnz = static_cast<int64_t>(hs[2 * s]);
         ctx->cur_nnz = static_cast<int64_t>(hs[2 * s + 1]);
+        ctx->log_nnz_doc[s] = ctx->cur_nnz;
         if (s == n - 1) {
             st.ms_last_sweep = tot;
             st.ms_last_sample = a;
@@ -509,7 +529,8 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
 }
 
 int lda_get_sweep_log(lda_ctx *ctx, int32_t cap, double *ms_sweep, double *ms_sample, double *ms_recount,
-                      double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int32_t *n_out) {
+                      double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int64_t *sum_nnz_doc,
+                      int32_t *n_out) {
     PRECHECK(ctx);
     const int32_t n = static_cast<int32_t>(ctx->log_ms.size());
     if (n_out) *n_out = n;
@@ -521,6 +542,7 @@ int lda_get_sweep_log(lda_ctx *ctx, int32_t cap, double *ms_sweep, double *ms_sa
         if (ms_theta) ms_theta[s] = ctx->log_ms_theta[s];
         if (ms_allreduce) ms_allreduce[s] = ctx->log_ms_comm[s];
         if (sum_nnz_tok) sum_nnz_tok[s] = ctx->log_nnz_tok[s];
+        if (sum_nnz_doc) sum_nnz_doc[s] = ctx->log_nnz_doc[s];
     }
     return LDA_OK;
 }

@@ -126,14 +126,25 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
         const int64_t nd = d1 - d0;
         const int64_t t0 = doc_ptr[d0];
-        // split the tile's docs across threads (contiguous, by doc count)
+        // Processing order inside the tile: documents by decreasing length,
+        // so that the 32 tokens a warp draws together (consecutive in a
+        // word's run) come from documents of similar length -> similar θ row
+        // lengths -> little SIMT divergence.  (The Philox counter does not
+        // depend on this order: each token carries its canonical rank.)
+        std::vector<int64_t> ord(nd);
+        for (int64_t i = 0; i < nd; ++i) ord[i] = d0 + i;
+        std::stable_sort(ord.begin(), ord.end(), [&](int64_t x, int64_t y) {
+            return doc_ptr[x + 1] - doc_ptr[x] > doc_ptr[y + 1] - doc_ptr[y];
+        });
+        // split the tile's docs across threads (contiguous in `ord`)
         int nth = (doc_ptr[d1] - t0) < (1 << 16) ? 1 : nthreads;
         std::vector<int64_t> tdoc(nth + 1);
-        for (int t = 0; t <= nth; ++t) tdoc[t] = d0 + nd * t / nth;
+        for (int t = 0; t <= nth; ++t) tdoc[t] = nd * t / nth;
         auto count_part = [&](int t) {
             auto &h = hist[t];
             std::fill(h.begin(), h.end(), 0u);
-            for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) h[words[i]]++;
+            for (int64_t k = tdoc[t]; k < tdoc[t + 1]; ++k)
+                for (int64_t i = doc_ptr[ord[k]]; i < doc_ptr[ord[k] + 1]; ++i) h[words[i]]++;
         };
         {
             std::vector<std::thread> th;
@@ -159,7 +170,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         }
         auto scatter_part = [&](int t) {
             auto &next = hist[t];
-            for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
+            for (int64_t k = tdoc[t]; k < tdoc[t + 1]; ++k) {
+                const int64_t d = ord[k];
                 uint32_t row = L.row_off32[d];
                 for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
                     uint32_t p = next[words[i]]++;
@@ -176,9 +188,46 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         }
     }
 
+    // Canonical rank of every token within its word on this rank, stored at
+    // its word-major position: c = cbase[w] + tok_crank[p] (X18).
+    L.tok_crank.assign(T, 0);
+    {
+        const int nth = T < (1 << 16) ? 1 : nthreads;
+        std::vector<int64_t> tdoc(nth + 1);
+        for (int t = 0; t <= nth; ++t) tdoc[t] = D * t / nth;
+        auto count_part = [&](int t) {
+            auto &h = hist[t];
+            std::fill(h.begin(), h.end(), 0u);
+            for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) h[words[i]]++;
+        };
+        {
+            std::vector<std::thread> th;
+            for (int t = 1; t < nth; ++t) th.emplace_back(count_part, t);
+            count_part(0);
+            for (auto &x : th) x.join();
+        }
+        for (int32_t w = 0; w < V; ++w) {
+            uint32_t run = 0;
+            for (int t = 0; t < nth; ++t) {
+                const uint32_t h = hist[t][w];
+                hist[t][w] = run;
+                run += h;
+            }
+        }
+        auto rank_part = [&](int t) {
+            auto &next = hist[t];
+            for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i)
+                L.tok_crank[L.doc_map[i]] = next[words[i]]++;
+        };
+        std::vector<std::thread> th;
+        for (int t = 1; t < nth; ++t) th.emplace_back(rank_part, t);
+        rank_part(0);
+        for (auto &x : th) x.join();
+    }
+
     // Per-word runs (tile order) + sentinel; segment index of each word's first run.
     L.segs.clear();
-    std::vector<uint64_t> wseg0(V);
+    std::vector<uint64_t> wseg0(V + 1);
     for (int32_t w = 0; w < V; ++w) {
         wseg0[w] = L.segs.size();
         uint32_t acc = 0;
@@ -190,6 +239,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         }
         L.segs.push_back(Seg{0u, acc});
     }
+    wseg0[V] = L.segs.size();
     if (L.segs.size() >= (uint64_t(1) << 32)) return "too many word runs";
     std::vector<uint32_t>().swap(tseg);
     auto seg_of = [&](int32_t w, uint32_t v) {
@@ -202,10 +252,12 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // chunk_tokens, each a virtual range spanning the word's runs; the
     // canonical index continues word w's run on this rank (cbase[w] + v).
     L.chunks.clear();
+    L.zero_words.clear();
     for (int32_t w = 0; w < V; ++w) {
         const int64_t n = L.word_count[w];
-        if (n == 0) continue;
         const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
+        if (pieces != 1) L.zero_words.push_back(w);
+        if (n == 0) continue;
         for (int64_t q = 0; q < pieces; ++q) {
             const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
             SampleChunk c;
@@ -213,7 +265,9 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             c.vbegin = static_cast<uint32_t>(vb);
             c.count = static_cast<uint32_t>(ve - vb);
             c.seg0 = seg_of(w, static_cast<uint32_t>(vb));
-            c.c_base = static_cast<uint64_t>(cbase[w] + vb);
+            c.segN = static_cast<uint32_t>(wseg0[w + 1] - 1);
+            c.pad = pieces > 1 ? 1u : 0u;  // bit 0: the word is split over chunks
+            c.c_base = static_cast<uint64_t>(cbase[w]);
             L.chunks.push_back(c);
         }
     }
@@ -234,6 +288,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             c.vbegin = static_cast<uint32_t>(vb);
             c.vcount = static_cast<uint32_t>(ve - vb);
             c.seg0 = n ? seg_of(w, static_cast<uint32_t>(vb)) : static_cast<uint32_t>(wseg0[w]);
+            c.segN = static_cast<uint32_t>(wseg0[w + 1] - 1);
+            c.pad[0] = c.pad[1] = c.pad[2] = 0;
             L.rchunks.push_back(c);
         }
     }

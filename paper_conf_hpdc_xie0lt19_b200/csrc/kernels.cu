@@ -28,12 +28,18 @@ constexpr unsigned kFull = 0xffffffffu;
 constexpr int kSweepThreads = 256;
 constexpr int kMaxBlk = 16;  // block-end prefixes kept per token for the sparse rescan
 #ifndef LDA_RING
-#define LDA_RING 6
+#define LDA_RING 3
+#endif
+#ifndef LDA_MATCH
+#define LDA_MATCH 0
+#endif
+#ifndef LDA_FUSE
+#define LDA_FUSE 1
 #endif
 #ifndef LDA_SWEEP_MINB
 #define LDA_SWEEP_MINB 3
 #endif
-constexpr int kRing = LDA_RING;  // 16-byte row quads in flight per sampler lane
+constexpr int kRing = LDA_RING;  // 32-byte row blocks in flight per sampler lane
 
 // ---------------------------------------------------------------------------
 // Philox4x32-10 (Salmon et al. SC'11), output word 0 only.  Counter
@@ -55,6 +61,19 @@ __device__ __forceinline__ uint32_t philox_x0(uint64_t c, uint32_t t, uint32_t k
     return c0;
 }
 
+// One 32-byte θ row block per lane: a single 256-bit load (sm_100 LDG.256).
+struct Blk8 {
+    uint32_t w[8];
+};
+__device__ __forceinline__ Blk8 ld_nc_v8(const uint32_t *p) {
+    Blk8 b;
+    asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(b.w[0]), "=r"(b.w[1]), "=r"(b.w[2]), "=r"(b.w[3]), "=r"(b.w[4]), "=r"(b.w[5]),
+                   "=r"(b.w[6]), "=r"(b.w[7])
+                 : "l"(p));
+    return b;
+}
+
 __device__ __forceinline__ uint4 ld_nc_v4(const uint4 *p) {
     uint4 v;
     asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -63,32 +82,41 @@ __device__ __forceinline__ uint4 ld_nc_v4(const uint4 *p) {
     return v;
 }
 
+// Bring the 32-byte sector at p into L2 (no register, no scoreboard).
+__device__ __forceinline__ void prefetch_l2(const void *p) {
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+
 // Bring [p, p + bytes) into L2 without a register or scoreboard slot (one
 // bulk-prefetch instruction per θ row; bytes a multiple of 16).
 __device__ __forceinline__ void prefetch_l2_bulk(const void *p, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
 }
 
-// Word-major position of virtual index v of a word, walking the word's runs
-// forward from run s (v must not decrease between calls with the same s).
-__device__ __forceinline__ uint32_t run_position(const Seg *__restrict__ segs, uint32_t &s, uint32_t v) {
-    while (segs[s + 1].vstart <= v) ++s;
-    return segs[s].pos + (v - segs[s].vstart);
+// Word-major position of virtual index v of a word whose item spans runs
+// [lo, hi) (hi = the word's sentinel): binary search of the run holding v.
+__device__ __forceinline__ uint32_t run_position(const Seg *__restrict__ segs, uint32_t lo, uint32_t hi,
+                                                 uint32_t v) {
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (segs[mid].vstart <= v) lo = mid;
+        else hi = mid;
+    }
+    return segs[lo].pos + (v - segs[lo].vstart);
 }
 
 // ---------------------------------------------------------------------------
 // a1: random initial assignment (L377-379; X10): z = (x0·K) >> 32, t = 0.
 // ---------------------------------------------------------------------------
 __global__ void init_kernel(const SampleChunk *__restrict__ chunks, int64_t n_chunks,
-                            const Seg *__restrict__ segs, uint16_t *__restrict__ z, uint32_t K, uint32_t k0,
-                            uint32_t k1) {
+                            const Seg *__restrict__ segs, const uint32_t *__restrict__ tok_crank,
+                            uint16_t *__restrict__ z, uint32_t K, uint32_t k0, uint32_t k1) {
     for (int64_t ci = blockIdx.x; ci < n_chunks; ci += gridDim.x) {
         const SampleChunk ch = chunks[ci];
-        uint32_t sg = ch.seg0;
         for (uint32_t j = threadIdx.x; j < ch.count; j += blockDim.x) {
-            const uint32_t x0 = philox_x0(ch.c_base + j, 0u, k0, k1);
-            z[run_position(segs, sg, ch.vbegin + j)] =
-                static_cast<uint16_t>((static_cast<uint64_t>(x0) * K) >> 32);
+            const uint32_t p = run_position(segs, ch.seg0, ch.segN, ch.vbegin + j);
+            const uint32_t x0 = philox_x0(ch.c_base + tok_crank[p], 0u, k0, k1);
+            z[p] = static_cast<uint16_t>((static_cast<uint64_t>(x0) * K) >> 32);
         }
     }
 }
@@ -124,12 +152,15 @@ struct SweepArgs {
     int64_t n_chunks;
     const Seg *segs;
     const uint32_t *tok_row;
+    const uint32_t *tok_crank;
     uint16_t *z;
     const uint4 *rows;
     const int32_t *nwk;
     const int32_t *nk;
     const double *denom;
     uint32_t *counter;
+    int32_t *nwk_next;  // fused recount target rows (V*K), or null
+    int32_t *nk_next;   // and its n_k
     double *gscratch;  // non-null when the K-length arrays do not fit in smem
     int K;
     double alpha, beta, Vbeta;
@@ -168,18 +199,61 @@ struct Mass {
     }
 };
 
-template <bool EXCL>
+// The exact (fp64) draw of one token, as the fp64 walk in sweep_kernel
+// computes it, by linear scans: fallback of the fp32 filter for tokens whose
+// uniform lies within the filter's error bound of a CDF boundary.
+__device__ __noinline__ int draw_exact(const uint32_t *rw, uint32_t len, const double *pstar, const double *P,
+                                       double Q, int K, uint32_t x0) {
+    const uint32_t nblk = (len + 8u) >> 3;
+    double S = 0.0;
+    for (uint32_t b = 0; b < nblk; ++b) {
+        const Blk8 u = ld_nc_v8(rw + 8 * b);
+        for (int e = (b == 0 ? 1 : 0); e < 8; ++e)
+            S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], S);
+    }
+    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
+    if (x < S) {
+        double C = 0.0;
+        for (uint32_t b = 0; b < nblk; ++b) {
+            const Blk8 u = ld_nc_v8(rw + 8 * b);
+            for (int e = (b == 0 ? 1 : 0); e < 8; ++e) {
+                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], C);
+                if (C > x) return static_cast<int>(u.w[e] >> 16);
+            }
+        }
+        return K - 1;
+    }
+    int lo = 0, hi = K - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (S + P[mid] > x) hi = mid;
+        else lo = mid + 1;
+    }
+    return lo;
+}
+
+// SMEMP: p*/P in shared memory (LDS addressing); else in a global scratch
+// slice per CTA (large K).
+template <bool EXCL, bool SMEMP, bool F32>
 __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(SweepArgs a) {
+    static_assert(!F32 || (SMEMP && !EXCL), "the fp32 filter needs p* in smem and exclude_self = 0");
     extern __shared__ double smem_d[];
     __shared__ int s_ci;
     __shared__ double s_wtot[kSweepThreads / 32];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int K = a.K;
-    // smem: [blkC: kMaxBlk x 256 fp64][p*: K][P: K] (p*/P in global scratch for large K)
+    // smem: [blkC: kMaxBlk x 256 fp64][p*: K][P: K][hist: K i32][nk partial: K i32]
+    // (SMEMP = false: p*/P in a global scratch slice, no fused recount)
     double *blkC = smem_d;
-    double *pstar = a.gscratch ? a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K
-                               : smem_d + kMaxBlk * kSweepThreads;
+    double *pstar = SMEMP ? smem_d + kMaxBlk * kSweepThreads : a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K;
     double *P = pstar + K;
+    float *p32 = reinterpret_cast<float *>(smem_d + kMaxBlk * kSweepThreads + 2 * K);  // fp32 copy of p*
+    float *blk32 = reinterpret_cast<float *>(blkC);
+    int *hist = reinterpret_cast<int *>(p32 + K);
+    int *nkp = hist + K;
+    if (SMEMP) {
+        for (int k = tid; k < 2 * K; k += kSweepThreads) hist[k] = 0;
+    }
     const int E = (K + kSweepThreads - 1) / kSweepThreads;
     int cur_word = -1;
 
@@ -200,6 +274,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                 if (k < K) {
                     const double ps = (static_cast<double>(__ldg(nwk_row + k)) + a.beta) / __ldg(a.denom + k);
                     pstar[k] = ps;
+                    if (SMEMP) p32[k] = static_cast<float>(ps);
                     run = run + a.alpha * ps;
                     P[k] = run;
                 }
@@ -225,22 +300,28 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
             cur_word = static_cast<int>(ch.word);
         }
         const double Q = P[K - 1];
+        const float Q32 = static_cast<float>(Q);
 
         // One sampler per lane; each thread draws tokens j, j+256, ...  The
-        // row is streamed in 16-byte quads through a ring of kRing quads held
-        // in registers, so ~kRing·16 B per thread are in flight (a 32-byte
-        // block = 2 quads; words past nnz in the last block are zero).
-        uint32_t sg = ch.seg0;
+        // row is streamed in 32-byte blocks (one 256-bit load per block per
+        // lane, sm_100 LDG.256) through a ring of kRing blocks held in
+        // registers; words past nnz in the last block are zero.
+        uint32_t pn = 0, rown = 0;
+        if (static_cast<uint32_t>(tid) < ch.count) {
+            pn = run_position(a.segs, ch.seg0, ch.segN, ch.vbegin + tid);
+            rown = __ldg(a.tok_row + pn);
+        }
         for (uint32_t j = tid; j < ch.count; j += kSweepThreads) {
-            const uint32_t p = run_position(a.segs, sg, ch.vbegin + j);
-            const uint32_t row = __ldg(a.tok_row + p);
-            const uint4 *r = a.rows + static_cast<size_t>(row) * 2;
-            uint4 q[kRing];
-            q[0] = ld_nc_v4(r);            // header quad: nnz + 3 entries
-#pragma unroll
-            for (int i = 1; i < kRing; ++i) q[i] = make_uint4(0u, 0u, 0u, 0u);
-            q[1] = ld_nc_v4(r + 1);        // every row has >= 1 block = 2 quads
-            const uint32_t x0 = philox_x0_sched(ch.c_base + j, a.t, a.key0, a.key1);
+            const uint32_t p = pn;
+            const uint32_t *rw = reinterpret_cast<const uint32_t *>(a.rows) + static_cast<size_t>(rown) * 8;
+            Blk8 q[kRing];
+            q[0] = ld_nc_v8(rw);           // block 0: nnz + 7 entries
+            const uint32_t jn = j + kSweepThreads;
+            if (jn < ch.count) {
+                pn = run_position(a.segs, ch.seg0, ch.segN, ch.vbegin + jn);
+                rown = __ldg(a.tok_row + pn);
+            }
+            const uint32_t x0 = philox_x0_sched(ch.c_base + __ldg(a.tok_crank + p), a.t, a.key0, a.key1);
             int zo = 0;
             double po_new = 0.0, delta = 0.0;
             if (EXCL) {
@@ -249,41 +330,103 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                          (static_cast<double>(a.nk[zo] - 1) + a.Vbeta);
                 delta = a.alpha * po_new - a.alpha * pstar[zo];
             }
-            const uint32_t len = q[0].x;
+            const uint32_t len = q[0].w[0];
             const uint32_t nblk = (len + 8u) >> 3;   // 32-byte blocks holding words 0..len
-            const uint32_t nq = 2u * nblk;           // quads to stream (zero-padded tail)
 #pragma unroll
-            for (int i = 2; i < kRing; ++i)
-                if (static_cast<uint32_t>(i) < nq) q[i] = ld_nc_v4(r + i);
+            for (int i = 1; i < kRing; ++i)
+                if (static_cast<uint32_t>(i) < nblk) q[i] = ld_nc_v8(rw + 8 * i);
+            int z;
+            if constexpr (F32) {
+                // fp32 filter (see draw_exact): the same walk in single
+                // precision plus a bound on its distance to the fp64 walk
+                float S = 0.0f;
+#pragma unroll
+                for (int e = 1; e < 8; ++e) S = fmaf(static_cast<float>(q[0].w[e] & 0xFFFFu), p32[q[0].w[e] >> 16], S);
+                blk32[tid] = S;
+                if (static_cast<uint32_t>(kRing) < nblk) q[0] = ld_nc_v8(rw + 8 * kRing);
+                for (uint32_t base = 0; base < nblk; base += kRing) {
+#pragma unroll
+                    for (int i = 0; i < kRing; ++i) {
+                        const uint32_t b = base + i;
+                        if (b == 0) continue;
+                        if (b >= nblk) break;
+                        const Blk8 u = q[i];
+                        const uint32_t nx = b + kRing;
+                        if (nx < nblk) q[i] = ld_nc_v8(rw + 8 * nx);
+#pragma unroll
+                        for (int e = 0; e < 8; ++e)
+                            S = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> 16], S);
+                        if (b < kMaxBlk) blk32[b * kSweepThreads + tid] = S;
+                    }
+                }
+                const float tot = S + Q32;
+                const float xf = __uint2float_rn(x0) * 2.3283064365386962890625e-10f * tot;
+                // |(C32 - x32) - (C64 - x64)| <= (2·nnz + 6)·2^-24·total (first order)
+                const float B = (2.0f * static_cast<float>(len) + 8.0f) * 6.0e-8f * tot;
+                bool ok = fabsf(xf - S) > B;
+                z = -1;
+                if (ok) {
+                    if (xf < S) {
+                        const uint32_t nb = nblk < kMaxBlk ? nblk : kMaxBlk;
+                        uint32_t b = 0;
+                        for (; b < nb; ++b) {
+                            const float d = blk32[b * kSweepThreads + tid] - xf;
+                            if (fabsf(d) <= B) { ok = false; break; }
+                            if (d > 0.0f) break;
+                        }
+                        float C = b == 0 ? 0.0f : blk32[(b - 1) * kSweepThreads + tid];
+                        for (; ok && z < 0 && b < nblk; ++b) {  // one block, or a linear tail past kMaxBlk
+                            const Blk8 u = ld_nc_v8(rw + 8 * b);
+#pragma unroll
+                            for (int e = 0; e < 8; ++e) {
+                                if (b == 0 && e == 0) continue;
+                                C = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> 16], C);
+                                const float d = C - xf;
+                                if (z < 0 && ok) {
+                                    if (fabsf(d) <= B) ok = false;
+                                    else if (d > 0.0f) z = static_cast<int>(u.w[e] >> 16);
+                                }
+                            }
+                        }
+                        if (z < 0) ok = false;
+                    } else {
+                        const double Sd = S, xd = xf, Bd = B;
+                        int lo = 0, hi = K - 1;
+                        while (lo < hi) {
+                            const int mid = (lo + hi) >> 1;
+                            const double d = (Sd + P[mid]) - xd;
+                            if (fabs(d) <= Bd) { ok = false; break; }
+                            if (d > 0.0) hi = mid;
+                            else lo = mid + 1;
+                        }
+                        z = lo;
+                    }
+                }
+                if (!ok) z = draw_exact(rw, len, pstar, P, Q, K, x0);
+            } else {
             // pass 1: S over the row, block-end prefixes to smem
             double S = 0.0;
-            S = Mass<EXCL>::fma_into(q[0].y, pstar, zo, po_new, S);
-            S = Mass<EXCL>::fma_into(q[0].z, pstar, zo, po_new, S);
-            S = Mass<EXCL>::fma_into(q[0].w, pstar, zo, po_new, S);
-            q[0] = (static_cast<uint32_t>(kRing) < nq) ? ld_nc_v4(r + kRing) : make_uint4(0u, 0u, 0u, 0u);
-            // quads 1 .. nq-1, ring slot (qi % kRing); qi odd ends a block
-            for (uint32_t base = 0; base < nq; base += kRing) {
+#pragma unroll
+            for (int e = 1; e < 8; ++e) S = Mass<EXCL>::fma_into(q[0].w[e], pstar, zo, po_new, S);
+            blkC[tid] = S;
+            if (static_cast<uint32_t>(kRing) < nblk) q[0] = ld_nc_v8(rw + 8 * kRing);
+            // blocks 1 .. nblk-1, ring slot (b % kRing)
+            for (uint32_t base = 0; base < nblk; base += kRing) {
 #pragma unroll
                 for (int i = 0; i < kRing; ++i) {
-                    const uint32_t qi = base + i;
-                    if (qi == 0) continue;
-                    if (qi >= nq) break;
-                    const uint4 u = q[i];
-                    const uint32_t nx = qi + kRing;
-                    q[i] = (nx < nq) ? ld_nc_v4(r + nx) : make_uint4(0u, 0u, 0u, 0u);
-                    S = Mass<EXCL>::fma_into(u.x, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u.y, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u.z, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u.w, pstar, zo, po_new, S);
-                    if (qi & 1u) {
-                        const uint32_t b = qi >> 1;
-                        if (b < kMaxBlk) blkC[b * kSweepThreads + tid] = S;
-                    }
+                    const uint32_t b = base + i;
+                    if (b == 0) continue;
+                    if (b >= nblk) break;
+                    const Blk8 u = q[i];
+                    const uint32_t nx = b + kRing;
+                    if (nx < nblk) q[i] = ld_nc_v8(rw + 8 * nx);
+#pragma unroll
+                    for (int e = 0; e < 8; ++e) S = Mass<EXCL>::fma_into(u.w[e], pstar, zo, po_new, S);
+                    if (b < kMaxBlk) blkC[b * kSweepThreads + tid] = S;
                 }
             }
             const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;  // x0 · 2^-32
             const double x = U * (S + (EXCL ? Q + delta : Q));
-            int z;
             if (x < S) {
                 // sparse bucket (p1): the first block whose end prefix exceeds x,
                 // then the identical recomputation inside it: first C > x
@@ -298,10 +441,10 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
         if (z < 0 && C > x) z = static_cast<int>((e) >> 16);          \
     }
                 for (; z < 0 && b < nblk; ++b) {  // one block, or a linear tail past kMaxBlk
-                    const uint4 u0 = ld_nc_v4(r + 2 * b), u1 = ld_nc_v4(r + 2 * b + 1);
-                    if (b > 0) LDA_STEP(u0.x)
-                    LDA_STEP(u0.y) LDA_STEP(u0.z) LDA_STEP(u0.w)
-                    LDA_STEP(u1.x) LDA_STEP(u1.y) LDA_STEP(u1.z) LDA_STEP(u1.w)
+                    const Blk8 u = ld_nc_v8(rw + 8 * b);
+                    if (b > 0) LDA_STEP(u.w[0])
+#pragma unroll
+                    for (int e = 1; e < 8; ++e) LDA_STEP(u.w[e])
                 }
 #undef LDA_STEP
                 if (z < 0) z = K - 1;  // unreachable: the last entry's prefix is S > x
@@ -317,279 +460,41 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                 }
                 z = lo;  // K-1 also when x >= S + Q by rounding (X6 fallback)
             }
+            }
             a.z[p] = static_cast<uint16_t>(z);
+            if (SMEMP) {
+#if LDA_MATCH
+                // one shared atomic per distinct topic among the active lanes
+                const unsigned peers = __match_any_sync(__activemask(), z);
+                if (lane == __ffs(peers) - 1) atomicAdd(&hist[z], __popc(peers));
+#else
+                atomicAdd(&hist[z], 1);
+#endif
+            }
         }
         __syncthreads();
-    }
-}
-
-// ---------------------------------------------------------------------------
-// a3 + a4, TMA-staged variant (the default sampler).
-//
-// Same arithmetic as sweep_kernel, but the θ rows are moved by the Tensor
-// Memory Accelerator instead of per-thread loads: each warp draws 32 tokens
-// at a time (one sampler per lane); a lane first loads its row's 32-byte
-// header block (nnz + 7 entries), then issues ONE cp.async.bulk copy of the
-// rest of its row into the warp's shared-memory stage, completing on an
-// mbarrier.  Two stages per warp: the bulk copies of batch i+1 and the header
-// loads of batch i+2 are in flight while batch i is drawn from shared memory,
-// so the memory system sees ~2 x 32 whole rows in flight per warp with no
-// registers tied up (the direct-load sampler above keeps ~1 block per thread
-// in flight and is latency-bound).
-// ---------------------------------------------------------------------------
-constexpr int kTW = 4;                // warps per CTA
-constexpr int kTThreads = 32 * kTW;   // 128
-constexpr int kTCap = 288;            // staged 32-byte blocks per warp per stage (~9 per lane)
-
-__device__ __forceinline__ uint32_t smem_u32(const void *p) {
-    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
-    uint32_t done = 0;
-    while (!done) {
-        asm volatile(
-            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
-            : "=r"(done)
-            : "r"(smem_u32(bar)), "r"(parity)
-            : "memory");
-    }
-}
-__device__ __forceinline__ void tma_row_to_smem(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-            smem_u32(dst)),
-        "l"(src), "r"(bytes), "r"(smem_u32(bar))
-        : "memory");
-}
-
-struct TBatch {
-    uint32_t p;     // word-major position of the lane's token
-    uint32_t row;   // θ row of its document, 32-byte units
-    uint4 h0, h1;   // row block 0: nnz + 7 entries
-    uint32_t off;   // first staged block in the warp's stage
-    uint32_t nst;   // staged blocks (row blocks 1..nst)
-    bool valid;
-};
-
-template <bool EXCL>
-__global__ void __launch_bounds__(kTThreads) sweep_tma_kernel(SweepArgs a) {
-    extern __shared__ __align__(128) unsigned char smem_t[];
-    __shared__ uint64_t mbar[2][kTW];
-    __shared__ int s_ci;
-    __shared__ double s_wtot[kTW];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int K = a.K;
-    // smem: [stage 0: kTW x kTCap x 32 B][stage 1][blkC: kMaxBlk x 128 fp64][p*: K][P: K]
-    uint4 *stage0 = reinterpret_cast<uint4 *>(smem_t);
-    double *blkC = reinterpret_cast<double *>(smem_t + 2 * kTW * kTCap * 32);
-    double *pstar = a.gscratch ? a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K : blkC + kMaxBlk * kTThreads;
-    double *P = pstar + K;
-    const int E = (K + kTThreads - 1) / kTThreads;
-    if (lane == 0) {
-        mbar_init(&mbar[0][warp], 1);
-        mbar_init(&mbar[1][warp], 1);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    __syncthreads();
-    uint32_t parity[2] = {0u, 0u};
-    int cur_word = -1;
-
-    for (;;) {
-        if (tid == 0) s_ci = static_cast<int>(atomicAdd(a.counter, 1u));
-        __syncthreads();
-        const int ci = s_ci;
-        if (ci >= a.n_chunks) break;
-        const SampleChunk ch = a.chunks[ci];
-        const int32_t *nwk_row = a.nwk + static_cast<size_t>(ch.word) * K;
-
-        if (static_cast<int>(ch.word) != cur_word) {
-            // p*(k) = (n_wk + β)/(n_k + Vβ) and the inclusive prefix of α·p*(k) (Eq. 8)
-            const int kb = tid * E;
-            double run = 0.0;
-            for (int e = 0; e < E; ++e) {
-                const int k = kb + e;
-                if (k < K) {
-                    const double ps = (static_cast<double>(__ldg(nwk_row + k)) + a.beta) / __ldg(a.denom + k);
-                    pstar[k] = ps;
-                    run = run + a.alpha * ps;
-                    P[k] = run;
-                }
-            }
-            double incl = run;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const double y = __shfl_up_sync(kFull, incl, o);
-                if (lane >= o) incl += y;
-            }
-            double lex = __shfl_up_sync(kFull, incl, 1);
-            if (lane == 0) lex = 0.0;
-            if (lane == 31) s_wtot[warp] = incl;
-            __syncthreads();
-            double off = 0.0;
-            for (int i = 0; i < warp; ++i) off += s_wtot[i];
-            off = off + lex;
-            for (int e = 0; e < E; ++e) {
-                const int k = kb + e;
-                if (k < K) P[k] = off + P[k];
-            }
-            __syncthreads();
-            cur_word = static_cast<int>(ch.word);
-        }
-        const double Q = P[K - 1];
-
-        // this warp's batches: tokens j = (i*kTW + warp)*32 + lane
-        uint32_t sg = ch.seg0;
-        auto load_header = [&](uint32_t i, TBatch &B) {
-            const uint32_t j = (i * kTW + warp) * 32u + lane;
-            B.valid = j < ch.count;
-            B.h0 = make_uint4(0u, 0u, 0u, 0u);
-            B.h1 = B.h0;
-            if (B.valid) {
-                B.p = run_position(a.segs, sg, ch.vbegin + j);
-                B.row = __ldg(a.tok_row + B.p);
-                const uint4 *r = a.rows + static_cast<size_t>(B.row) * 2;
-                B.h0 = ld_nc_v4(r);
-                B.h1 = ld_nc_v4(r + 1);
-            }
-        };
-        auto issue_body = [&](int s, TBatch &B) {
-            const uint32_t nblk = B.valid ? ((B.h0.x + 8u) >> 3) : 0u;
-            const uint32_t need = nblk ? nblk - 1u : 0u;
-            uint32_t incl = need;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(kFull, incl, o);
-                if (lane >= o) incl += y;
-            }
-            const uint32_t total = __shfl_sync(kFull, incl, 31);
-            B.off = incl - need;
-            B.nst = B.off >= static_cast<uint32_t>(kTCap) ? 0u : min(need, kTCap - B.off);
-            const uint32_t staged = min(total, static_cast<uint32_t>(kTCap));
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            __syncwarp();
-            if (lane == 0) mbar_arrive_expect_tx(&mbar[s][warp], staged * 32u);
-            __syncwarp();
-            if (B.nst) {
-                uint4 *dst = stage0 + (static_cast<size_t>(s) * kTW + warp) * kTCap * 2 + B.off * 2;
-                tma_row_to_smem(dst, a.rows + static_cast<size_t>(B.row) * 2 + 2, B.nst * 32u, &mbar[s][warp]);
-            }
-        };
-
-        const uint32_t nb = ch.count > static_cast<uint32_t>(warp) * 32u
-                                ? (ch.count - warp * 32u + kTW * 32u - 1u) / (kTW * 32u)
-                                : 0u;
-        TBatch Bc, Bn, Bnn;
-        if (nb > 0) {
-            load_header(0, Bc);
-            issue_body(0, Bc);
-            if (nb > 1) load_header(1, Bn);
-        }
-        for (uint32_t i = 0; i < nb; ++i) {
-            const int s = static_cast<int>(i & 1u);
-            if (i + 1 < nb) issue_body(s ^ 1, Bn);
-            if (i + 2 < nb) load_header(i + 2, Bnn);
-            mbar_wait(&mbar[s][warp], parity[s]);
-            parity[s] ^= 1u;
-
-            if (Bc.valid) {
-                const uint4 *stg = stage0 + (static_cast<size_t>(s) * kTW + warp) * kTCap * 2 + Bc.off * 2;
-                const uint4 *gr = a.rows + static_cast<size_t>(Bc.row) * 2;
-                const uint32_t j = (i * kTW + warp) * 32u + lane;
-                const uint32_t x0 = philox_x0_sched(ch.c_base + j, a.t, a.key0, a.key1);
-                int zo = 0;
-                double po_new = 0.0, delta = 0.0;
-                if (EXCL) {
-                    zo = static_cast<int>(a.z[Bc.p]);
-                    po_new = (static_cast<double>(nwk_row[zo] - 1) + a.beta) /
-                             (static_cast<double>(a.nk[zo] - 1) + a.Vbeta);
-                    delta = a.alpha * po_new - a.alpha * pstar[zo];
-                }
-                const uint32_t len = Bc.h0.x;
-                const uint32_t nblk = (len + 8u) >> 3;
-                // block b >= 1 of the row: staged copy, or global memory past the stage
-#define LDA_BLOCK(b, u0, u1)                                                     \
-    if ((b) <= Bc.nst) {                                                         \
-        u0 = stg[2 * ((b) - 1)];                                                 \
-        u1 = stg[2 * ((b) - 1) + 1];                                             \
-    } else {                                                                     \
-        u0 = ld_nc_v4(gr + 2 * (b));                                             \
-        u1 = ld_nc_v4(gr + 2 * (b) + 1);                                         \
-    }
-                double S = 0.0;
-                S = Mass<EXCL>::fma_into(Bc.h0.y, pstar, zo, po_new, S);
-                S = Mass<EXCL>::fma_into(Bc.h0.z, pstar, zo, po_new, S);
-                S = Mass<EXCL>::fma_into(Bc.h0.w, pstar, zo, po_new, S);
-                S = Mass<EXCL>::fma_into(Bc.h1.x, pstar, zo, po_new, S);
-                S = Mass<EXCL>::fma_into(Bc.h1.y, pstar, zo, po_new, S);
-                S = Mass<EXCL>::fma_into(Bc.h1.z, pstar, zo, po_new, S);
-                S = Mass<EXCL>::fma_into(Bc.h1.w, pstar, zo, po_new, S);
-                blkC[tid] = S;
-                for (uint32_t b = 1; b < nblk; ++b) {
-                    uint4 u0, u1;
-                    LDA_BLOCK(b, u0, u1)
-                    S = Mass<EXCL>::fma_into(u0.x, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u0.y, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u0.z, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u0.w, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u1.x, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u1.y, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u1.z, pstar, zo, po_new, S);
-                    S = Mass<EXCL>::fma_into(u1.w, pstar, zo, po_new, S);
-                    if (b < kMaxBlk) blkC[b * kTThreads + tid] = S;
-                }
-                const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;  // x0 · 2^-32
-                const double x = U * (S + (EXCL ? Q + delta : Q));
-                int z;
-                if (x < S) {
-                    const uint32_t nbk = nblk < kMaxBlk ? nblk : kMaxBlk;
-                    uint32_t b = 0;
-                    while (b < nbk && !(blkC[b * kTThreads + tid] > x)) ++b;
-                    double C = b == 0 ? 0.0 : blkC[(b - 1) * kTThreads + tid];
-                    z = -1;
-#define LDA_STEP(e)                                                   \
-    {                                                                 \
-        C = Mass<EXCL>::fma_into((e), pstar, zo, po_new, C);          \
-        if (z < 0 && C > x) z = static_cast<int>((e) >> 16);          \
-    }
-                    if (b == 0) {
-                        LDA_STEP(Bc.h0.y) LDA_STEP(Bc.h0.z) LDA_STEP(Bc.h0.w)
-                        LDA_STEP(Bc.h1.x) LDA_STEP(Bc.h1.y) LDA_STEP(Bc.h1.z) LDA_STEP(Bc.h1.w)
-                        b = 1;
-                    }
-                    for (; z < 0 && b < nblk; ++b) {
-                        uint4 u0, u1;
-                        LDA_BLOCK(b, u0, u1)
-                        LDA_STEP(u0.x) LDA_STEP(u0.y) LDA_STEP(u0.z) LDA_STEP(u0.w)
-                        LDA_STEP(u1.x) LDA_STEP(u1.y) LDA_STEP(u1.z) LDA_STEP(u1.w)
-                    }
-#undef LDA_STEP
-                    if (z < 0) z = K - 1;  // unreachable: the last entry's prefix is S > x
+        if (SMEMP) {
+            // fused n_wk recount (ϕ update, L1273-1285): this chunk's topic
+            // histogram -> the word's row of the next n_wk; atomics only when
+            // the word is split over several chunks
+            int32_t *row = a.nwk_next + static_cast<size_t>(ch.word) * K;
+            const bool split = (ch.pad & 1u) != 0u;
+            for (int k = tid; k < K; k += kSweepThreads) {
+                const int h = hist[k];
+                if (split) {
+                    if (h) atomicAdd(row + k, h);
                 } else {
-                    int lo = 0, hi = K - 1;
-                    while (lo < hi) {
-                        const int mid = (lo + hi) >> 1;
-                        double pk = P[mid];
-                        if (EXCL && mid >= zo) pk += delta;
-                        if (S + pk > x) hi = mid;
-                        else lo = mid + 1;
-                    }
-                    z = lo;
+                    row[k] = h;
                 }
-#undef LDA_BLOCK
-                a.z[Bc.p] = static_cast<uint16_t>(z);
+                nkp[k] += h;
+                hist[k] = 0;
             }
-            __syncwarp();
-            Bc = Bn;
-            Bn = Bnn;
         }
         __syncthreads();
+    }
+    if (SMEMP) {
+        for (int k = tid; k < K; k += kSweepThreads)
+            if (nkp[k]) atomicAdd(a.nk_next + k, nkp[k]);
     }
 }
 
@@ -621,9 +526,8 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
         const RecountChunk c = rc[ci];
         const uint32_t w = c.word & 0x7FFFFFFFu;
         const bool split = (c.word >> 31) != 0u;
-        uint32_t sg = c.seg0;
         for (uint32_t j = threadIdx.x; j < c.vcount; j += blockDim.x)
-            atomicAdd(&hist[z[run_position(segs, sg, c.vbegin + j)]], 1);
+            atomicAdd(&hist[z[run_position(segs, c.seg0, c.segN, c.vbegin + j)]], 1);
         __syncthreads();
         int32_t *row = nwk + static_cast<size_t>(w) * K;
         for (int k = threadIdx.x; k < K; k += blockDim.x) {
@@ -804,38 +708,28 @@ int configure_kernels(DevState &s) {
     int max_optin = 0;
     if ((e = cudaDeviceGetAttribute(&max_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev)) != cudaSuccess)
         return e;
-    // sampler
-    if (s.sampler == 1) {
-        const size_t fixed = 2 * kTW * kTCap * 32 + sizeof(double) * kMaxBlk * kTThreads;
-        const size_t want = fixed + static_cast<size_t>(16) * s.K;
-        s.sweep_smem = (want + 2048 <= static_cast<size_t>(max_optin)) ? want : fixed;
-        s.sweep_block = kTThreads;
-        const void *fns[2] = {reinterpret_cast<const void *>(&sweep_tma_kernel<false>),
-                              reinterpret_cast<const void *>(&sweep_tma_kernel<true>)};
-        for (int i = 0; i < 2; ++i)
-            if ((e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                          static_cast<int>(s.sweep_smem))) != cudaSuccess)
-                return e;
-        int bps = 1;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fns[s.exclude_self ? 1 : 0], kTThreads,
-                                                               s.sweep_smem)) != cudaSuccess)
-            return e;
-        s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
-    } else {
+    // sampler: p*/P (+ fused-recount histograms) in smem when they fit
+    {
         const size_t blk = sizeof(double) * kMaxBlk * kSweepThreads;
-        size_t want = blk + static_cast<size_t>(16) * s.K;
-        s.sweep_smem = (want + 2048 <= static_cast<size_t>(max_optin)) ? want : blk;
-        s.sweep_block = kSweepThreads;
-        const void *fns[2] = {reinterpret_cast<const void *>(&sweep_kernel<false>),
-                              reinterpret_cast<const void *>(&sweep_kernel<true>)};
+        const size_t want = blk + static_cast<size_t>(28) * s.K;
+        const bool smemp = LDA_FUSE && want + 2048 <= static_cast<size_t>(max_optin);
+        s.sweep_smem = smemp ? want : blk;
+        s.sweep_fused = smemp;
+        s.sweep_f32 = smemp && !s.exclude_self && s.filter32;
+        const void *fn = nullptr;
+        if (s.exclude_self)
+            fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<true, true, false>)
+                       : reinterpret_cast<const void *>(&sweep_kernel<true, false, false>);
+        else if (s.sweep_f32)
+            fn = reinterpret_cast<const void *>(&sweep_kernel<false, true, true>);
+        else
+            fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<false, true, false>)
+                       : reinterpret_cast<const void *>(&sweep_kernel<false, false, false>);
+        if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      static_cast<int>(s.sweep_smem))) != cudaSuccess)
+            return e;
         int bps = 1;
-        for (int i = 0; i < 2; ++i) {
-            if ((e = cudaFuncSetAttribute(fns[i], cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                          static_cast<int>(s.sweep_smem))) != cudaSuccess)
-                return e;
-        }
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fns[s.exclude_self ? 1 : 0], kSweepThreads,
-                                                               s.sweep_smem)) != cudaSuccess)
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, kSweepThreads, s.sweep_smem)) != cudaSuccess)
             return e;
         s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
     }
@@ -869,7 +763,7 @@ int configure_kernels(DevState &s) {
 int launch_init(const DevState &s, void *stream) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const int grid = static_cast<int>(std::min<int64_t>(s.n_chunks > 0 ? s.n_chunks : 1, 65535));
-    init_kernel<<<grid, 256, 0, st>>>(s.chunks, s.n_chunks, s.segs, s.tok_z, static_cast<uint32_t>(s.K),
+    init_kernel<<<grid, 256, 0, st>>>(s.chunks, s.n_chunks, s.segs, s.tok_crank, s.tok_z, static_cast<uint32_t>(s.K),
                                       static_cast<uint32_t>(s.seed), static_cast<uint32_t>(s.seed >> 32));
     return cudaGetLastError();
 }
@@ -918,17 +812,32 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
     ++*launches;
     if ((e = cudaMemsetAsync(s.counter, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
     SweepArgs a;
+    if (s.sweep_fused) {
+        // next n_wk: rows of words split over chunks (or without tokens) and n_k start at 0
+        a.nwk_next = s.nwk_alt;
+        a.nk_next = s.nwk_alt + static_cast<size_t>(s.V) * s.K;
+        if ((e = cudaMemsetAsync(a.nk_next, 0, sizeof(int32_t) * s.K, st)) != cudaSuccess) return e;
+        if (s.n_zero_words > 0) {
+            zero_rows_kernel<<<static_cast<int>(std::min<int64_t>(s.n_zero_words, 65535)), 256, 0, st>>>(
+                s.zero_words, s.n_zero_words, s.nwk_alt, s.K);
+            ++*launches;
+        }
+    } else {
+        a.nwk_next = nullptr;
+        a.nk_next = nullptr;
+    }
     a.chunks = s.chunks;
     a.n_chunks = s.n_chunks;
     a.segs = s.segs;
     a.tok_row = s.tok_row;
+    a.tok_crank = s.tok_crank;
     a.z = s.tok_z;
     a.rows = reinterpret_cast<const uint4 *>(s.rows);
     a.nwk = s.nwk;
     a.nk = nk;
     a.denom = s.denom;
     a.counter = s.counter;
-    a.gscratch = s.sweep_scratch;  // non-null only when p*/P do not fit in smem
+    a.gscratch = s.sweep_fused ? nullptr : s.sweep_scratch;
     a.K = s.K;
     a.alpha = s.alpha;
     a.beta = s.beta;
@@ -941,16 +850,14 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
         k0 += 0x9E3779B9u;
         k1 += 0xBB67AE85u;
     }
-    if (s.sampler == 1) {
-        if (s.exclude_self)
-            sweep_tma_kernel<true><<<s.sweep_grid, kTThreads, s.sweep_smem, st>>>(a);
-        else
-            sweep_tma_kernel<false><<<s.sweep_grid, kTThreads, s.sweep_smem, st>>>(a);
+    if (s.exclude_self) {
+        if (s.sweep_fused) sweep_kernel<true, true, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        else sweep_kernel<true, false, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+    } else if (s.sweep_f32) {
+        sweep_kernel<false, true, true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
     } else {
-        if (s.exclude_self)
-            sweep_kernel<true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
-        else
-            sweep_kernel<false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        if (s.sweep_fused) sweep_kernel<false, true, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        else sweep_kernel<false, false, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
     }
     ++*launches;
     return cudaGetLastError();

@@ -20,13 +20,16 @@ struct Seg {
 
 // One sampling work item: tokens [vbegin, vbegin+count) of one word (the
 // word-first order of L1189-1191; heavy words split over several items,
-// L1203-1221).  seg0 = index of the run holding vbegin; c_base = canonical
-// index of virtual index vbegin.
+// L1203-1221).  Runs [seg0, segN) hold the item (segN = the word's
+// sentinel); c_base = canonical index of the rank's first token of the word
+// (a token's index is c_base + tok_crank[p]).
 struct SampleChunk {
     uint32_t word;
     uint32_t vbegin;
     uint32_t count;
     uint32_t seg0;
+    uint32_t segN;
+    uint32_t pad;
     uint64_t c_base;
 };
 
@@ -38,6 +41,8 @@ struct RecountChunk {
     uint32_t vbegin;
     uint32_t vcount;
     uint32_t seg0;
+    uint32_t segN;
+    uint32_t pad[3];
 };
 
 // Host-side layout of one rank's shard (built by build_layout).
@@ -50,10 +55,12 @@ struct HostLayout {
     uint64_t rows32 = 0;               // θ row buffer size in 32-byte units (incl. tail pad)
     std::vector<uint32_t> tok_row;     // T   word-major: θ row (32 B units) of the token's doc
     std::vector<uint32_t> doc_map;     // T   doc-major token i -> word-major position (S7, L1297-1303)
+    std::vector<uint32_t> tok_crank;   // T   word-major: canonical rank of the token within its word
     std::vector<Seg> segs;             // per word: its runs, then a sentinel
     std::vector<SampleChunk> chunks;   // heavy-first
     std::vector<RecountChunk> rchunks; // heavy-first
-    std::vector<int32_t> split_words;  // words whose row is accumulated atomically
+    std::vector<int32_t> split_words;  // words whose row is accumulated atomically (recount)
+    std::vector<int32_t> zero_words;   // words split over sampler chunks or without tokens
     std::vector<int64_t> word_count;   // V local tokens per word
 };
 
@@ -81,11 +88,11 @@ struct DevState {
     double alpha = 0, beta = 0;
     uint64_t seed = 0;
     int exclude_self = 0;
-    int sampler = 1;                // 1 = TMA-staged rows (default), 0 = direct loads
     // corpus
     uint32_t *tok_row = nullptr;    // T
     uint16_t *tok_z = nullptr;      // T (word-major)
     uint32_t *doc_map = nullptr;    // T
+    uint32_t *tok_crank = nullptr;  // T (word-major)
     uint16_t *z_doc = nullptr;      // T, z in document order (two-phase θ rebuild only)
     uint32_t *doc_ptr32 = nullptr;  // D+1
     uint32_t *row_off32 = nullptr;  // D
@@ -98,7 +105,13 @@ struct DevState {
     int64_t n_split = 0;
     // model
     uint32_t *rows = nullptr;       // θ rows, rows32*8 words
-    int32_t *nwk = nullptr;         // V*K + K (n_k at offset V*K)
+    int32_t *nwk = nullptr;         // V*K + K (n_k at offset V*K), the current counts
+    int32_t *nwk_alt = nullptr;     // the other buffer: the sampler's fused recount writes here
+    int32_t *zero_words = nullptr;  // words whose next-n_wk row is zeroed before the sweep
+    int64_t n_zero_words = 0;
+    bool sweep_fused = false;
+    bool sweep_f32 = false;
+    int filter32 = 0;               // option: fp32 filter with exact fp64 fallback
     double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch
     uint32_t *counter = nullptr;    // work counters [4]

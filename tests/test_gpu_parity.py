@@ -109,7 +109,7 @@ def test_nytimes_shaped_midsize_many_chunks():
     z_ref = g.z()
     for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
                  dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3),
-                 dict(theta_mode=1), dict(sampler=0), dict(sampler=0, tile_tokens=20_000)]:
+                 dict(theta_mode=1), dict(theta_mode=1, tile_tokens=20_000), dict(filter32=1)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
@@ -120,11 +120,10 @@ def test_exclude_self_lockstep():
     doc_ptr, words = _corpus(500, 300, 30_000, 0.5, 16, 13)
     K = 24
     o = U.oracle_for(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3)
-    for sampler in (1, 0):
-        o = U.oracle_for(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3)
-        g = U.gpu_model(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3, exclude_self=1, sampler=sampler)
-        bad, unexc = U.lockstep(g, o, 3, exclude_self=1)
-        assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
+    o = U.oracle_for(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3)
+    g = U.gpu_model(500, 300, K, 50.0 / K, 0.01, doc_ptr, words, 3, exclude_self=1)
+    bad, unexc = U.lockstep(g, o, 3, exclude_self=1)
+    assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
 def test_edge_cases():
@@ -147,6 +146,19 @@ def test_edge_cases():
     o1 = U.oracle_for(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
     g1 = U.gpu_model(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
     U.lockstep(g1, o1, 5)
+
+
+def test_filter32_is_exact_at_scale():
+    """The fp32 filter + fp64 fallback must reproduce the always-fp64 walk bit
+    for bit: 10 sweeps of a NYTimes-shaped corpus, z compared."""
+    cfg = synth.scaled(synth.CONFIGS["nytimes"], 0.01)        # ~1 M tokens
+    doc_ptr, words = synth.to_numpy(*synth.generate_config(cfg, "cpu"))[:2]
+    g32 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, filter32=1)
+    g64 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, filter32=0)
+    for _ in range(10):
+        g32.iterate(1)
+        g64.iterate(1)
+        assert np.array_equal(g32.z(), g64.z())
 
 
 def test_set_z_and_determinism():
