@@ -75,6 +75,9 @@ typedef struct lda_stats {
     int64_t sum_nnz_doc;    /* Σ_d nnz_d of θ after the last sweep */
     int64_t n_launches;     /* library kernels launched by the last call */
     int64_t n_sample_chunks;/* sampler work items (word chunks) */
+    int64_t n_exact_redraws;/* quad sampler: tokens of the last lda_iterate call
+                               whose fp32 filter margin was too small and that
+                               were redrawn by the exact fp64 walk */
 } lda_stats;
 
 /* Create a context.  D = global number of documents, V = vocabulary size,
@@ -93,9 +96,19 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tile_tokens"   split the documents into tiles of about this many tokens
  *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
- *   "filter32"      1: draw each token in fp32 first and redo it in fp64 when
- *                   its uniform lies within the fp32 error bound of a CDF
- *                   boundary — results identical to 0 (always fp64, default)
+ *   "sampler"       1 (default): quad sampler -- the tokens of a word chunk
+ *                   grouped into (word, document) pairs, four lanes walk
+ *                   the pair's θ row line by line (128-byte lines), one
+ *                   draw per token; used when K fits its shared-memory
+ *                   layout (K <= ~8000) and exclude_self = 0, else 0.
+ *                   0: lane-per-token sampler (32-byte row blocks).
+ *                   The two differ only in fp64 summation order of the
+ *                   sparse prefix (draws differ only within rounding of a
+ *                   CDF boundary).
+ *   "filter32"      sampler 0 only.  1: draw each token in fp32 first and
+ *                   redo it in fp64 when its uniform lies within the fp32
+ *                   error bound of a CDF boundary — results identical to 0
+ *                   (always fp64, default)
  *   "theta_mode"    θ rebuild: 0 = fused gather+histogram (default),
  *                   1 = two-phase (z gathered into document order first)
  * Results do not depend on chunk_tokens, recount_tokens, tile_tokens or

@@ -28,6 +28,7 @@ struct lda_ctx {
     int64_t tile_tokens = 0;
     int theta_mode = 0;
     int filter32 = 0;
+    int sampler = 1;
     int threads = 0;
     // distribution
     int32_t rank = 0, world = 1;
@@ -240,6 +241,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "filter32") {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "filter32 must be 0 or 1");
         ctx->filter32 = static_cast<int>(value);
+    } else if (k == "sampler") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "sampler must be 0 or 1");
+        ctx->sampler = static_cast<int>(value);
     } else if (k == "theta_mode") {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_mode must be 0 or 1");
         ctx->theta_mode = static_cast<int>(value);
@@ -356,12 +360,18 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     lda_canonical_bases(V, ctx->world, ctx->rank, all.data(), cbase.data(), &run);
     ctx->T_global = run;
 
+    lda::DevState &S = ctx->S;
+    S.K = K;
+    S.exclude_self = ctx->exclude_self;
+    S.filter32 = ctx->filter32;
+    S.sampler = ctx->sampler;
+    KL(lda::configure_kernels(S));
+
     lda::HostLayout &H = ctx->H;
     std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
-                                      ctx->chunk_tokens, ctx->recount_tokens, ctx->threads, H);
+                                      ctx->chunk_tokens, ctx->recount_tokens, ctx->threads, S.sweep_quad, H);
     if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
 
-    lda::DevState &S = ctx->S;
     S.V = V;
     S.K = K;
     S.D = Dg;
@@ -370,9 +380,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.alpha = ctx->alpha;
     S.beta = ctx->beta;
     S.seed = seed;
-    S.exclude_self = ctx->exclude_self;
-    S.filter32 = ctx->filter32;
-    KL(lda::configure_kernels(S));
 
     DA(S.tok_row, Tg);
     DA(S.tok_z, Tg);
@@ -388,6 +395,11 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     DA(S.rchunks, H.rchunks.size());
     S.n_split = static_cast<int64_t>(H.split_words.size());
     DA(S.split_words, H.split_words.size());
+    S.n_pchunks = static_cast<int64_t>(H.pchunks.size());
+    if (S.sweep_quad) {
+        DA(S.pchunks, H.pchunks.size());
+        DA(S.pairs, H.pairs.size());
+    }
     DA(S.rows, H.rows32 * 8);
     DA(S.nwk, static_cast<size_t>(V) * K + K);
     if (S.sweep_fused) DA(S.nwk_alt, static_cast<size_t>(V) * K + K);
@@ -413,6 +425,10 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(h2d(S.rchunks, H.rchunks.data(), sizeof(lda::RecountChunk) * H.rchunks.size()));
     CU(h2d(S.split_words, H.split_words.data(), sizeof(int32_t) * H.split_words.size()));
     CU(h2d(S.zero_words, H.zero_words.data(), sizeof(int32_t) * H.zero_words.size()));
+    if (S.sweep_quad) {
+        CU(h2d(S.pchunks, H.pchunks.data(), sizeof(lda::PairChunk) * H.pchunks.size()));
+        CU(h2d(S.pairs, H.pairs.data(), sizeof(lda::PairRec) * H.pairs.size()));
+    }
     CU(cudaMemsetAsync(S.rows, 0, H.rows32 * 32, ctx->stream));
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
@@ -425,6 +441,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // host copies no longer needed on the device side (doc_map kept for get_counts)
     std::vector<uint32_t>().swap(H.tok_row);
     std::vector<uint32_t>().swap(H.tok_crank);
+    std::vector<lda::PairRec>().swap(H.pairs);
     ctx->loaded = true;
     ctx->sweeps = 0;
     ctx->stats.local_tokens = Tg;
@@ -456,6 +473,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         ctx->stat_log_cap = n;
     }
     int launches = 0;
+    CU(cudaMemsetAsync(S.stat + 2, 0, sizeof(unsigned long long), ctx->stream));
     for (int32_t s = 0; s < n; ++s) {
         cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
         const uint32_t t = static_cast<uint32_t>(++ctx->sweeps);
@@ -478,6 +496,9 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventRecord(E[5], ctx->stream));
     }
     CU(cudaStreamSynchronize(ctx->stream));
+    unsigned long long n_exact = 0;
+    CU(cudaMemcpy(&n_exact, S.stat + 2, sizeof(n_exact), cudaMemcpyDeviceToHost));
+    ctx->stats.n_exact_redraws = static_cast<int64_t>(n_exact);
     std::vector<unsigned long long> hs(2 * static_cast<size_t>(n));
     if (n)
         CU(cudaMemcpy(hs.data(), ctx->d_stat_log, hs.size() * sizeof(unsigned long long),

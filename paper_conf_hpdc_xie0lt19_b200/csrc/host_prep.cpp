@@ -73,7 +73,7 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
-                         HostLayout &L) {
+                         bool build_pairs, HostLayout &L) {
     const int64_t T = doc_ptr[D];
     L.D = D;
     L.T = T;
@@ -82,8 +82,9 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     nthreads = host_threads(nthreads);
 
     // θ rows: 1 header word (nnz) + capacity min(L_d, K) entries, rounded up
-    // to whole 32-byte sectors; words past nnz are kept zero (zero-mass
-    // padding the sampler may read without a bounds check).
+    // to whole 128-byte lines (the quad sampler reads a row line by line);
+    // words past nnz are kept zero (zero-mass padding the sampler reads
+    // without a bounds check).  Offsets are in 32-byte units.
     L.doc_ptr32.resize(D + 1);
     L.row_off32.resize(D);
     uint64_t off32 = 0;
@@ -92,7 +93,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         int64_t cap = std::min<int64_t>(len, K);
         L.doc_ptr32[d] = static_cast<uint32_t>(doc_ptr[d]);
         L.row_off32[d] = static_cast<uint32_t>(off32);
-        off32 += static_cast<uint64_t>((cap + 1 + 7) / 8);
+        off32 += 4 * static_cast<uint64_t>((cap + 1 + 31) / 32);
         if (off32 >= (uint64_t(1) << 32) - 64) return "θ row storage exceeds 2^32 x 32 bytes";
     }
     L.doc_ptr32[D] = static_cast<uint32_t>(T);
@@ -273,6 +274,73 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     }
     std::stable_sort(L.chunks.begin(), L.chunks.end(),
                      [](const SampleChunk &a, const SampleChunk &b) { return a.count > b.count; });
+
+    // Quad-sampler items: the same word chunks, their tokens (virtual order:
+    // tile by tile, documents by decreasing length) grouped into runs of
+    // equal θ row = (word, doc) pairs of at most 255 tokens.
+    L.pchunks.clear();
+    L.pairs.clear();
+    if (build_pairs) {
+        std::vector<uint16_t> row_cl(L.rows32, 0);  // θ row offset -> capacity in 128-byte lines
+        for (int64_t d = 0; d < D; ++d) {
+            const uint64_t end = d + 1 < D ? L.row_off32[d + 1] : off32;
+            row_cl[L.row_off32[d]] = static_cast<uint16_t>((end - L.row_off32[d]) / 4);
+        }
+        const int64_t nc = static_cast<int64_t>(L.chunks.size());
+        // visit the positions of chunk c in virtual order: f(position)
+        auto walk = [&](const SampleChunk &c, auto &&f) {
+            uint32_t s = c.seg0;
+            for (uint32_t v = c.vbegin; v < c.vbegin + c.count; ++v) {
+                while (L.segs[s + 1].vstart <= v) ++s;
+                f(L.segs[s].pos + (v - L.segs[s].vstart));
+            }
+        };
+        std::vector<uint32_t> np(nc + 1, 0);
+        parallel_for(nthreads, nc, [&](int, int64_t b, int64_t e) {
+            for (int64_t ci = b; ci < e; ++ci) {
+                uint32_t n = 0, prev_row = 0xFFFFFFFFu, m = 0;
+                walk(L.chunks[ci], [&](uint32_t p) {
+                    if (L.tok_row[p] != prev_row || m == 255) {
+                        ++n;
+                        prev_row = L.tok_row[p];
+                        m = 0;
+                    }
+                    ++m;
+                });
+                np[ci + 1] = n;
+            }
+        });
+        for (int64_t ci = 0; ci < nc; ++ci) np[ci + 1] += np[ci];
+        if (np[nc] >= (uint64_t(1) << 32) - 1) return "too many (word, doc) pairs";
+        L.pairs.resize(np[nc]);
+        L.pchunks.resize(nc);
+        parallel_for(nthreads, nc, [&](int, int64_t b, int64_t e) {
+            for (int64_t ci = b; ci < e; ++ci) {
+                const SampleChunk &c = L.chunks[ci];
+                PairRec *out = L.pairs.data() + np[ci];
+                int64_t n = -1;
+                walk(c, [&](uint32_t p) {
+                    const uint32_t row = L.tok_row[p];
+                    if (n < 0 || out[n].row != row || (out[n].mcl & 0xFFu) == 255u) {
+                        ++n;
+                        out[n].row = row;
+                        out[n].crank = L.tok_crank[p];
+                        out[n].pos = p;
+                        out[n].mcl = static_cast<uint32_t>(row_cl[row]) << 8;
+                    }
+                    out[n].mcl += 1;
+                });
+                PairChunk &q = L.pchunks[ci];
+                q.word = c.word;
+                q.pbegin = np[ci];
+                q.npairs = np[ci + 1] - np[ci];
+                q.ntok = c.count;
+                q.split = c.pad & 1u;
+                q.pad = 0;
+                q.c_base = c.c_base;
+            }
+        });
+    }
 
     // Recount work items: per word, pieces of at most recount_tokens.
     L.rchunks.clear();

@@ -232,6 +232,42 @@ __device__ __noinline__ int draw_exact(const uint32_t *rw, uint32_t len, const d
     return lo;
 }
 
+// The same exact walk, inlined (ptxas 12.9 crashes on a call to the
+// __noinline__ version from sweep_quad_kernel).
+__device__ __forceinline__ int draw_exact_inl(const uint32_t *rw, uint32_t len, const double *pstar,
+                                              const double *P, double Q, int K, uint32_t x0) {
+    const uint32_t nblk = (len + 8u) >> 3;
+    double S = 0.0;
+    for (uint32_t b = 0; b < nblk; ++b) {
+        Blk8 u = ld_nc_v8(rw + 8 * b);
+        if (b == 0u) u.w[0] = 0u;  // header word: zero mass
+#pragma unroll
+        for (int e = 0; e < 8; ++e) S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], S);
+    }
+    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
+    if (x < S) {
+        double C = 0.0;
+        int z = -1;
+        for (uint32_t b = 0; z < 0 && b < nblk; ++b) {
+            Blk8 u = ld_nc_v8(rw + 8 * b);
+            if (b == 0u) u.w[0] = 0u;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], C);
+                if (z < 0 && C > x) z = static_cast<int>(u.w[e] >> 16);
+            }
+        }
+        return z < 0 ? K - 1 : z;
+    }
+    int lo = 0, hi = K - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (S + P[mid] > x) hi = mid;
+        else lo = mid + 1;
+    }
+    return lo;
+}
+
 // SMEMP: p*/P in shared memory (LDS addressing); else in a global scratch
 // slice per CTA (large K).
 template <bool EXCL, bool SMEMP, bool F32>
@@ -499,6 +535,354 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
 }
 
 // ---------------------------------------------------------------------------
+// a3 + a4, quad sampler (the default path).
+//
+// Same chunk queue, p*/P prefix and fused recount as sweep_kernel; the
+// tokens of a chunk come as (word, doc) pairs (PairRec): consecutive tokens
+// of the word in one document share the document's θ row, hence S and the
+// sparse prefix of Eq. 6-7 -- one row walk per pair, one draw per token.
+// A warp takes 32 pairs at a time:
+//   H  (lane per pair)  the row header (nnz) of each pair -> its line count.
+//   A  (quad per pair)  four lanes read one 128-byte line of a θ row per
+//      step (lane `sub` holds entries 8·sub .. 8·sub+7 of the line: one
+//      256-bit load each, one L1 wavefront per line instead of one per
+//      32-byte block), each sums its 8 masses n_dk·p*(k) in fp32 from a
+//      4-byte p* table (half the shared-memory bank conflicts of the fp64
+//      table), a quad scan gives the prefix at every 8-entry block end
+//      (kept for kQBlk blocks) and the pair's S.  A register ring of R lines
+//      per lane runs ahead across the quad's four pairs.
+//   B  (lane per pair)  Philox uniform of each of the pair's m tokens,
+//      x = U·(S+Q) in fp64; sparse: binary search of the block-end prefixes
+//      and the sequential rescan of that block (first C > x, X5/X6); dense:
+//      binary search of S + P[k] (P exact fp64).  Every comparison is made
+//      only if it clears the fp32 error bound 2ε; a token with any closer
+//      comparison is redrawn by the exact fp64 walk in the oracle's order
+//      (draw_exact), so the filter never changes a draw except within
+//      fp64 rounding of a boundary (excused within 1e-6).
+//   z store + shared histogram (ϕ recount, fused as in sweep_kernel).
+// ---------------------------------------------------------------------------
+constexpr int kQBlk = 16;            // block-end prefixes kept per pair (blocks of 8 entries)
+constexpr int kQStride = kQBlk + 1;  // odd stride (words): lane-per-pair reads hit distinct banks
+constexpr int kQWarpWords = 32 * 4 + 32 + 32 + 32 * kQStride;  // per warp: recs, S, nnz, blk
+#ifndef LDA_QRING
+#define LDA_QRING 3
+#endif
+#ifndef LDA_QUAD_MINB
+#define LDA_QUAD_MINB 3
+#endif
+#ifndef LDA_QDEBUG
+#define LDA_QDEBUG 0
+#endif
+#if LDA_QDEBUG
+__device__ unsigned long long g_qdbg[8];
+#define QDBG(i) atomicAdd(&g_qdbg[i], 1ull)
+#else
+#define QDBG(i)
+#endif
+
+struct QuadArgs {
+    const PairChunk *chunks;
+    int64_t n_chunks;
+    const uint4 *pairs;
+    uint16_t *z;
+    const uint32_t *rows;
+    const int32_t *nwk;
+    const double *denom;
+    uint32_t *counter;
+    int32_t *nwk_next;
+    int32_t *nk_next;
+    unsigned long long *n_exact;  // tokens redrawn by the exact fp64 walk (statistics)
+    int K;
+    double alpha, beta;
+    uint32_t t;
+    uint32_t key0[10], key1[10];
+};
+
+// p*(k) = (n_wk + β)/(n_k + Vβ) (fp64, and its fp32 rounding p32) and the
+// inclusive prefix P of α·p*(k) in smem (Eq. 8); all threads of the CTA call
+// it; ends with a barrier.
+__device__ __forceinline__ void build_word_prefix(const int32_t *__restrict__ nwk_row,
+                                                  const double *__restrict__ denom, int K, double alpha,
+                                                  double beta, double *pstar, double *P, float *p32,
+                                                  double *s_wtot) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int E = (K + kSweepThreads - 1) / kSweepThreads;
+    const int kb = tid * E;
+    double run = 0.0;
+    for (int e = 0; e < E; ++e) {
+        const int k = kb + e;
+        if (k < K) {
+            const double ps = (static_cast<double>(__ldg(nwk_row + k)) + beta) / __ldg(denom + k);
+            pstar[k] = ps;
+            p32[k] = static_cast<float>(ps);
+            run = run + alpha * ps;
+            P[k] = run;
+        }
+    }
+    double incl = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const double y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+    }
+    double lex = __shfl_up_sync(kFull, incl, 1);
+    if (lane == 0) lex = 0.0;
+    if (lane == 31) s_wtot[warp] = incl;
+    __syncthreads();
+    double off = 0.0;
+    for (int i = 0; i < warp; ++i) off += s_wtot[i];
+    off = off + lex;
+    for (int e = 0; e < E; ++e) {
+        const int k = kb + e;
+        if (k < K) P[k] = off + P[k];
+    }
+    __syncthreads();
+}
+
+// count (low 16 bits of a θ entry) as float, exactly: 2^23 + c - 2^23
+__device__ __forceinline__ float count_f32(uint32_t e) {
+    return __int_as_float(static_cast<int>((e & 0xFFFFu) | 0x4B000000u)) - 8388608.0f;
+}
+__device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc) {
+    return fmaf(count_f32(e), p32[e >> 16], acc);
+}
+
+template <int R>
+__global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kernel(QuadArgs a) {
+    extern __shared__ double smem_d[];
+    __shared__ int s_ci;
+    __shared__ double s_wtot[kSweepThreads / 32];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int q = lane >> 2, sub = lane & 3;
+    const int K = a.K;
+    // smem: [p*: K f64][P: K f64][p32: K f32][hist: K i32][nk partial: K i32] (16-byte aligned end)
+    //       [per warp: recs uint4[32], S f32[32], nnz u32[32], blk f32[32][kQStride]]
+    double *pstar = smem_d;
+    double *P = pstar + K;
+    float *p32 = reinterpret_cast<float *>(P + K);
+    int *hist = reinterpret_cast<int *>(p32 + K);
+    int *nkp = hist + K;
+    uint32_t *wbase = reinterpret_cast<uint32_t *>(smem_d) + ((28 * K + 15) / 16) * 4 + warp * kQWarpWords;
+    uint4 *wR = reinterpret_cast<uint4 *>(wbase);
+    float *wS = reinterpret_cast<float *>(wbase + 128);
+    uint32_t *wN = wbase + 160;
+    float *wB = reinterpret_cast<float *>(wbase + 192);
+    for (int k = tid; k < 2 * K; k += kSweepThreads) hist[k] = 0;
+    int cur_word = -1;
+    unsigned n_exact = 0;
+
+    for (;;) {
+        if (tid == 0) s_ci = static_cast<int>(atomicAdd(a.counter, 1u));
+        __syncthreads();
+        const int ci = s_ci;
+        if (ci >= a.n_chunks) break;
+        const PairChunk ch = a.chunks[ci];
+        if (static_cast<int>(ch.word) != cur_word) {
+            build_word_prefix(a.nwk + static_cast<size_t>(ch.word) * K, a.denom, K, a.alpha, a.beta, pstar, P,
+                              p32, s_wtot);
+            cur_word = static_cast<int>(ch.word);
+        }
+        const double Q = P[K - 1];
+        const uint32_t nb = (ch.npairs + 31u) >> 5;
+
+        for (uint32_t b = static_cast<uint32_t>(warp); b < nb; b += kSweepThreads / 32) {
+            // ---- H: the batch's 32 pair records and their rows' nnz
+            const uint32_t pi = 32u * b + static_cast<uint32_t>(lane);
+            uint4 rec = make_uint4(0u, 0u, 0u, 0u);
+            uint32_t nnz = 0, nl = 0;
+            if (pi < ch.npairs) {
+                rec = ld_nc_v4(a.pairs + ch.pbegin + pi);
+                nnz = __ldg(a.rows + static_cast<size_t>(rec.x) * 8);
+                nl = (nnz + 32u) >> 5;  // 128-byte lines holding words 0..nnz
+            }
+            wR[lane] = rec;
+            wN[lane] = nnz;
+            const uint32_t lines = nl + __shfl_down_sync(kFull, nl, 8) + __shfl_down_sync(kFull, nl, 16) +
+                                   __shfl_down_sync(kFull, nl, 24);
+            const int nsteps = static_cast<int>(__reduce_max_sync(kFull, lane < 8 ? lines : 0u));
+            __syncwarp();
+
+            // ---- A: stream the quad's lines (pair r, line i) through a ring;
+            // pairs j = 8r + q; invalid pairs (nnz of an absent pair = 0 lines)
+            // only at the end.  A lane loads its 32-byte block only if the
+            // block holds a word <= nnz (words past nnz are zero).
+            int ir = 0;
+            uint32_t ii = 0, rwI = wR[q].x, nzI = wN[q], nlI = (pi - lane + q < ch.npairs) ? (nzI + 32u) >> 5 : 0u;
+            if (nlI == 0u) ir = 4;
+            Blk8 ring[R];
+#define LDA_QISSUE(slot)                                                                                  \
+    if (ir < 4) {                                                                                         \
+        if (32u * ii + 8u * sub <= nzI)                                                                   \
+            ring[slot] = ld_nc_v8(a.rows + (static_cast<size_t>(rwI) + 4u * ii + sub) * 8);              \
+        if (++ii >= nlI) {                                                                                \
+            ii = 0;                                                                                       \
+            if (++ir < 4) {                                                                               \
+                const uint32_t jn = 8u * ir + q;                                                          \
+                rwI = wR[jn].x;                                                                           \
+                nzI = wN[jn];                                                                             \
+                nlI = (pi - lane + jn < ch.npairs) ? (nzI + 32u) >> 5 : 0u;                              \
+                if (nlI == 0u) ir = 4;                                                                    \
+            }                                                                                             \
+        }                                                                                                 \
+    }
+#pragma unroll
+            for (int s2 = 0; s2 < R; ++s2) LDA_QISSUE(s2)
+            int cr = 0;
+            uint32_t ci2 = 0, nzC = wN[q], nlC = (pi - lane + q < ch.npairs) ? (nzC + 32u) >> 5 : 0u;
+            if (nlC == 0u) cr = 4;
+            float run = 0.0f;
+            for (int base = 0; base < nsteps; base += R) {
+#pragma unroll
+                for (int s2 = 0; s2 < R; ++s2) {
+                    if (base + s2 >= nsteps) break;
+                    Blk8 u = ring[s2];
+                    LDA_QISSUE(s2)
+                    const bool live = cr < 4;
+                    float sp = 0.0f;
+                    if (live && 32u * ci2 + 8u * sub <= nzC) {
+                        if (ci2 == 0u && sub == 0) u.w[0] = 0u;  // word 0 = nnz header, not an entry
+#pragma unroll
+                        for (int e = 0; e < 8; ++e) sp = entry_mass32(u.w[e], p32, sp);
+                    }
+                    float v = sp;
+                    float y = __shfl_up_sync(kFull, v, 1, 4);
+                    if (sub >= 1) v += y;
+                    y = __shfl_up_sync(kFull, v, 2, 4);
+                    if (sub >= 2) v += y;
+                    const float qt = __shfl_sync(kFull, v, 3, 4);
+                    if (live) {
+                        const int j = 8 * cr + q;
+                        const uint32_t bidx = 4u * ci2 + sub;
+                        if (bidx < static_cast<uint32_t>(kQBlk)) wB[j * kQStride + bidx] = run + v;
+                        run += qt;
+                        if (++ci2 >= nlC) {
+                            if (sub == 0) wS[j] = run;
+                            run = 0.0f;
+                            ci2 = 0;
+                            if (++cr < 4) {
+                                const uint32_t jn = 8u * cr + q;
+                                nzC = wN[jn];
+                                nlC = (pi - lane + jn < ch.npairs) ? (nzC + 32u) >> 5 : 0u;
+                                if (nlC == 0u) cr = 4;
+                            }
+                        }
+                    }
+                }
+            }
+#undef LDA_QISSUE
+            __syncwarp();
+
+            // ---- B: lane `lane` draws the m tokens of pair `lane`
+            const uint32_t m = rec.w & 0xFFu;
+            if (m) {
+                const double S = static_cast<double>(wS[lane]);  // fp32 S', exact in fp64
+                const double tot = S + Q;
+                // fp32 error bounds (first order, u = 2^-24), with nl lines:
+                //   prefix C' at a block end, after the rescan of a block:
+                //     |C' - C| <= (20 + nl)·u·C  (p32 rounding, 8 FFMA of a
+                //     lane block, 2 quad-scan and <= nl running additions,
+                //     8 rescan FFMA);  |S' - S| <= (12 + nl)·u·S
+                //   x = U·(S' + Q):  |x' - x| <= U·|S' - S|
+                //   y = x - S' (dense offset): |y' - y| <= (1 - U)·|S' - S|
+                // A decision is taken only with a margin above its bound
+                // (+ 2^-50·tot for the fp64 roundings); otherwise the token
+                // is redrawn by the exact fp64 walk.
+                const uint32_t nl = (nnz + 32u) >> 5;
+                const double es = static_cast<double>(12u + nl) * 5.9604644775390625e-08 * S;
+                const double ec = static_cast<double>(34u + 2u * nl) * 5.9604644775390625e-08;
+                const double er = 8.8817841970012523e-16 * tot;
+                const uint32_t nblk = (nnz + 8u) >> 3;  // 8-word blocks holding words 0..nnz
+                const int nbl = nblk < static_cast<uint32_t>(kQBlk) ? static_cast<int>(nblk) : kQBlk;
+                const uint32_t *rw = a.rows + static_cast<size_t>(rec.x) * 8;
+                const float *Bp = wB + lane * kQStride;
+                for (uint32_t k = 0; k < m; ++k) {
+                    const uint32_t x0 = philox_x0_sched(ch.c_base + rec.y + k, a.t, a.key0, a.key1);
+                    const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;
+                    const double x = U * tot;
+                    const double y = x - S;
+                    const double ed = (1.0 - U) * es + er;
+                    bool ok = fabs(y) > ed;
+                    QDBG(0);
+                    if (!ok) QDBG(1);
+                    int z = K - 1;
+                    if (ok && y < 0.0) {
+                        // sparse bucket: first stored block end > x, then the
+                        // sequential rescan of that block (past kQBlk: linear)
+                        const double ex = ec * x + er;
+                        int lo = 0, hi = nbl;
+                        while (lo < hi) {
+                            const int mid = (lo + hi) >> 1;
+                            const double c = static_cast<double>(Bp[mid]);
+                            const double d = c - x;
+                            if (fabs(d) <= ex + ec * c) { ok = false; QDBG(2); }
+                            if (d > 0.0) hi = mid;
+                            else lo = mid + 1;
+                        }
+                        float c32 = lo == 0 ? 0.0f : Bp[lo - 1];
+                        z = -1;
+                        for (uint32_t blk = static_cast<uint32_t>(lo); ok && z < 0 && blk < nblk; ++blk) {
+                            Blk8 u = ld_nc_v8(rw + 8 * blk);
+                            if (blk == 0u) u.w[0] = 0u;
+#pragma unroll
+                            for (int e = 0; e < 8; ++e) {
+                                c32 = entry_mass32(u.w[e], p32, c32);
+                                const double c = static_cast<double>(c32);
+                                const double d = c - x;
+                                if (z < 0 && (u.w[e] & 0xFFFFu)) {
+                                    if (fabs(d) <= ex + ec * c) { ok = false; QDBG(3); }
+                                    else if (d > 0.0) z = static_cast<int>(u.w[e] >> 16);
+                                }
+                            }
+                        }
+                        if (z < 0 && ok) { ok = false; QDBG(4); }
+                    } else if (ok) {
+                        // dense bucket: first k with P[k] > y, i.e. S + P[k] > x
+                        // (K-1 if none, X6)
+                        int lo = 0, hi = K - 1;
+                        while (lo < hi) {
+                            const int mid = (lo + hi) >> 1;
+                            const double d = P[mid] - y;
+                            if (fabs(d) <= ed) { ok = false; QDBG(5); }
+                            if (d > 0.0) hi = mid;
+                            else lo = mid + 1;
+                        }
+                        z = lo;
+                    }
+                    if (!ok) {
+                        z = draw_exact_inl(rw, nnz, pstar, P, Q, K, x0);
+                        ++n_exact;
+                    }
+                    a.z[rec.z + k] = static_cast<uint16_t>(z);
+                    atomicAdd(&hist[z], 1);
+                }
+            }
+            __syncwarp();
+        }
+        __syncthreads();
+        // fused n_wk recount (ϕ update, L1273-1285), as in sweep_kernel
+        int32_t *row = a.nwk_next + static_cast<size_t>(ch.word) * K;
+        const bool split = (ch.split & 1u) != 0u;
+        for (int k = tid; k < K; k += kSweepThreads) {
+            const int h = hist[k];
+            if (split) {
+                if (h) atomicAdd(row + k, h);
+            } else {
+                row[k] = h;
+            }
+            nkp[k] += h;
+            hist[k] = 0;
+        }
+        __syncthreads();
+    }
+    for (int k = tid; k < K; k += kSweepThreads)
+        if (nkp[k]) atomicAdd(a.nk_next + k, nkp[k]);
+    if (a.n_exact) {
+        const unsigned tot = __reduce_add_sync(kFull, n_exact);
+        if (lane == 0 && tot) atomicAdd(a.n_exact, static_cast<unsigned long long>(tot));
+    }
+}
+
+// ---------------------------------------------------------------------------
 // a4 epilogue (separate kernel): n_wk / n_k recount from z.
 // ---------------------------------------------------------------------------
 __global__ void zero_rows_kernel(const int32_t *__restrict__ words, int64_t n, int32_t *__restrict__ nwk,
@@ -586,13 +970,14 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
     const int64_t nw = static_cast<int64_t>(gridDim.x) * wpb;
     for (int64_t d = static_cast<int64_t>(blockIdx.x) * wpb + warp; d < D; d += nw) {
         const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1];
+        uint32_t *row = rows + static_cast<size_t>(row_off32[d]) * 8;
+        const uint32_t old_nnz = row[0];  // issued early: its latency overlaps the histogram
         for (uint32_t i = s + lane; i < e; i += 32) {
             const uint32_t k = GATHERED ? z[i] : z[doc_map[i]];
             atomicAdd(&cnt[k], 1u);
             atomicOr(&bits[k >> 5], 1u << (k & 31));
         }
         __syncwarp();
-        uint32_t *row = rows + static_cast<size_t>(row_off32[d]) * 8;
         uint32_t base = 0;
         for (int qb = 0; qb < Kw; qb += 32) {
             const int qq = qb + lane;
@@ -615,9 +1000,9 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
             if (qq < Kw) bits[qq] = 0u;
             base += __shfl_sync(kFull, incl, 31);
         }
-        // zero the words after the last entry up to the 32-byte boundary
-        const uint32_t pad = (8u - ((1u + base) & 7u)) & 7u;
-        if (static_cast<uint32_t>(lane) < pad) row[1 + base + lane] = 0u;
+        // words past the new last entry that held entries before are zeroed:
+        // every word of the row past 1 + nnz stays zero (rows start zeroed)
+        for (uint32_t i = 1u + base + lane; i < 1u + old_nnz; i += 32u) row[i] = 0u;
         if (lane == 0) {
             row[0] = base;
             s_nnz += base;
@@ -733,6 +1118,27 @@ int configure_kernels(DevState &s) {
             return e;
         s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
     }
+    // quad sampler (default): p*/P, histograms and per-warp pair prefixes in smem
+    {
+        const size_t want = static_cast<size_t>((28 * s.K + 15) / 16) * 16 +
+                            sizeof(uint32_t) * (kSweepThreads / 32) * kQWarpWords;
+        s.sweep_quad = s.sampler == 1 && !s.exclude_self && LDA_FUSE &&
+                       want + 2048 <= static_cast<size_t>(max_optin);
+        if (s.sweep_quad) {
+            const void *fn = reinterpret_cast<const void *>(&sweep_quad_kernel<LDA_QRING>);
+            s.quad_smem = want;
+            if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          static_cast<int>(want))) != cudaSuccess)
+                return e;
+            int bps = 1;
+            if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, kSweepThreads, want)) != cudaSuccess)
+                return e;
+            s.quad_grid = s.num_sms * (bps > 0 ? bps : 1);
+            if (!s.sweep_fused) {  // the quad sampler always fuses the recount
+                s.sweep_fused = true;
+            }
+        }
+    }
     // recount
     if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&recount_kernel),
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) != cudaSuccess)
@@ -826,6 +1232,34 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
         a.nwk_next = nullptr;
         a.nk_next = nullptr;
     }
+    if (s.sweep_quad) {
+        QuadArgs qa;
+        qa.chunks = s.pchunks;
+        qa.n_chunks = s.n_pchunks;
+        qa.pairs = reinterpret_cast<const uint4 *>(s.pairs);
+        qa.z = s.tok_z;
+        qa.rows = s.rows;
+        qa.nwk = s.nwk;
+        qa.denom = s.denom;
+        qa.counter = s.counter;
+        qa.nwk_next = a.nwk_next;
+        qa.nk_next = a.nk_next;
+        qa.n_exact = s.stat + 2;
+        qa.K = s.K;
+        qa.alpha = s.alpha;
+        qa.beta = s.beta;
+        qa.t = t;
+        uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
+        for (int r = 0; r < 10; ++r) {
+            qa.key0[r] = k0;
+            qa.key1[r] = k1;
+            k0 += 0x9E3779B9u;
+            k1 += 0xBB67AE85u;
+        }
+        sweep_quad_kernel<LDA_QRING><<<s.quad_grid, kSweepThreads, s.quad_smem, st>>>(qa);
+        ++*launches;
+        return cudaGetLastError();
+    }
     a.chunks = s.chunks;
     a.n_chunks = s.n_chunks;
     a.segs = s.segs;
@@ -862,6 +1296,12 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
     ++*launches;
     return cudaGetLastError();
 }
+
+#if LDA_QDEBUG
+extern "C" int lda_debug_counters(unsigned long long *out) {
+    return cudaMemcpyFromSymbol(out, g_qdbg, sizeof(g_qdbg));
+}
+#endif
 
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);

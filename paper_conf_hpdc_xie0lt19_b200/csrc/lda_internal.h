@@ -45,6 +45,26 @@ struct RecountChunk {
     uint32_t pad[3];
 };
 
+// Quad sampler (sweep_quad_kernel): a word chunk's tokens grouped into
+// (word, doc) pairs -- consecutive tokens of the word in the same document,
+// which share the document's θ row and therefore S and the sparse prefix
+// (Eq. 6-7): one row walk per pair, one Philox draw per token.
+struct PairRec {
+    uint32_t row;    // θ row of the document, in 32-byte units (128-byte aligned)
+    uint32_t crank;  // canonical rank (within its word) of the pair's first token
+    uint32_t pos;    // word-major position of the first token (z[pos .. pos+m))
+    uint32_t mcl;    // m (tokens, 1..255) | row capacity in 128-byte lines << 8
+};
+struct PairChunk {
+    uint32_t word;
+    uint32_t pbegin;  // pairs [pbegin, pbegin + npairs)
+    uint32_t npairs;
+    uint32_t ntok;
+    uint32_t split;   // bit 0: the word is split over several chunks
+    uint32_t pad;
+    uint64_t c_base;  // canonical index of the rank's first token of the word
+};
+
 // Host-side layout of one rank's shard (built by build_layout).
 struct HostLayout {
     int64_t D = 0, T = 0;
@@ -62,6 +82,8 @@ struct HostLayout {
     std::vector<int32_t> split_words;  // words whose row is accumulated atomically (recount)
     std::vector<int32_t> zero_words;   // words split over sampler chunks or without tokens
     std::vector<int64_t> word_count;   // V local tokens per word
+    std::vector<PairChunk> pchunks;    // quad sampler items (same split as `chunks`), heavy-first
+    std::vector<PairRec> pairs;        // their (word, doc) pairs, chunk by chunk
 };
 
 // cbase[w] = canonical index of this rank's first token of word w.
@@ -69,7 +91,7 @@ struct HostLayout {
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
-                         HostLayout &out);
+                         bool build_pairs, HostLayout &out);
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
@@ -103,6 +125,9 @@ struct DevState {
     int64_t n_rchunks = 0;
     int32_t *split_words = nullptr;
     int64_t n_split = 0;
+    PairRec *pairs = nullptr;       // quad sampler: (word, doc) pairs
+    PairChunk *pchunks = nullptr;
+    int64_t n_pchunks = 0;
     // model
     uint32_t *rows = nullptr;       // θ rows, rows32*8 words
     int32_t *nwk = nullptr;         // V*K + K (n_k at offset V*K), the current counts
@@ -111,6 +136,10 @@ struct DevState {
     int64_t n_zero_words = 0;
     bool sweep_fused = false;
     bool sweep_f32 = false;
+    int sampler = 1;                // option: 1 = quad-per-pair sampler, 0 = lane-per-token
+    bool sweep_quad = false;        // the quad sampler is used (sampler 1, fits in smem, no exclude_self)
+    size_t quad_smem = 0;
+    int quad_grid = 0;
     int filter32 = 0;               // option: fp32 filter with exact fp64 fallback
     double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch

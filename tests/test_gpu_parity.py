@@ -74,12 +74,15 @@ def test_tiny_config_free_running_ll_after_100():
     assert np.mean(g.z() != o.z) < 1e-3
 
 
+@pytest.mark.parametrize("sampler", [1, 0])
 @pytest.mark.parametrize("K", [1, 2, 37, 128, 1024])
-def test_k_variants_lockstep(K):
+def test_k_variants_lockstep(K, sampler):
+    """Both samplers (1 = quad per (word, doc) pair, the default; 0 = lane
+    per token) against the oracle."""
     doc_ptr, words = _corpus(600, 700, 60_000, 0.7, 16, 11)
     a, b = 50.0 / K, 0.01
     o = U.oracle_for(600, 700, K, a, b, doc_ptr, words, 5)
-    g = U.gpu_model(600, 700, K, a, b, doc_ptr, words, 5)
+    g = U.gpu_model(600, 700, K, a, b, doc_ptr, words, 5, sampler=sampler)
     assert np.array_equal(g.z(), o.z)
     U.check_counts_equal(g, o)
     bad, unexc = U.lockstep(g, o, 3)
@@ -109,11 +112,17 @@ def test_nytimes_shaped_midsize_many_chunks():
     z_ref = g.z()
     for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
                  dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3),
-                 dict(theta_mode=1), dict(theta_mode=1, tile_tokens=20_000), dict(filter32=1)]:
+                 dict(theta_mode=1), dict(theta_mode=1, tile_tokens=20_000)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
         assert np.array_equal(h.nwk(), g.nwk())
+    # the lane-per-token sampler (and its fp32 filter) on the same corpus
+    for opts in [dict(sampler=0), dict(sampler=0, filter32=1, chunk_tokens=100)]:
+        h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
+        o = U.oracle_for(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed)
+        bad, unexc = U.lockstep(h, o, 3)
+        assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * cfg.T * 3, opts
 
 
 def test_exclude_self_lockstep():
@@ -126,7 +135,8 @@ def test_exclude_self_lockstep():
     assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
-def test_edge_cases():
+@pytest.mark.parametrize("sampler", [1, 0])
+def test_edge_cases(sampler):
     rng = np.random.default_rng(4)
     # empty docs, single-token docs, a 65535-token doc, absent words, D=1
     L_d = np.array([0, 1, 0, 5, 65535, 1, 0, 3] + list(rng.integers(0, 20, 50)), np.int64)
@@ -135,7 +145,7 @@ def test_edge_cases():
     words = rng.integers(0, V // 2, size=doc_ptr[-1]).astype(np.int32)   # words >= 150 absent
     D, K = len(L_d), 40
     o = U.oracle_for(D, V, K, 0.3, 0.02, doc_ptr, words, 77)
-    g = U.gpu_model(D, V, K, 0.3, 0.02, doc_ptr, words, 77, chunk_tokens=64)
+    g = U.gpu_model(D, V, K, 0.3, 0.02, doc_ptr, words, 77, chunk_tokens=64, sampler=sampler)
     assert np.array_equal(g.z(), o.z)
     U.check_counts_equal(g, o)
     bad, unexc = U.lockstep(g, o, 3)
@@ -144,7 +154,7 @@ def test_edge_cases():
     assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
     # D = 1, a single token
     o1 = U.oracle_for(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
-    g1 = U.gpu_model(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
+    g1 = U.gpu_model(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1, sampler=sampler)
     U.lockstep(g1, o1, 5)
 
 
@@ -153,8 +163,8 @@ def test_filter32_is_exact_at_scale():
     for bit: 10 sweeps of a NYTimes-shaped corpus, z compared."""
     cfg = synth.scaled(synth.CONFIGS["nytimes"], 0.01)        # ~1 M tokens
     doc_ptr, words = synth.to_numpy(*synth.generate_config(cfg, "cpu"))[:2]
-    g32 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, filter32=1)
-    g64 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, filter32=0)
+    g32 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, filter32=1, sampler=0)
+    g64 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, filter32=0, sampler=0)
     for _ in range(10):
         g32.iterate(1)
         g64.iterate(1)

@@ -11,7 +11,8 @@ import sys
 
 
 def launches(path):
-    rows = list(csv.reader(open(path)))
+    lines = [l for l in open(path) if l.startswith('"')]   # skip ncu's ==WARNING==/==PROF== lines
+    rows = list(csv.reader(lines))
     hdr = rows[0]
     ix = {h: i for i, h in enumerate(hdr)}
     per = collections.defaultdict(list)
