@@ -96,15 +96,22 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tile_tokens"   split the documents into tiles of about this many tokens
  *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
- *   "sampler"       1 (default): quad sampler -- the tokens of a word chunk
- *                   grouped into (word, document) pairs, four lanes walk
- *                   the pair's θ row line by line (128-byte lines), one
- *                   draw per token; used when K fits its shared-memory
- *                   layout (K <= ~8000) and exclude_self = 0, else 0.
- *                   0: lane-per-token sampler (32-byte row blocks).
- *                   The two differ only in fp64 summation order of the
- *                   sparse prefix (draws differ only within rounding of a
- *                   CDF boundary).
+ *   "sampler"       2 (default): tile sampler -- work items are the tokens
+ *                   of one word inside one document tile, queued tile by
+ *                   tile so the tiles' θ rows stay in L2; one warp per item,
+ *                   the word's p*/dense-prefix table (built once per sweep)
+ *                   bulk-copied to shared memory, four lanes walk a θ row
+ *                   line by line, draws in fp32 certified against rigorous
+ *                   error bounds (uncertain tokens redrawn in fp64).
+ *                   Used when K fits its shared-memory layout and
+ *                   exclude_self = 0, else sampler 0.
+ *                   1: quad sampler over (word, document) pairs.
+ *                   0: lane-per-token fp64 sampler (32-byte row blocks).
+ *                   The samplers differ only in rounding at a CDF boundary
+ *                   (draws differ only within fp64 rounding of it).
+ *   "tail_per_tile" sampler 2: words with fewer than this many tokens per
+ *                   document tile on average are sampled as one corpus-wide
+ *                   item each (default 64; 0 = off)
  *   "filter32"      sampler 0 only.  1: draw each token in fp32 first and
  *                   redo it in fp64 when its uniform lies within the fp32
  *                   error bound of a CDF boundary — results identical to 0

@@ -28,7 +28,8 @@ struct lda_ctx {
     int64_t tile_tokens = 0;
     int theta_mode = 0;
     int filter32 = 0;
-    int sampler = 1;
+    int sampler = 2;
+    int64_t tail_per_tile = 64;
     int threads = 0;
     // distribution
     int32_t rank = 0, world = 1;
@@ -242,8 +243,11 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "filter32 must be 0 or 1");
         ctx->filter32 = static_cast<int>(value);
     } else if (k == "sampler") {
-        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "sampler must be 0 or 1");
+        if (value < 0 || value > 2) return fail(ctx, LDA_EINVAL, "sampler must be 0, 1 or 2");
         ctx->sampler = static_cast<int>(value);
+    } else if (k == "tail_per_tile") {
+        if (value < 0 || value > (int64_t(1) << 30)) return fail(ctx, LDA_EINVAL, "tail_per_tile out of range");
+        ctx->tail_per_tile = value;
     } else if (k == "theta_mode") {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_mode must be 0 or 1");
         ctx->theta_mode = static_cast<int>(value);
@@ -369,7 +373,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
 
     lda::HostLayout &H = ctx->H;
     std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
-                                      ctx->chunk_tokens, ctx->recount_tokens, ctx->threads, S.sweep_quad, H);
+                                      ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
+                                      S.sweep_tile ? 2 : (S.sweep_quad ? 1 : 0), ctx->tail_per_tile, H);
     if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
 
     S.V = V;
@@ -400,6 +405,12 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         DA(S.pchunks, H.pchunks.size());
         DA(S.pairs, H.pairs.size());
     }
+    S.n_titems = static_cast<int64_t>(H.titems.size());
+    if (S.sweep_tile) {
+        DA(S.titems, H.titems.size());
+        DA(S.cbase, V);
+        DA(S.wtab, S.wt_bytes * static_cast<size_t>(V));
+    }
     DA(S.rows, H.rows32 * 8);
     DA(S.nwk, static_cast<size_t>(V) * K + K);
     if (S.sweep_fused) DA(S.nwk_alt, static_cast<size_t>(V) * K + K);
@@ -429,6 +440,10 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         CU(h2d(S.pchunks, H.pchunks.data(), sizeof(lda::PairChunk) * H.pchunks.size()));
         CU(h2d(S.pairs, H.pairs.data(), sizeof(lda::PairRec) * H.pairs.size()));
     }
+    if (S.sweep_tile) {
+        CU(h2d(S.titems, H.titems.data(), sizeof(lda::TileItem) * H.titems.size()));
+        CU(h2d(S.cbase, cbase.data(), sizeof(uint64_t) * V));
+    }
     CU(cudaMemsetAsync(S.rows, 0, H.rows32 * 32, ctx->stream));
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
@@ -442,6 +457,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     std::vector<uint32_t>().swap(H.tok_row);
     std::vector<uint32_t>().swap(H.tok_crank);
     std::vector<lda::PairRec>().swap(H.pairs);
+    std::vector<lda::TileItem>().swap(H.titems);
     ctx->loaded = true;
     ctx->sweeps = 0;
     ctx->stats.local_tokens = Tg;
@@ -608,7 +624,7 @@ int lda_get_counts(lda_ctx *ctx, int32_t *n_wk, int32_t *n_k, int64_t *ndk_ptr, 
             const uint32_t *row = rows.data() + static_cast<size_t>(H.row_off32[d]) * 8;
             if (ndk_ptr) ndk_ptr[d] = pos;
             for (uint32_t j = 0; j < row[0]; ++j, ++pos) {
-                if (ndk_topic) ndk_topic[pos] = static_cast<uint16_t>(row[1 + j] >> 16);
+                if (ndk_topic) ndk_topic[pos] = static_cast<uint16_t>(row[1 + j] >> 18);
                 if (ndk_count) ndk_count[pos] = static_cast<int32_t>(row[1 + j] & 0xFFFFu);
             }
         }

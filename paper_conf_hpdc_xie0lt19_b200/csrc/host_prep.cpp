@@ -73,7 +73,8 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
-                         bool build_pairs, HostLayout &L) {
+                         int sampler, int64_t tail_per_tile, HostLayout &L) {
+    const bool build_pairs = sampler == 1;
     const int64_t T = doc_ptr[D];
     L.D = D;
     L.T = T;
@@ -113,7 +114,30 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         }
     }
     tile_doc.push_back(D);
-    const int nt = static_cast<int>(tile_doc.size()) - 1;
+    const int ndt = static_cast<int>(tile_doc.size()) - 1;  // document tiles
+
+    std::vector<std::vector<uint32_t>> hist(nthreads, std::vector<uint32_t>(V));
+    // Tail words (tile sampler only): words with too few tokens per document
+    // tile to amortise a per-(word, tile) work item get one corpus-wide run
+    // in an extra "tail tile" after the document tiles.
+    std::vector<uint8_t> tail(V, 0);
+    bool any_tail = false;
+    if (sampler == 2 && ndt > 1 && tail_per_tile > 0) {
+        std::vector<int64_t> wc(V, 0);
+        parallel_for(nthreads, T, [&](int t, int64_t b, int64_t e) {
+            auto &h = hist[t];
+            std::fill(h.begin(), h.end(), 0u);
+            for (int64_t i = b; i < e; ++i) h[words[i]]++;
+        });
+        for (int t = 0; t < (T < (1 << 16) ? 1 : nthreads); ++t)
+            for (int32_t w = 0; w < V; ++w) wc[w] += hist[t][w];
+        for (int32_t w = 0; w < V; ++w)
+            if (wc[w] > 0 && wc[w] < tail_per_tile * ndt) {
+                tail[w] = 1;
+                any_tail = true;
+            }
+    }
+    const int nt = ndt + (any_tail ? 1 : 0);
     L.ntiles = nt;
 
     L.tok_row.assign(T, 0);
@@ -122,11 +146,13 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     L.word_count.assign(V, 0);
     std::vector<std::vector<uint32_t>> tile_cnt(nt);
 
-    std::vector<std::vector<uint32_t>> hist(nthreads, std::vector<uint32_t>(V));
+    uint64_t pos = 0;
     for (int b = 0; b < nt; ++b) {
-        const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
+        const bool tail_tile = b == ndt;
+        // document range: a document tile, or all documents for the tail tile
+        const int64_t d0 = tail_tile ? 0 : tile_doc[b], d1 = tail_tile ? D : tile_doc[b + 1];
         const int64_t nd = d1 - d0;
-        const int64_t t0 = doc_ptr[d0];
+        const uint8_t want = tail_tile ? 1 : 0;  // which words this tile holds
         // Processing order inside the tile: documents by decreasing length,
         // so that the 32 tokens a warp draws together (consecutive in a
         // word's run) come from documents of similar length -> similar θ row
@@ -138,14 +164,15 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             return doc_ptr[x + 1] - doc_ptr[x] > doc_ptr[y + 1] - doc_ptr[y];
         });
         // split the tile's docs across threads (contiguous in `ord`)
-        int nth = (doc_ptr[d1] - t0) < (1 << 16) ? 1 : nthreads;
+        int nth = (doc_ptr[d1] - doc_ptr[d0]) < (1 << 16) ? 1 : nthreads;
         std::vector<int64_t> tdoc(nth + 1);
         for (int t = 0; t <= nth; ++t) tdoc[t] = nd * t / nth;
         auto count_part = [&](int t) {
             auto &h = hist[t];
             std::fill(h.begin(), h.end(), 0u);
             for (int64_t k = tdoc[t]; k < tdoc[t + 1]; ++k)
-                for (int64_t i = doc_ptr[ord[k]]; i < doc_ptr[ord[k] + 1]; ++i) h[words[i]]++;
+                for (int64_t i = doc_ptr[ord[k]]; i < doc_ptr[ord[k] + 1]; ++i)
+                    if (tail[words[i]] == want) h[words[i]]++;
         };
         {
             std::vector<std::thread> th;
@@ -156,7 +183,6 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         // segment starts and per-thread scatter bases
         auto &cnt = tile_cnt[b];
         cnt.assign(V, 0);
-        uint64_t pos = static_cast<uint64_t>(t0);
         for (int32_t w = 0; w < V; ++w) {
             tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
             uint64_t run = pos;
@@ -175,6 +201,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                 const int64_t d = ord[k];
                 uint32_t row = L.row_off32[d];
                 for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
+                    if (tail[words[i]] != want) continue;
                     uint32_t p = next[words[i]]++;
                     L.doc_map[i] = p;
                     L.tok_row[p] = row;
@@ -188,6 +215,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             for (auto &x : th) x.join();
         }
     }
+    if (pos != static_cast<uint64_t>(T)) return "internal: token layout does not cover the corpus";
 
     // Canonical rank of every token within its word on this rank, stored at
     // its word-major position: c = cbase[w] + tok_crank[p] (X18).
@@ -224,6 +252,29 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         for (int t = 1; t < nth; ++t) th.emplace_back(rank_part, t);
         rank_part(0);
         for (auto &x : th) x.join();
+    }
+
+    // Tile sampler items: the (tile, word) runs in pieces of at most
+    // chunk_tokens, tile by tile, heavy-first inside each tile.
+    L.titems.clear();
+    if (sampler == 2) {
+        for (int b = 0; b < nt; ++b) {
+            const size_t first = L.titems.size();
+            for (int32_t w = 0; w < V; ++w) {
+                const int64_t n = tile_cnt[b][w];
+                if (n == 0) continue;
+                const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
+                const uint32_t pos = tseg[static_cast<size_t>(b) * V + w];
+                for (int64_t q = 0; q < pieces; ++q) {
+                    const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
+                    L.titems.push_back(TileItem{static_cast<uint32_t>(w), pos + static_cast<uint32_t>(vb),
+                                                static_cast<uint32_t>(ve - vb), static_cast<uint32_t>(b)});
+                }
+            }
+            std::stable_sort(L.titems.begin() + first, L.titems.end(),
+                             [](const TileItem &x, const TileItem &y) { return x.n > y.n; });
+        }
+        if (L.titems.size() >= (uint64_t(1) << 32) - 1) return "too many tile sampler items";
     }
 
     // Per-word runs (tile order) + sentinel; segment index of each word's first run.

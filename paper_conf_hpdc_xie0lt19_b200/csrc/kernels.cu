@@ -18,6 +18,7 @@
 // (Table 1, 0.19-0.33 flop/B, L555-563).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 
 #include "lda_internal.h"
@@ -25,6 +26,10 @@
 namespace lda {
 
 constexpr unsigned kFull = 0xffffffffu;
+// θ row entry: topic << kTS | count (count < 2^16 in bits 0-15, bits 16-17
+// zero), so that e >> 16 is the byte offset 4·topic of the topic in an fp32
+// table.  K <= 16384 (14 topic bits).
+constexpr int kTS = 18;
 constexpr int kSweepThreads = 256;
 constexpr int kMaxBlk = 16;  // block-end prefixes kept per token for the sparse rescan
 #ifndef LDA_RING
@@ -144,7 +149,7 @@ __global__ void prologue_kernel(const int32_t *__restrict__ nk, int K, double Vb
 //   draw     x = U·(S+Q), U = x0·2^-32 from Philox(seed; c, t) (X4, X8, X9)
 //   sparse   x < S: rescan the row, first entry with prefix > x (X5, X6)
 //   dense    else: binary search of the first k with S + P[k] > x (Fig. 5)
-// θ rows: word 0 = nnz, words 1..nnz = topic << 16 | count (ascending topics,
+// θ rows: word 0 = nnz, words 1..nnz = topic << 18 | count (ascending topics,
 // X7), zero words up to the next 32-byte boundary.
 // ---------------------------------------------------------------------------
 struct SweepArgs {
@@ -185,10 +190,10 @@ __device__ __forceinline__ uint32_t philox_x0_sched(uint64_t c, uint32_t t, cons
 
 template <bool EXCL>
 struct Mass {
-    // mass of one θ entry e = topic << 16 | count under the word's p*
+    // mass of one θ entry e = topic << 18 | count under the word's p*
     __device__ __forceinline__ static double fma_into(uint32_t e, const double *__restrict__ pstar, int zo,
                                                       double po_new, double acc) {
-        const uint32_t tp = e >> 16;
+        const uint32_t tp = e >> kTS;
         uint32_t cn = e & 0xFFFFu;
         double p = pstar[tp];
         if (EXCL && static_cast<int>(tp) == zo && cn != 0u) {
@@ -209,7 +214,7 @@ __device__ __noinline__ int draw_exact(const uint32_t *rw, uint32_t len, const d
     for (uint32_t b = 0; b < nblk; ++b) {
         const Blk8 u = ld_nc_v8(rw + 8 * b);
         for (int e = (b == 0 ? 1 : 0); e < 8; ++e)
-            S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], S);
+            S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], S);
     }
     const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
     if (x < S) {
@@ -217,8 +222,8 @@ __device__ __noinline__ int draw_exact(const uint32_t *rw, uint32_t len, const d
         for (uint32_t b = 0; b < nblk; ++b) {
             const Blk8 u = ld_nc_v8(rw + 8 * b);
             for (int e = (b == 0 ? 1 : 0); e < 8; ++e) {
-                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], C);
-                if (C > x) return static_cast<int>(u.w[e] >> 16);
+                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], C);
+                if (C > x) return static_cast<int>(u.w[e] >> kTS);
             }
         }
         return K - 1;
@@ -242,7 +247,7 @@ __device__ __forceinline__ int draw_exact_inl(const uint32_t *rw, uint32_t len, 
         Blk8 u = ld_nc_v8(rw + 8 * b);
         if (b == 0u) u.w[0] = 0u;  // header word: zero mass
 #pragma unroll
-        for (int e = 0; e < 8; ++e) S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], S);
+        for (int e = 0; e < 8; ++e) S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], S);
     }
     const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
     if (x < S) {
@@ -253,8 +258,8 @@ __device__ __forceinline__ int draw_exact_inl(const uint32_t *rw, uint32_t len, 
             if (b == 0u) u.w[0] = 0u;
 #pragma unroll
             for (int e = 0; e < 8; ++e) {
-                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> 16], C);
-                if (z < 0 && C > x) z = static_cast<int>(u.w[e] >> 16);
+                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], C);
+                if (z < 0 && C > x) z = static_cast<int>(u.w[e] >> kTS);
             }
         }
         return z < 0 ? K - 1 : z;
@@ -377,7 +382,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                 // precision plus a bound on its distance to the fp64 walk
                 float S = 0.0f;
 #pragma unroll
-                for (int e = 1; e < 8; ++e) S = fmaf(static_cast<float>(q[0].w[e] & 0xFFFFu), p32[q[0].w[e] >> 16], S);
+                for (int e = 1; e < 8; ++e) S = fmaf(static_cast<float>(q[0].w[e] & 0xFFFFu), p32[q[0].w[e] >> kTS], S);
                 blk32[tid] = S;
                 if (static_cast<uint32_t>(kRing) < nblk) q[0] = ld_nc_v8(rw + 8 * kRing);
                 for (uint32_t base = 0; base < nblk; base += kRing) {
@@ -391,7 +396,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                         if (nx < nblk) q[i] = ld_nc_v8(rw + 8 * nx);
 #pragma unroll
                         for (int e = 0; e < 8; ++e)
-                            S = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> 16], S);
+                            S = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> kTS], S);
                         if (b < kMaxBlk) blk32[b * kSweepThreads + tid] = S;
                     }
                 }
@@ -416,11 +421,11 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
 #pragma unroll
                             for (int e = 0; e < 8; ++e) {
                                 if (b == 0 && e == 0) continue;
-                                C = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> 16], C);
+                                C = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> kTS], C);
                                 const float d = C - xf;
                                 if (z < 0 && ok) {
                                     if (fabsf(d) <= B) ok = false;
-                                    else if (d > 0.0f) z = static_cast<int>(u.w[e] >> 16);
+                                    else if (d > 0.0f) z = static_cast<int>(u.w[e] >> kTS);
                                 }
                             }
                         }
@@ -474,7 +479,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
 #define LDA_STEP(e)                                                   \
     {                                                                 \
         C = Mass<EXCL>::fma_into((e), pstar, zo, po_new, C);          \
-        if (z < 0 && C > x) z = static_cast<int>((e) >> 16);          \
+        if (z < 0 && C > x) z = static_cast<int>((e) >> kTS);          \
     }
                 for (; z < 0 && b < nblk; ++b) {  // one block, or a linear tail past kMaxBlk
                     const Blk8 u = ld_nc_v8(rw + 8 * b);
@@ -639,12 +644,16 @@ __device__ __forceinline__ void build_word_prefix(const int32_t *__restrict__ nw
     __syncthreads();
 }
 
-// count (low 16 bits of a θ entry) as float, exactly: 2^23 + c - 2^23
+// count (low 16 bits of a θ entry) as float, exactly: bits 0x4B00:count = 2^23 + c
 __device__ __forceinline__ float count_f32(uint32_t e) {
-    return __int_as_float(static_cast<int>((e & 0xFFFFu) | 0x4B000000u)) - 8388608.0f;
+    return __uint_as_float(__byte_perm(e, 0x4B00u, 0x5410)) - 8388608.0f;
+}
+// the entry's topic in an fp32 table: byte offset e >> 16 = 4·topic
+__device__ __forceinline__ float tab32(const float *__restrict__ p32, uint32_t e) {
+    return *reinterpret_cast<const float *>(reinterpret_cast<const char *>(p32) + (e >> 16));
 }
 __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc) {
-    return fmaf(count_f32(e), p32[e >> 16], acc);
+    return fmaf(count_f32(e), tab32(p32, e), acc);
 }
 
 template <int R>
@@ -830,7 +839,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kerne
                                 const double d = c - x;
                                 if (z < 0 && (u.w[e] & 0xFFFFu)) {
                                     if (fabs(d) <= ex + ec * c) { ok = false; QDBG(3); }
-                                    else if (d > 0.0) z = static_cast<int>(u.w[e] >> 16);
+                                    else if (d > 0.0) z = static_cast<int>(u.w[e] >> kTS);
                                 }
                             }
                         }
@@ -880,6 +889,585 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kerne
         const unsigned tot = __reduce_add_sync(kFull, n_exact);
         if (lane == 0 && tot) atomicAdd(a.n_exact, static_cast<unsigned long long>(tot));
     }
+}
+
+// ---------------------------------------------------------------------------
+// a3 + a4, tile sampler (sampler 2, the default).
+//
+// Work items are (word, doc tile) runs: the tokens of word w inside one tile
+// of documents, contiguous in the word-major stream (L1189-1191), at most
+// chunk_tokens each, queued tile by tile (heavy-first inside a tile,
+// L1203-1221).  All warps of the GPU work on the same tile at a time, so the
+// θ rows the tile's tokens gather (tens of MB) are read from HBM about once
+// and re-read from the 126 MB L2.  Each WARP owns an item (no CTA barriers):
+//   prologue  p32(k) = (n_wk + β)·fl32(1/(n_k + Vβ)) and the inclusive
+//             prefix P32 of α·p32 in the warp's shared memory (Eq. 8 and the
+//             dense bucket p2 of Eq. 6, shared by the word's tokens, Fig. 6)
+//   walk      32 tokens per batch; a quad (4 lanes) walks one token's θ row
+//             one 128-byte line per step (lane `sub` holds entries
+//             8·sub .. 8·sub+7: one 256-bit load, one L1 wavefront per line),
+//             S = Σ c_j·p32(t_j) (p1 of Eq. 6-7) with the prefix at every
+//             8-entry block end kept in smem (first kTBlk blocks)
+//   draw      lane per token: x = U·(S+Q), U = x0·2^-32 from Philox (X4, X8,
+//             X9); sparse: binary search of the block-end prefixes, rescan of
+//             one block (first C > x, X5/X6); dense: binary search of P32
+//   verify    every comparison above is taken only if its margin exceeds a
+//             rigorous bound on the fp32 error (γ·u terms below); a token
+//             with any closer comparison is redrawn by the warp in fp64 from
+//             the counts (draw_exact_warp) -- so the draw is the exact-
+//             arithmetic draw of Eq. 1, i.e. the oracle's up to fp64 rounding
+//             at a CDF boundary (excused within 1e-6)
+//   recount   z stored, n_wk of the next sweep += 1 (one global reduction per
+//             distinct topic of the batch), n_k in a per-CTA smem histogram
+//             (the ϕ update, L1273-1285, fused)
+// ---------------------------------------------------------------------------
+#ifndef LDA_TRING
+#define LDA_TRING 2
+#endif
+
+struct TileArgs {
+    const TileItem *items;
+    int64_t n_items;
+    const uint64_t *cbase;     // V: canonical index of the rank's first token of each word
+    const uint32_t *tok_row;   // word-major: θ row of the token's doc (32-byte units, 128-byte aligned)
+    const uint32_t *tok_crank; // word-major: canonical rank within the word
+    uint16_t *z;
+    const uint32_t *rows;
+    const int32_t *nwk;        // frozen counts (V*K, n_k after)
+    const double *denom;       // K: n_k + Vβ
+    uint32_t *counter;
+    int32_t *nwk_next;         // zeroed next counts, V*K
+    int32_t *nk_next;          // and n_k
+    unsigned long long *n_exact;
+    int K;
+    double alpha, beta;
+    int lmax;                  // max θ-row lines per batch (per-warp smem)
+    const char *wtab;          // word tables (word_table_kernel), wt_bytes per word
+    uint32_t wt_bytes;
+    uint32_t t;
+    uint32_t key0[10], key1[10];
+};
+
+__device__ __forceinline__ double warp_sum_d(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    return v;
+}
+__device__ __forceinline__ double warp_incl_scan_d(double v, int lane) {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const double y = __shfl_up_sync(kFull, v, o);
+        if (lane >= o) v += y;
+    }
+    return v;
+}
+__device__ __forceinline__ double pstar64(const int32_t *nwk_row, const double *denom, double beta, uint32_t k) {
+    return (static_cast<double>(__ldg(nwk_row + k)) + beta) / __ldg(denom + k);
+}
+
+// Exact (fp64) draw of one token by the whole warp, from the counts in global
+// memory: p*(k) = (n_wk+β)/(n_k+Vβ) as the oracle computes it, S over the
+// doc row, Q = Σ_k α·p*(k) (cached per item in *q64 / *have_q), x = U·(S+Q),
+// then the first bin of [sparse ‖ dense] whose prefix exceeds x (X4-X6).
+// Only the summation order differs from the oracle's.
+__device__ __noinline__ int draw_exact_warp(const int32_t *nwk_row, const double *denom, const uint32_t *rw,
+                                            uint32_t nnz, uint32_t x0, int K, double alpha, double beta,
+                                            double *q64, int *have_q) {
+    const int lane = threadIdx.x & 31;
+    if (!*have_q) {
+        double q = 0.0;
+        for (int k = lane; k < K; k += 32) q += alpha * pstar64(nwk_row, denom, beta, k);
+        *q64 = warp_sum_d(q);
+        *have_q = 1;
+    }
+    double s = 0.0;
+    for (uint32_t j = 1 + lane; j <= nnz; j += 32) {
+        const uint32_t e = __ldg(rw + j);
+        s = fma(static_cast<double>(e & 0xFFFFu), pstar64(nwk_row, denom, beta, e >> kTS), s);
+    }
+    const double S = warp_sum_d(s);
+    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + *q64);
+    if (x < S) {
+        double carry = 0.0;
+        for (uint32_t j0 = 1; j0 <= nnz; j0 += 32) {
+            const uint32_t j = j0 + lane;
+            double m = 0.0;
+            uint32_t tp = 0;
+            if (j <= nnz) {
+                const uint32_t e = __ldg(rw + j);
+                tp = e >> kTS;
+                m = static_cast<double>(e & 0xFFFFu) * pstar64(nwk_row, denom, beta, tp);
+            }
+            const double c = carry + warp_incl_scan_d(m, lane);
+            const unsigned hit = __ballot_sync(kFull, j <= nnz && m > 0.0 && c > x);
+            if (hit) return static_cast<int>(__shfl_sync(kFull, tp, __ffs(hit) - 1));
+            carry = __shfl_sync(kFull, c, 31);
+        }
+        return K - 1;
+    }
+    double carry = S;
+    for (int k0 = 0; k0 < K; k0 += 32) {
+        const int k = k0 + lane;
+        const double m = k < K ? alpha * pstar64(nwk_row, denom, beta, k) : 0.0;
+        const double c = carry + warp_incl_scan_d(m, lane);
+        const unsigned hit = __ballot_sync(kFull, k < K && c > x);
+        if (hit) return k0 + __ffs(hit) - 1;
+        carry = __shfl_sync(kFull, c, 31);
+    }
+    return K - 1;
+}
+
+// Positive normal fp32 <-> fp64 by bit manipulation (ALU pipe instead of the
+// conversion unit).  f2d_pos is exact; d2f_trunc truncates (relative error
+// < 2^-23); values below 2^-126 map to 0.
+__device__ __forceinline__ double f2d_pos(float f) {
+    const uint32_t b = __float_as_uint(f);
+    const uint32_t hi = b ? (b >> 3) + 0x38000000u : 0u;
+    return __hiloint2double(static_cast<int>(hi), static_cast<int>(b << 29));
+}
+__device__ __forceinline__ float d2f_trunc(double d) {
+    const uint32_t hi = static_cast<uint32_t>(__double2hiint(d)), lo = static_cast<uint32_t>(__double2loint(d));
+    return hi < 0x38100000u ? 0.0f : __uint_as_float(((hi - 0x38000000u) << 3) | (lo >> 29));
+}
+// n (0 <= n < 2^31) as double, exactly: (2^52 + n) - 2^52
+__device__ __forceinline__ double i2d_pos(int n) {
+    return __hiloint2double(0x43300000, n) - 4503599627370496.0;
+}
+
+// a3, hoisted out of the sampler: the word table of every word, built once
+// per sweep from the frozen counts (Eq. 8).  p*(k) = (n_wk + β)·(1/(n_k + Vβ))
+// in fp64; p32 = its truncation to fp32 (relative error < 2u, u = 2^-24) for
+// the sparse walk; the dense prefix of α·p* in two levels: Pc[c] = Σ over
+// the 128-topic chunks before c (fp64), L32[k] = the prefix inside k's chunk
+// (fp64, truncated to fp32: error < 2u·L32), Pc[NC] = Q = Σ_k α·p*(k).
+// Layout per word (wt_bytes, a multiple of 16): [Pc: NC+1 doubles, padded
+// to an even count][p32: K4 floats][L32: K4 floats].  One warp per word;
+// lane l holds k = 128c + 4l .. 4l+3 of chunk c.
+__host__ __device__ constexpr int tab_nc2(int K) { return ((K + 127) / 128 + 2) / 2 * 2; }
+__host__ __device__ constexpr size_t tab_bytes(int K) {
+    return static_cast<size_t>(tab_nc2(K)) * 8 + static_cast<size_t>(8) * ((K + 3) & ~3);
+}
+
+template <bool VEC>
+__global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double *__restrict__ denom, int V, int K,
+                                  double alpha, double beta, char *__restrict__ tab) {
+    extern __shared__ double inv64[];
+    const int lane = threadIdx.x & 31;
+    for (int k = threadIdx.x; k < K; k += blockDim.x) inv64[k] = 1.0 / denom[k];
+    __syncthreads();
+    const int K4 = (K + 3) & ~3;
+    const size_t wt = tab_bytes(K);
+    const int nwarp = gridDim.x * (blockDim.x >> 5);
+    for (int w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < V; w += nwarp) {
+        const int32_t *nwk_row = nwk + static_cast<size_t>(w) * K;
+        double *Pc = reinterpret_cast<double *>(tab + wt * w);
+        float *p32 = reinterpret_cast<float *>(Pc + tab_nc2(K));
+        float *L32 = p32 + K4;
+        double carry = 0.0;
+        for (int k0 = 0, c = 0; k0 < K; k0 += 128, ++c) {
+            const int k = k0 + 4 * lane;
+            double a4[4] = {0.0, 0.0, 0.0, 0.0};
+            if (VEC) {
+                if (k < K) {
+                    const int4 n = __ldg(reinterpret_cast<const int4 *>(nwk_row + k));
+                    const double p0 = (i2d_pos(n.x) + beta) * inv64[k], p1 = (i2d_pos(n.y) + beta) * inv64[k + 1];
+                    const double p2 = (i2d_pos(n.z) + beta) * inv64[k + 2], p3 = (i2d_pos(n.w) + beta) * inv64[k + 3];
+                    *reinterpret_cast<float4 *>(p32 + k) =
+                        make_float4(d2f_trunc(p0), d2f_trunc(p1), d2f_trunc(p2), d2f_trunc(p3));
+                    a4[0] = alpha * p0;
+                    a4[1] = alpha * p1;
+                    a4[2] = alpha * p2;
+                    a4[3] = alpha * p3;
+                }
+            } else {
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                    if (k + e < K) {
+                        const double pe = (i2d_pos(__ldg(nwk_row + k + e)) + beta) * inv64[k + e];
+                        p32[k + e] = d2f_trunc(pe);
+                        a4[e] = alpha * pe;
+                    }
+            }
+            const double l0 = a4[0], l1 = l0 + a4[1], l2 = l1 + a4[2], l3 = l2 + a4[3];
+            double incl = l3;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const double y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            double excl = __shfl_up_sync(kFull, incl, 1);
+            if (lane == 0) excl = 0.0;
+            const float f0 = d2f_trunc(excl + l0), f1 = d2f_trunc(excl + l1);
+            const float f2 = d2f_trunc(excl + l2), f3 = d2f_trunc(excl + l3);
+            if (VEC) {
+                if (k < K) *reinterpret_cast<float4 *>(L32 + k) = make_float4(f0, f1, f2, f3);
+            } else {
+                const float ff[4] = {f0, f1, f2, f3};
+#pragma unroll
+                for (int e = 0; e < 4; ++e)
+                    if (k + e < K) L32[k + e] = ff[e];
+            }
+            if (lane == 0) Pc[c] = carry;
+            carry += __shfl_sync(kFull, incl, 31);
+        }
+        if (lane == 0) Pc[(K + 127) / 128] = carry;
+        // zero the padding so that the table bytes are deterministic
+        if (lane == 1 && tab_nc2(K) > (K + 127) / 128 + 1) Pc[tab_nc2(K) - 1] = 0.0;
+        for (int k = K + lane; k < K4; k += 32) {
+            p32[k] = 0.0f;
+            L32[k] = 0.0f;
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    uint32_t done = 0;
+    while (!done) {
+        asm volatile(
+            "{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    }
+}
+// Bulk copy (TMA engine, no LSU wavefronts) global -> this CTA's smem,
+// completion counted on the mbarrier.
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+// Per-warp shared memory of the tile sampler (bytes): the word table, block
+// sums, line table, per-token row / line base, mbarrier.
+__host__ __device__ constexpr size_t tile_warp_bytes(int K, int lmax) {
+    return tab_bytes(K) + static_cast<size_t>(lmax) * (16 + 4 + 4) + 32 * 4 + 16;
+}
+
+template <int R>
+__global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
+    extern __shared__ double smem_dd[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int q = lane >> 2, sub = lane & 3;
+    const int K = a.K;
+    const int K4 = (K + 3) & ~3;
+    const int NC = (K + 127) / 128;
+    const int LM = a.lmax;
+    int *nkh = reinterpret_cast<int *>(smem_dd);
+    char *wb = reinterpret_cast<char *>(nkh + K4) + static_cast<size_t>(warp) * tile_warp_bytes(K, LM);
+    double *Pc = reinterpret_cast<double *>(wb);
+    float *p32 = reinterpret_cast<float *>(Pc + tab_nc2(K));
+    float *L32 = p32 + K4;
+    float *blk = L32 + K4;                 // 4 block sums per line
+    float *lsm = blk + 4 * LM;             // line sums
+    uint32_t *lrow = reinterpret_cast<uint32_t *>(lsm + LM);
+    uint32_t *tcum = lrow + LM;
+    uint64_t *bar = reinterpret_cast<uint64_t *>(tcum + 32);
+    for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
+    if (lane == 0) mbar_init(bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    __syncthreads();
+    unsigned n_exact = 0;
+    int cur_word = -1;
+    uint32_t phase = 0;
+    const double u = 5.9604644775390625e-08;  // fp32 unit roundoff 2^-24
+    // rounding bound of every prefix of the walk: p32 2u + 4-FFMA chain + 1
+    // (block sum) + 2 (quad line sum), accumulated in fp64
+    const double gS = 9.5 * u;
+
+    auto claim = [&]() {
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(a.counter, 1u);
+        return __shfl_sync(kFull, c, 0);
+    };
+    const TileItem none = {0u, 0u, 0u, 0u};
+    uint32_t ci = claim();
+    if (ci >= a.n_items) ci = 0xFFFFFFFFu;
+    TileItem it = ci != 0xFFFFFFFFu ? a.items[ci] : none;
+    uint32_t cn = ci != 0xFFFFFFFFu ? claim() : 0xFFFFFFFFu;
+    TileItem itn = cn < a.n_items ? a.items[cn] : none;
+    if (lane == 0 && cn < a.n_items && itn.word != it.word)
+        prefetch_l2_bulk(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
+    // the batch data of the next batch, loaded one batch ahead
+    uint32_t n_row = 0, n_crank = 0, n_nnz = 0;
+    if (lane < it.n) {
+        n_row = __ldg(a.tok_row + it.pos + lane);
+        n_crank = __ldg(a.tok_crank + it.pos + lane);
+        n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+    }
+    uint32_t b0 = 0;
+    bool new_item = true;
+    const int32_t *nwk_row = nullptr;
+    int32_t *row_next = nullptr;
+    uint64_t cb = 0;
+    double Q64 = 0.0, q64x = 0.0;
+    int have_q = 0;
+    while (ci != 0xFFFFFFFFu) {
+        if (new_item) {
+            if (static_cast<int>(it.word) != cur_word) {
+                // the word's table -> smem by one bulk copy (all lanes are past their last read)
+                __syncwarp();
+                if (lane == 0) {
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                    mbar_arrive_expect_tx(bar, a.wt_bytes);
+                    bulk_g2s(Pc, a.wtab + static_cast<size_t>(it.word) * a.wt_bytes, a.wt_bytes, bar);
+                }
+                mbar_wait(bar, phase);
+                phase ^= 1u;
+                cur_word = static_cast<int>(it.word);
+            }
+            Q64 = Pc[NC];
+            cb = __ldg(a.cbase + it.word);
+            nwk_row = a.nwk + static_cast<size_t>(it.word) * K;
+            row_next = a.nwk_next + static_cast<size_t>(it.word) * K;
+            have_q = 0;
+            new_item = false;
+        }
+        // ---- batch: up to 32 tokens whose θ rows have at most LM lines in total;
+        // consecutive tokens of one document (a (word, doc) pair) share the
+        // walk of its row
+        const uint32_t j = b0 + lane;
+        const bool valid = j < it.n;
+        const uint32_t p = it.pos + j;
+        const uint32_t row = n_row, crank = n_crank, nnz = n_nnz;
+        const uint32_t prow = __shfl_up_sync(kFull, row, 1);
+        const bool dup = valid && lane > 0 && prow == row;
+        const uint32_t nl = valid ? (nnz + 32u) >> 5 : 0u;  // 128-byte lines holding words 0..nnz
+        const uint32_t nlw = dup ? 0u : nl;                  // lines this token walks
+        uint32_t incl = nlw;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const bool take = valid && (incl <= static_cast<uint32_t>(LM) || lane == 0);
+        const int nb = __popc(__ballot_sync(kFull, take));
+        const uint32_t lsum = __shfl_sync(kFull, incl, nb - 1);
+        uint32_t c0 = incl - nlw;
+        {
+            // a duplicate's lines are those of the last non-duplicate lane before it
+            const unsigned heads = __ballot_sync(kFull, !dup);
+            const int hl = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));
+            c0 = __shfl_sync(kFull, c0, hl);
+        }
+        if (take && !dup)
+            for (uint32_t i = 0; i < nl; ++i) lrow[c0 + i] = (row + 4u * i) | (i == 0 ? 0x80000000u : 0u);
+        __syncwarp();
+        // first lines of the walk in flight
+        Blk8 ring[R];
+#pragma unroll
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t L = q + 8u * s2;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) ring[s2].w[e] = 0u;
+            if (L < lsum) ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lrow[L] & 0x7FFFFFFFu) + sub) * 8);
+        }
+        // ---- the next batch: this item's next tokens, else the next item's first
+        const uint32_t b1 = b0 + static_cast<uint32_t>(nb);
+        const bool more = b1 < it.n;
+        const uint32_t nxt_pos = more ? it.pos + b1 : itn.pos;
+        const uint32_t nxt_n = more ? it.n - b1 : (cn < a.n_items ? itn.n : 0u);
+        const bool nxt_valid = static_cast<uint32_t>(lane) < nxt_n;
+        if (nxt_valid) {
+            n_row = __ldg(a.tok_row + nxt_pos + lane);
+            n_crank = __ldg(a.tok_crank + nxt_pos + lane);
+        }
+        // ---- walk: quad q takes lines q, q+8, ... of the batch; lane `sub`
+        // sums entries 8·sub .. 8·sub+7 of the line (two FFMA chains); the
+        // quad's line sum by two xor-shuffles.  Branch-free over the R lines
+        // in flight (a lane past the end sums stale entries and discards them).
+        for (uint32_t base = 0; base < lsum; base += 8u * R) {
+            float bs[R];
+#pragma unroll
+            for (int s2 = 0; s2 < R; ++s2) {
+                const uint32_t L = base + 8u * s2 + q;
+                const uint32_t lr = lrow[min(L, static_cast<uint32_t>(LM) - 1u)];
+                const uint32_t w0 = (sub == 0 && (lr >> 31)) ? 0u : ring[s2].w[0];  // header word
+                float s0 = count_f32(w0) * tab32(p32, w0);
+                float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
+                s0 = entry_mass32(ring[s2].w[2], p32, s0);
+                s1 = entry_mass32(ring[s2].w[3], p32, s1);
+                s0 = entry_mass32(ring[s2].w[4], p32, s0);
+                s1 = entry_mass32(ring[s2].w[5], p32, s1);
+                s0 = entry_mass32(ring[s2].w[6], p32, s0);
+                s1 = entry_mass32(ring[s2].w[7], p32, s1);
+                bs[s2] = s0 + s1;
+            }
+#pragma unroll
+            for (int s2 = 0; s2 < R; ++s2) {
+                const uint32_t Ln = base + 8u * (s2 + R) + q;
+                if (Ln < lsum) ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lrow[Ln] & 0x7FFFFFFFu) + sub) * 8);
+            }
+#pragma unroll
+            for (int s2 = 0; s2 < R; ++s2) {
+                const uint32_t L = base + 8u * s2 + q;
+                float ls = bs[s2] + __shfl_xor_sync(kFull, bs[s2], 1);
+                ls += __shfl_xor_sync(kFull, ls, 2);
+                if (L < lsum) {
+                    blk[4 * L + sub] = bs[s2];
+                    if (sub == 0) lsm[L] = ls;
+                }
+            }
+        }
+        if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+        __syncwarp();
+
+        // ---- draw: lane per token (lanes < nb).  Every search below runs on
+        // the approximate (monotone) prefixes with plain comparisons; the
+        // draw is then certified by the margins of the two prefixes that
+        // bracket x, each against a rigorous bound on its error (the other
+        // prefixes are farther from x by monotonicity); uncertain -> flag.
+        int z = 0;
+        bool flag = false;
+        uint32_t x0 = 0;
+        if (take) {
+            const float *ln = lsm + c0;
+            double S = 0.0;
+            for (uint32_t i = 0; i < nl; ++i) S += f2d_pos(ln[i]);
+            x0 = philox_x0_sched(cb + crank, a.t, a.key0, a.key1);
+            const double U = (__hiloint2double(0x43300000, static_cast<int>(x0)) - 4503599627370496.0) *
+                             2.3283064365386962890625e-10;  // x0·2^-32, exact
+            const double tot = S + Q64;
+            const double x = U * tot;
+            const double eps = 1.0e-13 * tot;        // fp64 roundings of this path
+            const double eX = U * gS * S + eps;      // |x' - x|
+            const double d = S - x;                   // sparse iff > 0
+            if (fabs(d) <= (1.0 - U) * gS * S + eps) {
+                flag = true;
+            } else if (d > 0.0) {
+                // sparse bucket: the line, then the block, whose end prefix first exceeds x
+                double C = 0.0, Cn = 0.0;
+                uint32_t i = 0;
+                for (;; ++i) {
+                    Cn = C + f2d_pos(ln[i]);
+                    if (Cn > x || i + 1 >= nl) break;
+                    C = Cn;
+                }
+                const float *bk = blk + 4 * (c0 + i);
+                uint32_t b = 0;
+                for (; b < 3; ++b) {
+                    const double Cb = C + f2d_pos(bk[b]);
+                    if (Cb > x) {
+                        Cn = Cb;
+                        break;
+                    }
+                    C = Cb;
+                }
+                // certify: C <= x < Cn with margins (C = 0 needs none)
+                flag = (x - C <= gS * C + eX && C > 0.0) || (Cn - x <= gS * Cn + eX);
+                b += 4 * i;
+                // the block's entries in order, relative to r = x - C (fp32):
+                // first e with local prefix s_e > r; certify s_{e-1}, s_e
+                const float r32 = static_cast<float>(x - C);
+                const float eR = static_cast<float>((eX + gS * C + u * (x - C)) * 1.0001 + 1e-30);
+                Blk8 w = ld_nc_v8(a.rows + (static_cast<size_t>(row) + b) * 8);
+                if (b == 0) w.w[0] = 0u;
+                float sl = 0.0f, sp = 0.0f, se = 0.0f;
+                int ez = -1;
+                uint32_t we = 0;
+#pragma unroll
+                for (int e = 0; e < 8; ++e) {
+                    const float sn = entry_mass32(w.w[e], p32, sl);
+                    if (ez < 0 && sn > r32) {
+                        ez = e;
+                        sp = sl;
+                        se = sn;
+                        we = w.w[e];
+                    }
+                    sl = sn;
+                }
+                if (ez < 0) {
+                    flag = true;
+                } else {
+                    flag = flag || (se - r32 <= fmaf(6.2e-7f, se, eR)) ||
+                           (sp > 0.0f && r32 - sp <= fmaf(6.2e-7f, sp, eR));   // (2u + 8u)·s
+                    z = static_cast<int>(we >> kTS);
+                }
+            } else {
+                // dense bucket: first k with P[k] > y = x - S = U·Q - (1-U)·S;
+                // chunk by the fp64 bases Pc, then inside the chunk by L32
+                const double y = U * Q64 - (1.0 - U) * S;
+                const double ey = (1.0 - U) * gS * S + eps;
+                int c = 0;
+                for (int n = NC; n > 1;) {  // last chunk c with Pc[c] <= y
+                    const int h = n >> 1;
+                    if (Pc[c + h] <= y) c += h;
+                    n -= h;
+                }
+                const double r = y - Pc[c];
+                const float r32 = static_cast<float>(r);
+                const float eR = static_cast<float>((ey + u * fabs(r)) * 1.0001 + 1e-30);
+                const int kb = 128 * c, kn = min(K, kb + 128) - kb;
+                int k = 0;  // first k in the chunk with L32 > r (kn - 1 if none)
+                for (int n = kn; n > 1;) {
+                    const int h = n >> 1;
+                    if (L32[kb + k + h - 1] <= r32) k += h;
+                    n -= h;
+                }
+                z = kb + k;
+                // certify the bracket: L[z-1] <= y < L[z] (Pc[c] when k = 0)
+                const float le = L32[z], lp = k > 0 ? L32[z - 1] : 0.0f;
+                flag = (z < K - 1 && le - r32 <= fmaf(1.3e-7f, le, eR)) ||
+                       (k > 0 && r32 - lp <= fmaf(1.3e-7f, lp, eR)) ||
+                       (k == 0 && c > 0 && r <= ey);
+            }
+        }
+        // ---- exact fp64 redraw of the uncertain tokens, one at a time by the warp
+        unsigned fl = __ballot_sync(kFull, flag);
+        while (fl) {
+            const int f = __ffs(fl) - 1;
+            fl &= fl - 1;
+            const uint32_t rf = __shfl_sync(kFull, row, f);
+            const uint32_t nf = __shfl_sync(kFull, nnz, f);
+            const uint32_t xf = __shfl_sync(kFull, x0, f);
+            const int zf = draw_exact_warp(nwk_row, a.denom, a.rows + static_cast<size_t>(rf) * 8, nf, xf, K,
+                                           a.alpha, a.beta, &q64x, &have_q);
+            if (lane == f) z = zf;
+            ++n_exact;
+        }
+        // ---- z and the fused recount
+        if (take) {
+            a.z[p] = static_cast<uint16_t>(z);
+            const unsigned act = __activemask();
+            const unsigned peers = __match_any_sync(act, z);
+            if (lane == __ffs(peers) - 1) {
+                const int c = __popc(peers);
+                atomicAdd(row_next + z, c);
+                atomicAdd(&nkh[z], c);
+            }
+        }
+        __syncwarp();
+        // ---- advance
+        if (more) {
+            b0 = b1;
+        } else {
+            ci = cn < a.n_items ? cn : 0xFFFFFFFFu;
+            if (ci == 0xFFFFFFFFu) break;
+            it = itn;
+            b0 = 0;
+            new_item = true;
+            cn = claim();
+            itn = cn < a.n_items ? a.items[cn] : none;
+            if (lane == 0 && cn < a.n_items && itn.word != it.word)
+                prefetch_l2_bulk(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
+        }
+    }
+    __syncthreads();
+    for (int k = threadIdx.x; k < K; k += blockDim.x)
+        if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
+    if (a.n_exact && lane == 0 && n_exact) atomicAdd(a.n_exact, static_cast<unsigned long long>(n_exact));
 }
 
 // ---------------------------------------------------------------------------
@@ -933,7 +1521,7 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
 // ---------------------------------------------------------------------------
 // a5: θ rebuild.  One warp per document: gather z through the doc-word map,
 // count topics in a per-warp shared histogram + bitmap, then write the row
-// as ascending (topic << 16 | count) entries with a popc scan over the bitmap.
+// as ascending (topic << 18 | count) entries with a popc scan over the bitmap.
 // O(L_d + K/32) per document instead of the paper's dense O(K) row.
 // ---------------------------------------------------------------------------
 // Two-phase variant, phase A: z in document order, zd[i] = z[doc_map[i]]
@@ -994,7 +1582,7 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
                 const int b = __ffs(bw) - 1;
                 bw &= bw - 1;
                 const uint32_t k = static_cast<uint32_t>(qq) * 32 + b;
-                row[1 + pos++] = (k << 16) | cnt[k];
+                row[1 + pos++] = (k << kTS) | cnt[k];
                 cnt[k] = 0u;
             }
             if (qq < Kw) bits[qq] = 0u;
@@ -1139,6 +1727,36 @@ int configure_kernels(DevState &s) {
             }
         }
     }
+    // tile sampler (default): per CTA the n_k histogram, per warp the word
+    // table and the batch scratch; <= 8 warps per CTA
+    {
+        const size_t K4 = static_cast<size_t>((s.K + 3) & ~3);
+        s.tile_lmax = std::max(160, ((s.K + 1 + 31) / 32 + 3) & ~3);
+        const size_t cta = 4 * K4, per_warp = tile_warp_bytes(s.K, s.tile_lmax);
+        int wpc = 0;
+        while (wpc < 8 && cta + per_warp * (wpc + 1) + 1024 <= static_cast<size_t>(max_optin)) ++wpc;
+        s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1;
+        s.wt_bytes = tab_bytes(s.K);
+        if (s.sweep_tile) {
+            const void *fn = reinterpret_cast<const void *>(&sweep_tile_kernel<LDA_TRING>);
+            s.tile_block = 32 * wpc;
+            s.tile_smem = cta + per_warp * wpc;
+            if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          static_cast<int>(s.tile_smem))) != cudaSuccess)
+                return e;
+            int bps = 1;
+            if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, s.tile_block, s.tile_smem)) !=
+                cudaSuccess)
+                return e;
+            s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
+            s.sweep_fused = true;
+            for (const void *f : {reinterpret_cast<const void *>(&word_table_kernel<true>),
+                                  reinterpret_cast<const void *>(&word_table_kernel<false>)})
+                if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) !=
+                    cudaSuccess)
+                    return e;
+        }
+    }
     // recount
     if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&recount_kernel),
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) != cudaSuccess)
@@ -1231,6 +1849,49 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
     } else {
         a.nwk_next = nullptr;
         a.nk_next = nullptr;
+    }
+    if (s.sweep_tile) {
+        // every row of the next n_wk is accumulated (words span tiles)
+        if ((e = cudaMemsetAsync(s.nwk_alt, 0, sizeof(int32_t) * (static_cast<size_t>(s.V) * s.K + s.K), st)) !=
+            cudaSuccess)
+            return e;
+        const int wtb = static_cast<int>(std::min<int64_t>((static_cast<int64_t>(s.V) + 7) / 8, 8 * s.num_sms));
+        if ((s.K & 3) == 0)
+            word_table_kernel<true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta, s.wtab);
+        else
+            word_table_kernel<false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta, s.wtab);
+        ++*launches;
+        TileArgs ta;
+        ta.items = s.titems;
+        ta.n_items = s.n_titems;
+        ta.cbase = s.cbase;
+        ta.tok_row = s.tok_row;
+        ta.tok_crank = s.tok_crank;
+        ta.z = s.tok_z;
+        ta.rows = s.rows;
+        ta.nwk = s.nwk;
+        ta.denom = s.denom;
+        ta.counter = s.counter;
+        ta.nwk_next = s.nwk_alt;
+        ta.nk_next = s.nwk_alt + static_cast<size_t>(s.V) * s.K;
+        ta.n_exact = s.stat + 2;
+        ta.K = s.K;
+        ta.alpha = s.alpha;
+        ta.beta = s.beta;
+        ta.lmax = s.tile_lmax;
+        ta.wtab = s.wtab;
+        ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
+        ta.t = t;
+        uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
+        for (int r = 0; r < 10; ++r) {
+            ta.key0[r] = k0;
+            ta.key1[r] = k1;
+            k0 += 0x9E3779B9u;
+            k1 += 0xBB67AE85u;
+        }
+        sweep_tile_kernel<LDA_TRING><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
+        ++*launches;
+        return cudaGetLastError();
     }
     if (s.sweep_quad) {
         QuadArgs qa;

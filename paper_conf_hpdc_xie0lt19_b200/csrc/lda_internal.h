@@ -65,6 +65,16 @@ struct PairChunk {
     uint64_t c_base;  // canonical index of the rank's first token of the word
 };
 
+// Tile sampler (sweep_tile_kernel) work item: the tokens of one word inside
+// one document tile -- contiguous word-major positions [pos, pos + n) --
+// or a piece of them (at most chunk_tokens).  Items are queued tile by tile.
+struct TileItem {
+    uint32_t word;
+    uint32_t pos;
+    uint32_t n;
+    uint32_t tile;
+};
+
 // Host-side layout of one rank's shard (built by build_layout).
 struct HostLayout {
     int64_t D = 0, T = 0;
@@ -84,6 +94,7 @@ struct HostLayout {
     std::vector<int64_t> word_count;   // V local tokens per word
     std::vector<PairChunk> pchunks;    // quad sampler items (same split as `chunks`), heavy-first
     std::vector<PairRec> pairs;        // their (word, doc) pairs, chunk by chunk
+    std::vector<TileItem> titems;      // tile sampler items: tile-major, heavy-first inside a tile
 };
 
 // cbase[w] = canonical index of this rank's first token of word w.
@@ -91,7 +102,7 @@ struct HostLayout {
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
-                         bool build_pairs, HostLayout &out);
+                         int sampler, int64_t tail_per_tile, HostLayout &out);
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
@@ -128,6 +139,9 @@ struct DevState {
     PairRec *pairs = nullptr;       // quad sampler: (word, doc) pairs
     PairChunk *pchunks = nullptr;
     int64_t n_pchunks = 0;
+    TileItem *titems = nullptr;     // tile sampler items
+    int64_t n_titems = 0;
+    uint64_t *cbase = nullptr;      // V: canonical index of the rank's first token of each word
     // model
     uint32_t *rows = nullptr;       // θ rows, rows32*8 words
     int32_t *nwk = nullptr;         // V*K + K (n_k at offset V*K), the current counts
@@ -136,10 +150,15 @@ struct DevState {
     int64_t n_zero_words = 0;
     bool sweep_fused = false;
     bool sweep_f32 = false;
-    int sampler = 1;                // option: 1 = quad-per-pair sampler, 0 = lane-per-token
+    int sampler = 2;                // option: 2 = tile sampler, 1 = quad-per-pair, 0 = lane-per-token
     bool sweep_quad = false;        // the quad sampler is used (sampler 1, fits in smem, no exclude_self)
     size_t quad_smem = 0;
     int quad_grid = 0;
+    bool sweep_tile = false;        // the tile sampler is used (sampler 2, fits in smem, no exclude_self)
+    size_t tile_smem = 0;
+    int tile_grid = 0, tile_block = 0, tile_lmax = 160;
+    char *wtab = nullptr;           // tile sampler: per-word tables (p32, dense prefix), rebuilt every sweep
+    size_t wt_bytes = 0;
     int filter32 = 0;               // option: fp32 filter with exact fp64 fallback
     double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch

@@ -74,11 +74,11 @@ def test_tiny_config_free_running_ll_after_100():
     assert np.mean(g.z() != o.z) < 1e-3
 
 
-@pytest.mark.parametrize("sampler", [1, 0])
+@pytest.mark.parametrize("sampler", [2, 1, 0])
 @pytest.mark.parametrize("K", [1, 2, 37, 128, 1024])
 def test_k_variants_lockstep(K, sampler):
-    """Both samplers (1 = quad per (word, doc) pair, the default; 0 = lane
-    per token) against the oracle."""
+    """Every sampler (2 = tile sampler, the default; 1 = quad per (word, doc)
+    pair; 0 = lane per token) against the oracle."""
     doc_ptr, words = _corpus(600, 700, 60_000, 0.7, 16, 11)
     a, b = 50.0 / K, 0.01
     o = U.oracle_for(600, 700, K, a, b, doc_ptr, words, 5)
@@ -117,8 +117,8 @@ def test_nytimes_shaped_midsize_many_chunks():
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
         assert np.array_equal(h.nwk(), g.nwk())
-    # the lane-per-token sampler (and its fp32 filter) on the same corpus
-    for opts in [dict(sampler=0), dict(sampler=0, filter32=1, chunk_tokens=100)]:
+    # the other samplers (and the fp32 filter of sampler 0) on the same corpus
+    for opts in [dict(sampler=1), dict(sampler=0), dict(sampler=0, filter32=1, chunk_tokens=100)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         o = U.oracle_for(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed)
         bad, unexc = U.lockstep(h, o, 3)
@@ -135,7 +135,7 @@ def test_exclude_self_lockstep():
     assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
-@pytest.mark.parametrize("sampler", [1, 0])
+@pytest.mark.parametrize("sampler", [2, 1, 0])
 def test_edge_cases(sampler):
     rng = np.random.default_rng(4)
     # empty docs, single-token docs, a 65535-token doc, absent words, D=1
@@ -156,6 +156,33 @@ def test_edge_cases(sampler):
     o1 = U.oracle_for(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1)
     g1 = U.gpu_model(1, 1, 3, 0.5, 0.1, np.array([0, 1]), np.array([0], np.int32), 1, sampler=sampler)
     U.lockstep(g1, o1, 5)
+
+
+def test_tile_sampler_decomposition_and_fallback_rate():
+    """The tile sampler (default) on a ~1 M-token NYTimes-shaped corpus: the
+    draws do not depend on the tile / item decomposition, match the fp64
+    lane-per-token sampler except within fp64 rounding of a CDF boundary,
+    and the fp32 filter sends only a small fraction of tokens to the exact
+    fp64 redraw."""
+    cfg = synth.scaled(synth.CONFIGS["nytimes"], 0.01)
+    doc_ptr, words = synth.to_numpy(*synth.generate_config(cfg, "cpu"))[:2]
+    ga = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=100_000)
+    gb = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=0,
+                     chunk_tokens=77)
+    g0 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, sampler=0)
+    n_exact = 0
+    for _ in range(6):
+        ga.iterate(1)
+        n_exact += ga.stats()["n_exact_redraws"]
+        gb.iterate(1)
+        g0.iterate(1)
+        za = ga.z()
+        assert np.array_equal(za, gb.z())
+        diff = np.count_nonzero(za != g0.z())
+        assert diff <= 1e-6 * cfg.T + 2
+        if diff:                       # keep the chains in lock step
+            g0.set_z(za)
+    assert n_exact <= 2e-3 * cfg.T * 6, n_exact
 
 
 def test_filter32_is_exact_at_scale():

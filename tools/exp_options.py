@@ -61,7 +61,7 @@ def main():
                "sample": round(st["ms_sample"] / n, 3), "theta": round(st["ms_theta"] / n, 3),
                "recount": round(st["ms_recount"] / n, 3), "nnz": round(nnz, 2),
                "sample_GBs": round(bs / (st["ms_sample"] / n / 1e3) / 1e9, 1), "load_s": round(tl, 1),
-               "ll": round(m.loglik(), 5)}
+               "n_exact_per_sweep": st["n_exact_redraws"] / n, "ll": round(m.loglik(), 5)}
         print(json.dumps(out), flush=True)
         m.close()
 
