@@ -75,9 +75,11 @@ typedef struct lda_stats {
     int64_t sum_nnz_doc;    /* Σ_d nnz_d of θ after the last sweep */
     int64_t n_launches;     /* library kernels launched by the last call */
     int64_t n_sample_chunks;/* sampler work items (word chunks) */
-    int64_t n_exact_redraws;/* quad sampler: tokens of the last lda_iterate call
-                               whose fp32 filter margin was too small and that
-                               were redrawn by the exact fp64 walk */
+    int64_t n_exact_redraws;/* samplers 1, 2: tokens of the last lda_iterate
+                               call whose fp32 draw could not be certified and
+                               that were redrawn by the exact fp64 walk */
+    double ms_table;        /* sampler 2: the per-word table kernel (a3), part of
+                               ms_sample; ms_sample - ms_table = sampling kernel */
 } lda_stats;
 
 /* Create a context.  D = global number of documents, V = vocabulary size,
@@ -99,7 +101,7 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "sampler"       2 (default): tile sampler -- work items are the tokens
  *                   of one word inside one document tile, queued tile by
  *                   tile so the tiles' θ rows stay in L2; one warp per item,
- *                   the word's p*/dense-prefix table (built once per sweep)
+ *                   the word's p* and dense-prefix table (built once per sweep)
  *                   bulk-copied to shared memory, four lanes walk a θ row
  *                   line by line, draws in fp32 certified against rigorous
  *                   error bounds (uncertain tokens redrawn in fp64).

@@ -45,7 +45,8 @@ class lda_stats(ctypes.Structure):
                 ("ms_allreduce", ctypes.c_double), ("ms_last_sweep", ctypes.c_double),
                 ("ms_last_sample", ctypes.c_double), ("sum_nnz_tok", ctypes.c_int64),
                 ("sum_nnz_doc", ctypes.c_int64), ("n_launches", ctypes.c_int64),
-                ("n_sample_chunks", ctypes.c_int64), ("n_exact_redraws", ctypes.c_int64)]
+                ("n_sample_chunks", ctypes.c_int64), ("n_exact_redraws", ctypes.c_int64),
+                ("ms_table", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -475,7 +475,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     if (n < 0) return fail(ctx, LDA_EINVAL, "negative sweep count");
     CU(cudaSetDevice(ctx->device));
     lda::DevState &S = ctx->S;
-    const int per = 6;
+    const int per = 7;
     int r = ensure_events(ctx, static_cast<size_t>(per) * std::max(n, 1));
     if (r != LDA_OK) return r;
     if (ctx->stat_log_cap < static_cast<size_t>(n)) {
@@ -494,7 +494,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
         const uint32_t t = static_cast<uint32_t>(++ctx->sweeps);
         CU(cudaEventRecord(E[0], ctx->stream));
-        KL(lda::launch_sweep(S, t, ctx->stream, &launches));
+        KL(lda::launch_sweep(S, t, ctx->stream, &launches, E[6]));
         CU(cudaEventRecord(E[1], ctx->stream));
         if (S.sweep_fused) std::swap(S.nwk, S.nwk_alt);  // the sampler wrote the next counts
         else KL(lda::launch_recount(S, ctx->stream, &launches));
@@ -522,7 +522,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     lda_stats &st = ctx->stats;
     st.last_n = n;
     st.sweeps_done = static_cast<int64_t>(ctx->sweeps);
-    st.ms_total = st.ms_sample = st.ms_recount = st.ms_theta = st.ms_allreduce = 0;
+    st.ms_total = st.ms_sample = st.ms_recount = st.ms_theta = st.ms_allreduce = st.ms_table = 0;
     st.ms_last_sweep = st.ms_last_sample = 0;
     ctx->log_ms.assign(n, 0);
     ctx->log_ms_sample.assign(n, 0);
@@ -535,6 +535,9 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
         float a = 0, b = 0, c = 0, d = 0, tot = 0;
         CU(cudaEventElapsedTime(&a, E[0], E[1]));
+        float tb = 0;
+        CU(cudaEventElapsedTime(&tb, E[0], E[6]));
+        st.ms_table += tb;
         CU(cudaEventElapsedTime(&b, E[1], E[2]));
         CU(cudaEventElapsedTime(&c, E[2], E[3]));
         CU(cudaEventElapsedTime(&tot, E[0], E[5]));

@@ -1827,13 +1827,16 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
     return cudaGetLastError();
 }
 
-int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
+int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     const double Vbeta = static_cast<double>(s.V) * s.beta;
     const int32_t *nk = s.nwk + static_cast<size_t>(s.V) * s.K;
     prologue_kernel<<<(s.K + 255) / 256, 256, 0, st>>>(nk, s.K, Vbeta, s.denom);
     ++*launches;
+    if (!s.sweep_tile && table_done_event &&
+        (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
+        return e;
     if ((e = cudaMemsetAsync(s.counter, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
     SweepArgs a;
     if (s.sweep_fused) {
@@ -1861,6 +1864,8 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches) {
         else
             word_table_kernel<false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta, s.wtab);
         ++*launches;
+        if (table_done_event && (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
+            return e;
         TileArgs ta;
         ta.items = s.titems;
         ta.n_items = s.n_titems;

@@ -178,7 +178,7 @@ int configure_kernels(DevState &s);
 int launch_init(const DevState &s, void *stream);
 int launch_recount(const DevState &s, void *stream, int *launches);
 int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches);
-int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches);
+int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event);
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches);
 
 }  // namespace lda

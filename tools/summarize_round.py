@@ -40,7 +40,7 @@ def main(tag, cfg, bench_path):
     lines += ["## Launch list (ncu `gpu__time_duration.sum`, `--clock-control none`; cold-cache, serialised)", "",
               "The first launches are corpus load (init, recount, θ build); the rest are the sweeps.", "",
               "| kernel | launches | mean ms | share of sweep kernels |", "|---|---|---|---|"]
-    sweep_kernels = {"sweep_kernel", "prologue_kernel", "zero_rows_kernel", "gather_z_kernel", "theta_kernel",
+    sweep_kernels = {"sweep_kernel", "sweep_tile_kernel", "sweep_quad_kernel", "word_table_kernel", "prologue_kernel", "zero_rows_kernel", "gather_z_kernel", "theta_kernel",
                      "recount_kernel"}
     tot = sum(sum(v) for k, v in per.items() if any(s in k for s in sweep_kernels))
     for k, v in sorted(per.items(), key=lambda kv: -sum(kv[1])):
