@@ -265,7 +265,8 @@ def run_b200(args):
     # stream (the per-word table kernel before it is reported separately)
     t_sample = (float(np.sum(log["ms_sample"])) - float(st["ms_table"])) / 1e3
     achieved = b_sample / t_sample / 1e9
-    kernel = "sweep_tile_kernel" if opts.get("sampler", 2) == 2 else "sweep_kernel"
+    smp = opts.get("sampler", -1)
+    kernel = "sweep_tile_kernel" if smp == 2 or (smp == -1 and cfg.K <= 4096) else "sweep_kernel"
     b_sweep = sum(C.bytes_sweep(T_g, D_g, cfg.V, cfg.K, int(a), int(b)) for a, b in
                   zip(log["sum_nnz_tok"], log["sum_nnz_doc"]))
     sweep_gbs = b_sweep / (float(np.sum(log["ms_sweep"])) / 1e3) / 1e9

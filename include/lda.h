@@ -98,15 +98,18 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tile_tokens"   split the documents into tiles of about this many tokens
  *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
- *   "sampler"       2 (default): tile sampler -- work items are the tokens
+ *   "sampler"       -1 (default): 2 if K <= 4096, else 0.
+ *                   2: tile sampler -- work items are the tokens
  *                   of one word inside one document tile, queued tile by
  *                   tile so the tiles' θ rows stay in L2; one warp per item,
  *                   the word's p* and dense-prefix table (built once per sweep)
  *                   bulk-copied to shared memory, four lanes walk a θ row
  *                   line by line, draws in fp32 certified against rigorous
  *                   error bounds (uncertain tokens redrawn in fp64).
- *                   Used when K fits its shared-memory layout and
- *                   exclude_self = 0, else sampler 0.
+ *                   Needs exclude_self = 0 and K within its shared-memory
+ *                   layout (else sampler 0); at K = 8192 its per-warp
+ *                   tables leave too few warps per SM (measured slower
+ *                   than sampler 0, hence the default).
  *                   1: quad sampler over (word, document) pairs.
  *                   0: lane-per-token fp64 sampler (32-byte row blocks).
  *                   The samplers differ only in rounding at a CDF boundary
@@ -114,6 +117,9 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tail_per_tile" sampler 2: words with fewer than this many tokens per
  *                   document tile on average are sampled as one corpus-wide
  *                   item each (default 64; 0 = off)
+ *   "certify_slack" sampler 2, tests only: multiply every certification
+ *                   bound by this factor (default 1) -- more tokens take the
+ *                   exact fp64 redraw; the draws must not change
  *   "filter32"      sampler 0 only.  1: draw each token in fp32 first and
  *                   redo it in fp64 when its uniform lies within the fp32
  *                   error bound of a CDF boundary — results identical to 0

@@ -28,8 +28,9 @@ struct lda_ctx {
     int64_t tile_tokens = 0;
     int theta_mode = 0;
     int filter32 = 0;
-    int sampler = 2;
+    int sampler = -1;  // auto
     int64_t tail_per_tile = 64;
+    int64_t certify_slack = 1;
     int threads = 0;
     // distribution
     int32_t rank = 0, world = 1;
@@ -243,11 +244,14 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "filter32 must be 0 or 1");
         ctx->filter32 = static_cast<int>(value);
     } else if (k == "sampler") {
-        if (value < 0 || value > 2) return fail(ctx, LDA_EINVAL, "sampler must be 0, 1 or 2");
+        if (value < -1 || value > 2) return fail(ctx, LDA_EINVAL, "sampler must be -1 (auto), 0, 1 or 2");
         ctx->sampler = static_cast<int>(value);
     } else if (k == "tail_per_tile") {
         if (value < 0 || value > (int64_t(1) << 30)) return fail(ctx, LDA_EINVAL, "tail_per_tile out of range");
         ctx->tail_per_tile = value;
+    } else if (k == "certify_slack") {
+        if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
+        ctx->certify_slack = value;
     } else if (k == "theta_mode") {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_mode must be 0 or 1");
         ctx->theta_mode = static_cast<int>(value);
@@ -369,6 +373,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.exclude_self = ctx->exclude_self;
     S.filter32 = ctx->filter32;
     S.sampler = ctx->sampler;
+    S.certify_slack = static_cast<double>(ctx->certify_slack);
     KL(lda::configure_kernels(S));
 
     lda::HostLayout &H = ctx->H;

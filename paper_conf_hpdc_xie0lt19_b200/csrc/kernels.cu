@@ -924,6 +924,13 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kerne
 #ifndef LDA_TRING
 #define LDA_TRING 2
 #endif
+#ifndef LDA_TILE_WPC
+#define LDA_TILE_WPC 8
+#endif
+#ifndef LDA_TILE_MAXK
+#define LDA_TILE_MAXK 4096
+#endif
+constexpr int kTileMaxK = LDA_TILE_MAXK;
 
 struct TileArgs {
     const TileItem *items;
@@ -942,6 +949,7 @@ struct TileArgs {
     int K;
     double alpha, beta;
     int lmax;                  // max θ-row lines per batch (per-warp smem)
+    double slack;              // multiplier of every certification bound (1; > 1 only in tests)
     const char *wtab;          // word tables (word_table_kernel), wt_bytes per word
     uint32_t wt_bytes;
     uint32_t t;
@@ -1185,7 +1193,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     const double u = 5.9604644775390625e-08;  // fp32 unit roundoff 2^-24
     // rounding bound of every prefix of the walk: p32 2u + 4-FFMA chain + 1
     // (block sum) + 2 (quad line sum), accumulated in fp64
-    const double gS = 9.5 * u;
+    const double gS = 9.5 * u * a.slack;
 
     auto claim = [&]() {
         uint32_t c = 0;
@@ -1341,9 +1349,10 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
                              2.3283064365386962890625e-10;  // x0·2^-32, exact
             const double tot = S + Q64;
             const double x = U * tot;
-            const double eps = 1.0e-13 * tot;        // fp64 roundings of this path
-            const double eX = U * gS * S + eps;      // |x' - x|
-            const double d = S - x;                   // sparse iff > 0
+            const double eps = 1.0e-13 * tot * a.slack;  // fp64 roundings of this path
+            const double eX = U * gS * S + eps;          // |x' - x|
+            const double d = S - x;                       // sparse iff > 0
+            const float g32 = static_cast<float>(a.slack);
             if (fabs(d) <= (1.0 - U) * gS * S + eps) {
                 flag = true;
             } else if (d > 0.0) {
@@ -1391,8 +1400,8 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
                 if (ez < 0) {
                     flag = true;
                 } else {
-                    flag = flag || (se - r32 <= fmaf(6.2e-7f, se, eR)) ||
-                           (sp > 0.0f && r32 - sp <= fmaf(6.2e-7f, sp, eR));   // (2u + 8u)·s
+                    flag = flag || (se - r32 <= fmaf(6.2e-7f * g32, se, eR)) ||
+                           (sp > 0.0f && r32 - sp <= fmaf(6.2e-7f * g32, sp, eR));   // (2u + 8u)·s
                     z = static_cast<int>(we >> kTS);
                 }
             } else {
@@ -1419,8 +1428,8 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
                 z = kb + k;
                 // certify the bracket: L[z-1] <= y < L[z] (Pc[c] when k = 0)
                 const float le = L32[z], lp = k > 0 ? L32[z - 1] : 0.0f;
-                flag = (z < K - 1 && le - r32 <= fmaf(1.3e-7f, le, eR)) ||
-                       (k > 0 && r32 - lp <= fmaf(1.3e-7f, lp, eR)) ||
+                flag = (z < K - 1 && le - r32 <= fmaf(1.3e-7f * g32, le, eR)) ||
+                       (k > 0 && r32 - lp <= fmaf(1.3e-7f * g32, lp, eR)) ||
                        (k == 0 && c > 0 && r <= ey);
             }
         }
@@ -1734,7 +1743,11 @@ int configure_kernels(DevState &s) {
         s.tile_lmax = std::max(160, ((s.K + 1 + 31) / 32 + 3) & ~3);
         const size_t cta = 4 * K4, per_warp = tile_warp_bytes(s.K, s.tile_lmax);
         int wpc = 0;
-        while (wpc < 8 && cta + per_warp * (wpc + 1) + 1024 <= static_cast<size_t>(max_optin)) ++wpc;
+        while (wpc < LDA_TILE_WPC && cta + per_warp * (wpc + 1) + 1024 <= static_cast<size_t>(max_optin)) ++wpc;
+        // sampler -1 (auto): the tile sampler up to K = kTileMaxK; at large K its
+        // per-warp tables of 8·K bytes leave too few warps per SM (measured at
+        // K = 8192 on the NYTimes shape: sampler 0 is faster)
+        if (s.sampler < 0) s.sampler = s.K <= kTileMaxK ? 2 : 0;
         s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1;
         s.wt_bytes = tab_bytes(s.K);
         if (s.sweep_tile) {
@@ -1884,6 +1897,7 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.alpha = s.alpha;
         ta.beta = s.beta;
         ta.lmax = s.tile_lmax;
+        ta.slack = s.certify_slack;
         ta.wtab = s.wtab;
         ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
         ta.t = t;

@@ -150,7 +150,7 @@ struct DevState {
     int64_t n_zero_words = 0;
     bool sweep_fused = false;
     bool sweep_f32 = false;
-    int sampler = 2;                // option: 2 = tile sampler, 1 = quad-per-pair, 0 = lane-per-token
+    int sampler = -1;               // option: -1 auto, 2 = tile sampler, 1 = quad-per-pair, 0 = lane-per-token
     bool sweep_quad = false;        // the quad sampler is used (sampler 1, fits in smem, no exclude_self)
     size_t quad_smem = 0;
     int quad_grid = 0;
@@ -159,6 +159,7 @@ struct DevState {
     int tile_grid = 0, tile_block = 0, tile_lmax = 160;
     char *wtab = nullptr;           // tile sampler: per-word tables (p32, dense prefix), rebuilt every sweep
     size_t wt_bytes = 0;
+    double certify_slack = 1.0;     // test option: scales the tile sampler's certification bounds
     int filter32 = 0;               // option: fp32 filter with exact fp64 fallback
     double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch

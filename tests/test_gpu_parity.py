@@ -90,11 +90,13 @@ def test_k_variants_lockstep(K, sampler):
     assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
 
 
-def test_k8192_small():
+@pytest.mark.parametrize("sampler", [-1, 2])
+def test_k8192_small(sampler):
+    """K = 8192: the default (auto -> sampler 0) and the tile sampler forced."""
     doc_ptr, words = _corpus(300, 400, 40_000, 0.7, 64, 12)
     K = 8192
     o = U.oracle_for(300, 400, K, 50.0 / K, 0.01, doc_ptr, words, 9)
-    g = U.gpu_model(300, 400, K, 50.0 / K, 0.01, doc_ptr, words, 9)
+    g = U.gpu_model(300, 400, K, 50.0 / K, 0.01, doc_ptr, words, 9, sampler=sampler)
     bad, unexc = U.lockstep(g, o, 2)
     assert unexc == 0
 
@@ -183,6 +185,34 @@ def test_tile_sampler_decomposition_and_fallback_rate():
         if diff:                       # keep the chains in lock step
             g0.set_z(za)
     assert n_exact <= 2e-3 * cfg.T * 6, n_exact
+
+
+@pytest.mark.parametrize("K", [37, 1024])
+def test_tile_sampler_exact_redraw_path(K):
+    """Inflating the tile sampler's certification bounds (certify_slack) sends
+    most tokens through the warp-collective fp64 redraw; the chains must still
+    match the oracle in lock step (the redraw is the exact path, not a
+    different sampler) and the filtered run."""
+    doc_ptr, words = _corpus(800, 900, 80_000, 0.7, 16, 31)
+    a, b = 50.0 / K, 0.01
+    o = U.oracle_for(800, 900, K, a, b, doc_ptr, words, 6)
+    g = U.gpu_model(800, 900, K, a, b, doc_ptr, words, 6, certify_slack=1 << 20, tile_tokens=20_000)
+    h = U.gpu_model(800, 900, K, a, b, doc_ptr, words, 6, tile_tokens=20_000)
+    n_exact = 0
+    for _ in range(3):
+        margins = o.iterate(1, margins=True)
+        g.iterate(1)
+        h.iterate(1)
+        n_exact += g.stats()["n_exact_redraws"]
+        zg = g.z()
+        bad = np.nonzero(zg != o.z)[0]
+        assert (margins[bad] < U.MARGIN_EXCUSE).all()
+        assert np.count_nonzero(zg != h.z()) <= 2
+        if len(bad):
+            g.set_z(o.z)
+            h.set_z(o.z)
+    assert n_exact > 0.3 * 80_000 * 3, n_exact
+    U.check_counts_equal(g, o)
 
 
 def test_filter32_is_exact_at_scale():
