@@ -922,7 +922,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kerne
 //             (the ϕ update, L1273-1285, fused)
 // ---------------------------------------------------------------------------
 #ifndef LDA_TRING
-#define LDA_TRING 2
+#define LDA_TRING 3
 #endif
 #ifndef LDA_TILE_WPC
 #define LDA_TILE_WPC 8
@@ -1208,13 +1208,58 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     TileItem itn = cn < a.n_items ? a.items[cn] : none;
     if (lane == 0 && cn < a.n_items && itn.word != it.word)
         prefetch_l2_bulk(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
-    // the batch data of the next batch, loaded one batch ahead
-    uint32_t n_row = 0, n_crank = 0, n_nnz = 0;
+    // Batch head (up to 32 tokens whose θ rows have at most LM lines in
+    // total; consecutive tokens of one document -- a (word, doc) pair --
+    // share the walk of its row): line table in smem, first R lines of the
+    // walk in flight.  Built for the next batch before the current batch's
+    // draw, so that its loads overlap the draw.
+    Blk8 ring[R];
+    struct Head {
+        bool take, dup;
+        int nb;
+        uint32_t lsum, c0, nl;
+    };
+    auto head = [&](uint32_t row, uint32_t nnz, bool valid) {
+        Head h;
+        const uint32_t prow = __shfl_up_sync(kFull, row, 1);
+        h.dup = valid && lane > 0 && prow == row;
+        h.nl = valid ? (nnz + 32u) >> 5 : 0u;  // 128-byte lines holding words 0..nnz
+        const uint32_t nlw = h.dup ? 0u : h.nl;
+        uint32_t incl = nlw;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += y;
+        }
+        h.take = valid && (incl <= static_cast<uint32_t>(LM) || lane == 0);
+        h.nb = __popc(__ballot_sync(kFull, h.take));
+        const uint32_t ls = __shfl_sync(kFull, incl, h.nb > 0 ? h.nb - 1 : 0);
+        h.lsum = h.nb > 0 ? ls : 0u;
+        uint32_t c0 = incl - nlw;
+        // a duplicate's lines are those of the last non-duplicate lane before it
+        const unsigned heads = __ballot_sync(kFull, !h.dup);
+        const int hl = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));
+        h.c0 = __shfl_sync(kFull, c0, hl);
+        if (h.take && !h.dup)
+            for (uint32_t i = 0; i < h.nl; ++i) lrow[h.c0 + i] = (row + 4u * i) | (i == 0 ? 0x80000000u : 0u);
+        __syncwarp();
+#pragma unroll
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t L = q + 8u * s2;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) ring[s2].w[e] = 0u;
+            if (L < h.lsum) ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lrow[L] & 0x7FFFFFFFu) + sub) * 8);
+        }
+        return h;
+    };
+    // the first batch
+    uint32_t row = 0, crank = 0, nnz = 0;
     if (lane < it.n) {
-        n_row = __ldg(a.tok_row + it.pos + lane);
-        n_crank = __ldg(a.tok_crank + it.pos + lane);
-        n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+        row = __ldg(a.tok_row + it.pos + lane);
+        crank = __ldg(a.tok_crank + it.pos + lane);
+        nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
     }
+    Head hd = head(row, nnz, static_cast<uint32_t>(lane) < it.n);
     uint32_t b0 = 0;
     bool new_item = true;
     const int32_t *nwk_row = nullptr;
@@ -1243,60 +1288,32 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
             have_q = 0;
             new_item = false;
         }
-        // ---- batch: up to 32 tokens whose θ rows have at most LM lines in total;
-        // consecutive tokens of one document (a (word, doc) pair) share the
-        // walk of its row
-        const uint32_t j = b0 + lane;
-        const bool valid = j < it.n;
-        const uint32_t p = it.pos + j;
-        const uint32_t row = n_row, crank = n_crank, nnz = n_nnz;
-        const uint32_t prow = __shfl_up_sync(kFull, row, 1);
-        const bool dup = valid && lane > 0 && prow == row;
-        const uint32_t nl = valid ? (nnz + 32u) >> 5 : 0u;  // 128-byte lines holding words 0..nnz
-        const uint32_t nlw = dup ? 0u : nl;                  // lines this token walks
-        uint32_t incl = nlw;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(kFull, incl, o);
-            if (lane >= o) incl += y;
-        }
-        const bool take = valid && (incl <= static_cast<uint32_t>(LM) || lane == 0);
-        const int nb = __popc(__ballot_sync(kFull, take));
-        const uint32_t lsum = __shfl_sync(kFull, incl, nb - 1);
-        uint32_t c0 = incl - nlw;
-        {
-            // a duplicate's lines are those of the last non-duplicate lane before it
-            const unsigned heads = __ballot_sync(kFull, !dup);
-            const int hl = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));
-            c0 = __shfl_sync(kFull, c0, hl);
-        }
-        if (take && !dup)
-            for (uint32_t i = 0; i < nl; ++i) lrow[c0 + i] = (row + 4u * i) | (i == 0 ? 0x80000000u : 0u);
-        __syncwarp();
-        // first lines of the walk in flight
-        Blk8 ring[R];
-#pragma unroll
-        for (int s2 = 0; s2 < R; ++s2) {
-            const uint32_t L = q + 8u * s2;
-#pragma unroll
-            for (int e = 0; e < 8; ++e) ring[s2].w[e] = 0u;
-            if (L < lsum) ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lrow[L] & 0x7FFFFFFFu) + sub) * 8);
-        }
+        // ---- this batch
+        const uint32_t p = it.pos + b0 + lane;
+        const bool take = hd.take;
+        const int nb = hd.nb;
+        const uint32_t lsum = hd.lsum, c0 = hd.c0, nl = hd.nl;
         // ---- the next batch: this item's next tokens, else the next item's first
         const uint32_t b1 = b0 + static_cast<uint32_t>(nb);
         const bool more = b1 < it.n;
         const uint32_t nxt_pos = more ? it.pos + b1 : itn.pos;
         const uint32_t nxt_n = more ? it.n - b1 : (cn < a.n_items ? itn.n : 0u);
         const bool nxt_valid = static_cast<uint32_t>(lane) < nxt_n;
+        uint32_t n_row = 0, n_crank = 0, n_nnz = 0;
         if (nxt_valid) {
             n_row = __ldg(a.tok_row + nxt_pos + lane);
             n_crank = __ldg(a.tok_crank + nxt_pos + lane);
         }
+        bool nnz_issued = false;
         // ---- walk: quad q takes lines q, q+8, ... of the batch; lane `sub`
         // sums entries 8·sub .. 8·sub+7 of the line (two FFMA chains); the
         // quad's line sum by two xor-shuffles.  Branch-free over the R lines
         // in flight (a lane past the end sums stale entries and discards them).
         for (uint32_t base = 0; base < lsum; base += 8u * R) {
+            if (base == 8u * R) {  // the next batch's row headers, once its rows have arrived
+                if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+                nnz_issued = true;
+            }
             float bs[R];
 #pragma unroll
             for (int s2 = 0; s2 < R; ++s2) {
@@ -1329,8 +1346,10 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
                 }
             }
         }
-        if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+        if (!nnz_issued && nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
         __syncwarp();
+        // ---- the next batch's head: its line table and first lines, in flight during this draw
+        const Head hn = head(n_row, n_nnz, nxt_valid);
 
         // ---- draw: lane per token (lanes < nb).  Every search below runs on
         // the approximate (monotone) prefixes with plain comparisons; the
@@ -1459,6 +1478,10 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
         }
         __syncwarp();
         // ---- advance
+        row = n_row;
+        crank = n_crank;
+        nnz = n_nnz;
+        hd = hn;
         if (more) {
             b0 = b1;
         } else {
