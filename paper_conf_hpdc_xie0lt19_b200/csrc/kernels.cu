@@ -1560,13 +1560,19 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
 // (independent gathers with high memory-level parallelism, in doc order).
 __global__ void gather_z_kernel(const uint32_t *__restrict__ doc_map, const uint16_t *__restrict__ z,
                                 uint16_t *__restrict__ zd, int64_t T) {
-    const int64_t i0 = (static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x) * 4;
-    if (i0 + 3 < T) {
-        const uint4 m = __ldcs(reinterpret_cast<const uint4 *>(doc_map + i0));
-        const uint16_t a = z[m.x], b = z[m.y], c = z[m.z], d = z[m.w];
-        ushort4 o;
-        o.x = a; o.y = b; o.z = c; o.w = d;
-        *reinterpret_cast<ushort4 *>(zd + i0) = o;
+    // 8 independent gathers per thread (two 16-byte reads of the map)
+    const int64_t i0 = (static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x) * 8;
+    if (i0 + 7 < T) {
+        const uint4 m0 = __ldcs(reinterpret_cast<const uint4 *>(doc_map + i0));
+        const uint4 m1 = __ldcs(reinterpret_cast<const uint4 *>(doc_map + i0 + 4));
+        const uint16_t a0 = z[m0.x], a1 = z[m0.y], a2 = z[m0.z], a3 = z[m0.w];
+        const uint16_t a4 = z[m1.x], a5 = z[m1.y], a6 = z[m1.z], a7 = z[m1.w];
+        uint4 o;
+        o.x = a0 | (static_cast<uint32_t>(a1) << 16);
+        o.y = a2 | (static_cast<uint32_t>(a3) << 16);
+        o.z = a4 | (static_cast<uint32_t>(a5) << 16);
+        o.w = a6 | (static_cast<uint32_t>(a7) << 16);
+        __stcs(reinterpret_cast<uint4 *>(zd + i0), o);
     } else {
         for (int64_t i = i0; i < T; ++i) zd[i] = z[doc_map[i]];
     }
@@ -1850,7 +1856,7 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
     cudaError_t e;
     if ((e = cudaMemsetAsync(stat_out, 0, 2 * sizeof(unsigned long long), st)) != cudaSuccess) return e;
     if (s.z_doc) {
-        const int64_t thr = (s.T + 3) / 4;
+        const int64_t thr = (s.T + 7) / 8;
         gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, st>>>(s.doc_map, s.tok_z, s.z_doc, s.T);
         ++*launches;
         theta_kernel<true><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.doc_map,

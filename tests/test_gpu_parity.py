@@ -245,3 +245,18 @@ def test_set_z_and_determinism():
     g3.iterate(2)
     assert np.array_equal(g1.z(), g3.z())
     assert np.array_equal(g1.nwk(), g3.nwk())
+
+
+def test_convergence_harness_ll_rises():
+    """the LL-vs-time harness on the tiny config — time
+    accumulates and the per-token LL rises from the random initialisation."""
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "convergence", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                                    "tools", "convergence.py"))
+    conv = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(conv)
+    pts = conv.run("tiny", sweeps=20, every=5, device_index=0, quiet=True)
+    assert [p["sweep"] for p in pts] == [0, 5, 10, 15, 20]
+    assert all(b["ms"] > a["ms"] for a, b in zip(pts, pts[1:]))
+    assert pts[-1]["ll_per_token"] > pts[0]["ll_per_token"] + 0.05
