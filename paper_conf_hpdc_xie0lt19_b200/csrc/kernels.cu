@@ -1594,14 +1594,38 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
     __syncwarp();
     unsigned long long s_lnnz = 0, s_nnz = 0;
     const int64_t nw = static_cast<int64_t>(gridDim.x) * wpb;
-    for (int64_t d = static_cast<int64_t>(blockIdx.x) * wpb + warp; d < D; d += nw) {
-        const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1];
-        uint32_t *row = rows + static_cast<size_t>(row_off32[d]) * 8;
+    int64_t d = static_cast<int64_t>(blockIdx.x) * wpb + warp;
+    // the next document's bounds and row, loaded one document ahead
+    uint32_t n_s = 0, n_e = 0, n_off = 0;
+    if (d < D) {
+        n_s = doc_ptr32[d];
+        n_e = doc_ptr32[d + 1];
+        n_off = row_off32[d];
+    }
+    for (; d < D; d += nw) {
+        const uint32_t s = n_s, e = n_e;
+        uint32_t *row = rows + static_cast<size_t>(n_off) * 8;
         const uint32_t old_nnz = row[0];  // issued early: its latency overlaps the histogram
-        for (uint32_t i = s + lane; i < e; i += 32) {
-            const uint32_t k = GATHERED ? z[i] : z[doc_map[i]];
-            atomicAdd(&cnt[k], 1u);
-            atomicOr(&bits[k >> 5], 1u << (k & 31));
+        if (d + nw < D) {
+            n_s = doc_ptr32[d + nw];
+            n_e = doc_ptr32[d + nw + 1];
+            n_off = row_off32[d + nw];
+        }
+        // up to 4 topics per lane in flight, then the shared histogram
+        for (uint32_t i0 = s; i0 < e; i0 += 128) {
+            uint32_t kk[4];
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                const uint32_t i = i0 + 32u * r + lane;
+                kk[r] = i < e ? (GATHERED ? z[i] : z[doc_map[i]]) : 0xFFFFFFFFu;
+            }
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                if (kk[r] != 0xFFFFFFFFu) {
+                    atomicAdd(&cnt[kk[r]], 1u);
+                    atomicOr(&bits[kk[r] >> 5], 1u << (kk[r] & 31));
+                }
+            }
         }
         __syncwarp();
         uint32_t base = 0;
