@@ -335,7 +335,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         return fail(ctx, LDA_EINVAL, "with world == 1 the whole corpus [0, D) must be loaded");
     const int64_t Dg = doc_end - doc_begin;
     bool range_err = false;
+    lda::tmark(nullptr);
     std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err);
+    lda::tmark("validate");
     if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
     if (ctx->K > 16384)
         return fail(ctx, LDA_ERANGE, "K > 16384 is not supported by this build's shared-memory layout");
@@ -349,7 +351,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // Local word histogram -> canonical bases.  c for rank g's tokens of word
     // w starts at Σ_{w'<w} T(w') + Σ_{g'<g} T_{g'}(w)   (X18, §8(c) step 2).
     std::vector<int64_t> local(V, 0);
-    for (int64_t i = 0; i < Tg; ++i) local[words[i]]++;
+    lda::word_histogram(words, Tg, V, ctx->threads, local.data());
     std::vector<int64_t> all(static_cast<size_t>(V) * ctx->world, 0);
     if (ctx->world > 1) {
         int64_t *d_all = nullptr;
@@ -377,6 +379,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     KL(lda::configure_kernels(S));
 
     lda::HostLayout &H = ctx->H;
+    lda::tmark("histogram, streams, configure");
     std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
                                       S.sweep_tile ? 2 : (S.sweep_quad ? 1 : 0), ctx->tail_per_tile, H);
@@ -431,6 +434,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     auto h2d = [&](void *dst, const void *src, size_t bytes) {
         return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream) : cudaSuccess;
     };
+    lda::tmark("device allocation");
     CU(h2d(S.tok_row, H.tok_row.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.doc_map, H.doc_map.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.tok_crank, H.tok_crank.data(), sizeof(uint32_t) * Tg));
@@ -453,16 +457,20 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
     // a1: random init (t = 0), then the count rebuild.
+    CU(cudaStreamSynchronize(ctx->stream));
+    lda::tmark("H2D copies");
     KL(lda::launch_init(S, ctx->stream));
     int launches = 1;
     int r = rebuild_counts(ctx, &launches);
     if (r != LDA_OK) return r;
     CU(cudaStreamSynchronize(ctx->stream));
+    lda::tmark("init + count rebuild");
     // host copies no longer needed on the device side (doc_map kept for get_counts)
-    std::vector<uint32_t>().swap(H.tok_row);
-    std::vector<uint32_t>().swap(H.tok_crank);
+    H.tok_row.release();
+    H.tok_crank.release();
     std::vector<lda::PairRec>().swap(H.pairs);
     std::vector<lda::TileItem>().swap(H.titems);
+    lda::tmark("free host copies");
     ctx->loaded = true;
     ctx->sweeps = 0;
     ctx->stats.local_tokens = Tg;

@@ -2,13 +2,50 @@
 // validation, the word-first token order (L1189-1191), the document-word map
 // (L1297-1303), fixed-capacity θ rows (CSR with short column index,
 // L1235-1243) and the heavy-first work-item tables (L1203-1221).
+#include <sys/mman.h>
+
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <thread>
 
 #include "lda_internal.h"
 
 namespace lda {
+
+template <class T>
+bool HostBuf<T>::allocate(size_t n) {
+    release();
+    const size_t align = size_t(2) << 20;
+    const size_t bytes = (std::max<size_t>(n, 1) * sizeof(T) + align - 1) / align * align;
+    void *q = std::aligned_alloc(align, bytes);
+    if (!q) return false;
+#ifdef MADV_HUGEPAGE
+    madvise(q, bytes, MADV_HUGEPAGE);
+#endif
+    p_ = static_cast<T *>(q);
+    n_ = n;
+    return true;
+}
+template <class T>
+void HostBuf<T>::release() {
+    std::free(p_);
+    p_ = nullptr;
+    n_ = 0;
+}
+template class HostBuf<uint32_t>;
+
+void tmark(const char *what) {
+    static const bool on = std::getenv("LDA_TIMING") != nullptr;
+    static auto last = std::chrono::steady_clock::now();
+    const auto now = std::chrono::steady_clock::now();
+    if (on && what)
+        std::fprintf(stderr, "[lda] %-28s %9.1f ms\n", what,
+                     std::chrono::duration<double, std::milli>(now - last).count());
+    last = now;
+}
 
 int host_threads(int requested) {
     unsigned hw = std::thread::hardware_concurrency();
@@ -31,6 +68,26 @@ static void parallel_for(int nthreads, int64_t n, F f) {
         th.emplace_back([=, &f] { f(t, b, e); });
     }
     for (auto &x : th) x.join();
+}
+
+void word_histogram(const int32_t *words, int64_t T, int32_t V, int nthreads, int64_t *out) {
+    nthreads = host_threads(nthreads);
+    const int nth = T < (1 << 16) ? 1 : nthreads;
+    std::vector<std::vector<uint32_t>> h(nth, std::vector<uint32_t>(V, 0u));
+    std::vector<std::thread> th;
+    auto part = [&](int t) {
+        auto &hh = h[t];
+        const int64_t b = T * t / nth, e = T * (t + 1) / nth;
+        for (int64_t i = b; i < e; ++i) hh[words[i]]++;
+    };
+    for (int t = 1; t < nth; ++t) th.emplace_back(part, t);
+    part(0);
+    for (auto &x : th) x.join();
+    for (int32_t w = 0; w < V; ++w) {
+        int64_t s = 0;
+        for (int t = 0; t < nth; ++t) s += h[t][w];
+        out[w] = s;
+    }
 }
 
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
@@ -116,144 +173,138 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     tile_doc.push_back(D);
     const int ndt = static_cast<int>(tile_doc.size()) - 1;  // document tiles
 
-    std::vector<std::vector<uint32_t>> hist(nthreads, std::vector<uint32_t>(V));
+    // Word counts of the shard (parallel histogram).
+    std::vector<int64_t> wc(V, 0);
+    word_histogram(words, T, V, nthreads, wc.data());
+    L.word_count = wc;
+
     // Tail words (tile sampler only): words with too few tokens per document
     // tile to amortise a per-(word, tile) work item get one corpus-wide run
     // in an extra "tail tile" after the document tiles.
     std::vector<uint8_t> tail(V, 0);
     bool any_tail = false;
-    if (sampler == 2 && ndt > 1 && tail_per_tile > 0) {
-        std::vector<int64_t> wc(V, 0);
-        parallel_for(nthreads, T, [&](int t, int64_t b, int64_t e) {
-            auto &h = hist[t];
-            std::fill(h.begin(), h.end(), 0u);
-            for (int64_t i = b; i < e; ++i) h[words[i]]++;
-        });
-        for (int t = 0; t < (T < (1 << 16) ? 1 : nthreads); ++t)
-            for (int32_t w = 0; w < V; ++w) wc[w] += hist[t][w];
+    if (sampler == 2 && ndt > 1 && tail_per_tile > 0)
         for (int32_t w = 0; w < V; ++w)
             if (wc[w] > 0 && wc[w] < tail_per_tile * ndt) {
                 tail[w] = 1;
                 any_tail = true;
             }
-    }
     const int nt = ndt + (any_tail ? 1 : 0);
     L.ntiles = nt;
 
-    L.tok_row.assign(T, 0);
-    L.doc_map.assign(T, 0);
+    if (!L.tok_row.allocate(T) || !L.doc_map.allocate(T) || !L.tok_crank.allocate(T))
+        return "host allocation of the token tables failed";
+    HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
+    if (!ctmp.allocate(T)) return "host allocation of the token tables failed";
+    // first touch in parallel (every entry is written below)
+    parallel_for(nthreads, T, [&](int, int64_t b, int64_t e) {
+        std::fill(L.tok_row.data() + b, L.tok_row.data() + e, 0u);
+        std::fill(L.doc_map.data() + b, L.doc_map.data() + e, 0u);
+        std::fill(L.tok_crank.data() + b, L.tok_crank.data() + e, 0u);
+        std::fill(ctmp.data() + b, ctmp.data() + e, 0u);
+    });
+    tmark("layout: host tables");
     std::vector<uint32_t> tseg(static_cast<size_t>(nt) * V, 0);  // run start of (tile, word)
-    L.word_count.assign(V, 0);
     std::vector<std::vector<uint32_t>> tile_cnt(nt);
-
-    uint64_t pos = 0;
-    for (int b = 0; b < nt; ++b) {
-        const bool tail_tile = b == ndt;
-        // document range: a document tile, or all documents for the tail tile
-        const int64_t d0 = tail_tile ? 0 : tile_doc[b], d1 = tail_tile ? D : tile_doc[b + 1];
-        const int64_t nd = d1 - d0;
-        const uint8_t want = tail_tile ? 1 : 0;  // which words this tile holds
-        // Processing order inside the tile: documents by decreasing length,
-        // so that the 32 tokens a warp draws together (consecutive in a
-        // word's run) come from documents of similar length -> similar θ row
-        // lengths -> little SIMT divergence.  (The Philox counter does not
-        // depend on this order: each token carries its canonical rank.)
-        std::vector<int64_t> ord(nd);
-        for (int64_t i = 0; i < nd; ++i) ord[i] = d0 + i;
-        std::stable_sort(ord.begin(), ord.end(), [&](int64_t x, int64_t y) {
-            return doc_ptr[x + 1] - doc_ptr[x] > doc_ptr[y + 1] - doc_ptr[y];
-        });
-        // split the tile's docs across threads (contiguous in `ord`)
-        int nth = (doc_ptr[d1] - doc_ptr[d0]) < (1 << 16) ? 1 : nthreads;
-        std::vector<int64_t> tdoc(nth + 1);
-        for (int t = 0; t <= nth; ++t) tdoc[t] = nd * t / nth;
-        auto count_part = [&](int t) {
-            auto &h = hist[t];
-            std::fill(h.begin(), h.end(), 0u);
-            for (int64_t k = tdoc[t]; k < tdoc[t + 1]; ++k)
-                for (int64_t i = doc_ptr[ord[k]]; i < doc_ptr[ord[k] + 1]; ++i)
-                    if (tail[words[i]] == want) h[words[i]]++;
-        };
-        {
-            std::vector<std::thread> th;
-            for (int t = 1; t < nth; ++t) th.emplace_back(count_part, t);
-            count_part(0);
-            for (auto &x : th) x.join();
-        }
-        // segment starts and per-thread scatter bases
-        auto &cnt = tile_cnt[b];
-        cnt.assign(V, 0);
-        for (int32_t w = 0; w < V; ++w) {
-            tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
-            uint64_t run = pos;
-            for (int t = 0; t < nth; ++t) {
-                uint32_t h = hist[t][w];
-                hist[t][w] = static_cast<uint32_t>(run);  // becomes the thread's next position
-                run += h;
-            }
-            cnt[w] = static_cast<uint32_t>(run - pos);
-            L.word_count[w] += cnt[w];
-            pos = run;
-        }
-        auto scatter_part = [&](int t) {
-            auto &next = hist[t];
-            for (int64_t k = tdoc[t]; k < tdoc[t + 1]; ++k) {
-                const int64_t d = ord[k];
-                uint32_t row = L.row_off32[d];
-                for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
-                    if (tail[words[i]] != want) continue;
-                    uint32_t p = next[words[i]]++;
-                    L.doc_map[i] = p;
-                    L.tok_row[p] = row;
-                }
-            }
-        };
-        {
-            std::vector<std::thread> th;
-            for (int t = 1; t < nth; ++t) th.emplace_back(scatter_part, t);
-            scatter_part(0);
-            for (auto &x : th) x.join();
-        }
-    }
-    if (pos != static_cast<uint64_t>(T)) return "internal: token layout does not cover the corpus";
-
-    // Canonical rank of every token within its word on this rank, stored at
-    // its word-major position: c = cbase[w] + tok_crank[p] (X18).
-    L.tok_crank.assign(T, 0);
+    // tail region: after every document tile's segment, word by word
+    int64_t tail_tokens = 0;
+    for (int32_t w = 0; w < V; ++w)
+        if (tail[w]) tail_tokens += wc[w];
+    std::vector<uint32_t> tail_next(V, 0);  // next free position of each tail word
     {
-        const int nth = T < (1 << 16) ? 1 : nthreads;
+        uint64_t tp = static_cast<uint64_t>(T - tail_tokens);
+        if (any_tail) tile_cnt[ndt].assign(V, 0);
+        for (int32_t w = 0; w < V; ++w)
+            if (tail[w]) {
+                tail_next[w] = static_cast<uint32_t>(tp);
+                tseg[static_cast<size_t>(ndt) * V + w] = static_cast<uint32_t>(tp);
+                tile_cnt[ndt][w] = static_cast<uint32_t>(wc[w]);
+                tp += wc[w];
+            }
+    }
+    std::vector<uint32_t> crank_run(V, 0);   // tokens of each word in earlier tiles (canonical order)
+    std::vector<std::vector<uint32_t>> cnt(nthreads, std::vector<uint32_t>(V));
+    std::vector<std::vector<uint32_t>> pnext(nthreads, std::vector<uint32_t>(V));
+    std::vector<std::vector<uint32_t>> cnext(nthreads, std::vector<uint32_t>(V));
+
+    uint64_t pos = 0;  // start of the current tile's segment
+    for (int b = 0; b < ndt; ++b) {
+        const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
+        // the tile's documents in nth contiguous parts (original order), balanced by tokens
+        const int nth = (doc_ptr[d1] - doc_ptr[d0]) < (1 << 16) ? 1 : nthreads;
         std::vector<int64_t> tdoc(nth + 1);
-        for (int t = 0; t <= nth; ++t) tdoc[t] = D * t / nth;
-        auto count_part = [&](int t) {
-            auto &h = hist[t];
+        tdoc[0] = d0;
+        for (int t = 1; t < nth; ++t) {
+            const int64_t target = doc_ptr[d0] + (doc_ptr[d1] - doc_ptr[d0]) * t / nth;
+            tdoc[t] = std::max(tdoc[t - 1], std::lower_bound(doc_ptr + d0, doc_ptr + d1, target) - doc_ptr);
+        }
+        tdoc[nth] = d1;
+        auto run_parts = [&](auto &&f) {
+            std::vector<std::thread> th;
+            for (int t = 1; t < nth; ++t) th.emplace_back(f, t);
+            f(0);
+            for (auto &x : th) x.join();
+        };
+        // count (all words)
+        run_parts([&](int t) {
+            auto &h = cnt[t];
             std::fill(h.begin(), h.end(), 0u);
             for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) h[words[i]]++;
-        };
-        {
-            std::vector<std::thread> th;
-            for (int t = 1; t < nth; ++t) th.emplace_back(count_part, t);
-            count_part(0);
-            for (auto &x : th) x.join();
-        }
+        });
+        // bases: word-major positions (head words: this tile's segment; tail
+        // words: their tail run) and canonical ranks, part by part
+        auto &tc = tile_cnt[b];
+        tc.assign(V, 0);
         for (int32_t w = 0; w < V; ++w) {
-            uint32_t run = 0;
+            uint32_t run_p = tail[w] ? tail_next[w] : static_cast<uint32_t>(pos);
+            uint32_t run_c = crank_run[w];
+            if (!tail[w]) tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
             for (int t = 0; t < nth; ++t) {
-                const uint32_t h = hist[t][w];
-                hist[t][w] = run;
-                run += h;
+                const uint32_t h = cnt[t][w];
+                pnext[t][w] = run_p;
+                cnext[t][w] = run_c;
+                run_p += h;
+                run_c += h;
+            }
+            const uint32_t n = run_c - crank_run[w];
+            crank_run[w] = run_c;
+            if (tail[w]) {
+                tail_next[w] = run_p;
+            } else {
+                tc[w] = n;
+                pos += n;
             }
         }
-        auto rank_part = [&](int t) {
-            auto &next = hist[t];
-            for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i)
-                L.tok_crank[L.doc_map[i]] = next[words[i]]++;
-        };
-        std::vector<std::thread> th;
-        for (int t = 1; t < nth; ++t) th.emplace_back(rank_part, t);
-        rank_part(0);
-        for (auto &x : th) x.join();
+        // scatter: canonical ranks in document order, then positions with the
+        // part's documents by decreasing length, so that the 32 tokens a warp
+        // draws together (consecutive in a word's run) come from documents of
+        // similar length -> similar θ row lengths -> little SIMT divergence.
+        // (The Philox counter does not depend on this order: each token
+        // carries its canonical rank.)
+        run_parts([&](int t) {
+            auto &cn = cnext[t];
+            for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) ctmp[i] = cn[words[i]]++;
+            std::vector<int64_t> ord(tdoc[t + 1] - tdoc[t]);
+            for (size_t k = 0; k < ord.size(); ++k) ord[k] = tdoc[t] + static_cast<int64_t>(k);
+            std::stable_sort(ord.begin(), ord.end(), [&](int64_t x, int64_t y) {
+                return doc_ptr[x + 1] - doc_ptr[x] > doc_ptr[y + 1] - doc_ptr[y];
+            });
+            auto &next = pnext[t];
+            for (const int64_t d : ord) {
+                const uint32_t row = L.row_off32[d];
+                for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
+                    const uint32_t p = next[words[i]]++;
+                    L.doc_map[i] = p;
+                    L.tok_row[p] = row;
+                    L.tok_crank[p] = ctmp[i];
+                }
+            }
+        });
     }
-
+    if (pos != static_cast<uint64_t>(T - tail_tokens)) return "internal: token layout does not cover the corpus";
+    ctmp.release();
+    tmark("layout: tiles (count, ranks, scatter)");
+    tmark("layout: canonical ranks");
     // Tile sampler items: the (tile, word) runs in pieces of at most
     // chunk_tokens, tile by tile, heavy-first inside each tile.
     L.titems.clear();
@@ -277,6 +328,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         if (L.titems.size() >= (uint64_t(1) << 32) - 1) return "too many tile sampler items";
     }
 
+    tmark("layout: tile items");
     // Per-word runs (tile order) + sentinel; segment index of each word's first run.
     L.segs.clear();
     std::vector<uint64_t> wseg0(V + 1);
@@ -326,6 +378,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     std::stable_sort(L.chunks.begin(), L.chunks.end(),
                      [](const SampleChunk &a, const SampleChunk &b) { return a.count > b.count; });
 
+    tmark("layout: runs + sampler chunks");
     // Quad-sampler items: the same word chunks, their tokens (virtual order:
     // tile by tile, documents by decreasing length) grouped into runs of
     // equal θ row = (word, doc) pairs of at most 255 tokens.
@@ -414,6 +467,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     }
     std::stable_sort(L.rchunks.begin(), L.rchunks.end(),
                      [](const RecountChunk &a, const RecountChunk &b) { return a.vcount > b.vcount; });
+    tmark("layout: pairs + recount chunks");
     return "";
 }
 

@@ -8,6 +8,30 @@
 
 namespace lda {
 
+// Owning host array for the large per-token tables: uninitialised, 2 MB
+// aligned with transparent huge pages requested (the layout's random
+// scatters would otherwise miss the TLB on every write), first touched in
+// parallel by the threads that fill it.
+template <class T>
+class HostBuf {
+  public:
+    HostBuf() = default;
+    HostBuf(const HostBuf &) = delete;
+    HostBuf &operator=(const HostBuf &) = delete;
+    ~HostBuf() { release(); }
+    bool allocate(size_t n);   // defined in host_prep.cpp (explicit instantiations)
+    void release();
+    T *data() { return p_; }
+    const T *data() const { return p_; }
+    size_t size() const { return n_; }
+    T &operator[](size_t i) { return p_[i]; }
+    const T &operator[](size_t i) const { return p_[i]; }
+
+  private:
+    T *p_ = nullptr;
+    size_t n_ = 0;
+};
+
 // A run of word w's tokens inside one document tile.  Word w's local tokens
 // have "virtual" indices 0..n_w-1 in (doc, position) order, i.e. canonical
 // order (X18) restricted to this rank; the run stores virtual indices
@@ -83,9 +107,9 @@ struct HostLayout {
     std::vector<uint32_t> doc_ptr32;   // D+1 doc-major token offsets
     std::vector<uint32_t> row_off32;   // D   θ row start, in 32-byte units
     uint64_t rows32 = 0;               // θ row buffer size in 32-byte units (incl. tail pad)
-    std::vector<uint32_t> tok_row;     // T   word-major: θ row (32 B units) of the token's doc
-    std::vector<uint32_t> doc_map;     // T   doc-major token i -> word-major position (S7, L1297-1303)
-    std::vector<uint32_t> tok_crank;   // T   word-major: canonical rank of the token within its word
+    HostBuf<uint32_t> tok_row;         // T   word-major: θ row (32 B units) of the token's doc
+    HostBuf<uint32_t> doc_map;         // T   doc-major token i -> word-major position (S7, L1297-1303)
+    HostBuf<uint32_t> tok_crank;       // T   word-major: canonical rank of the token within its word
     std::vector<Seg> segs;             // per word: its runs, then a sentinel
     std::vector<SampleChunk> chunks;   // heavy-first
     std::vector<RecountChunk> rchunks; // heavy-first
@@ -110,6 +134,13 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
                             bool *range_error);
 
 int host_threads(int requested);
+
+// out[w] = number of tokens of word w (parallel over host threads).
+void word_histogram(const int32_t *words, int64_t T, int32_t V, int nthreads, int64_t *out);
+
+// Phase timer for corpus loading: prints "[lda] <what> <ms>" to stderr when
+// the environment variable LDA_TIMING is set (diagnostics only).
+void tmark(const char *what);
 
 // ---------------------------------------------------------------------------
 // Kernel launchers (kernels.cu).  All return cudaError_t as int.
