@@ -222,10 +222,14 @@ def run_b200(args):
     te0 = time.perf_counter()
     m = make_model()
     m.load(doc_ptr, words, cfg.seed, d0, d1)
+    te1 = time.perf_counter()
     m.iterate(args.steps)
+    te2 = time.perf_counter()
     z_host = m.z()
     barrier()
     te = time.perf_counter() - te0
+    e2e_parts = {"create_load_s": round(te1 - te0, 3), "iterate_s": round(te2 - te1, 3),
+                 "z_d2h_s": round(te0 + te - te2, 3)}
     e2e_times = torch.tensor([te], device=dev, dtype=torch.float64)
     if world > 1:
         dist.all_reduce(e2e_times, op=dist.ReduceOp.MAX)
@@ -317,7 +321,7 @@ def run_b200(args):
             "per_sweep_ms": [round(x, 4) for x in log["ms_sweep"].tolist()],
             "clocks": clocks,
             "e2e": {"value": e2e_value, "unit": "tokens/s", "h2d_bytes_per_step": int(h2d),
-                    "d2h_bytes_per_step": int(d2h),
+                    "d2h_bytes_per_step": int(d2h), "breakdown": e2e_parts,
                     "what": "lda_create+lda_load_corpus(host arrays: H2D, prep, init)+lda_iterate(K)+z D2H"},
             "gpu_launches": int(st["n_launches"]),
             "cpu_baseline": cpu,

@@ -6,6 +6,9 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <condition_variable>
+#include <mutex>
+#include <thread>
 #include <cstdlib>
 #include <cmath>
 #include <cstring>
@@ -379,11 +382,66 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     KL(lda::configure_kernels(S));
 
     lda::HostLayout &H = ctx->H;
+    // the per-token tables go to the device tile by tile, copied by a helper
+    // thread while the host prepares the next tile
+    DA(S.tok_row, Tg);
+    DA(S.doc_map, Tg);
+    DA(S.tok_crank, Tg);
     lda::tmark("histogram, streams, configure");
+    struct Job {
+        uint64_t p0, p1, t0, t1;
+    };
+    std::vector<Job> jobs;
+    std::mutex mu;
+    std::condition_variable cv;
+    bool jobs_done = false;
+    cudaError_t copy_err = cudaSuccess;
+    std::thread copier([&] {
+        cudaSetDevice(ctx->device);
+        cudaStream_t cs = nullptr;
+        cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+        for (;;) {
+            Job j;
+            {
+                std::unique_lock<std::mutex> lk(mu);
+                cv.wait(lk, [&] { return !jobs.empty() || jobs_done; });
+                if (jobs.empty()) break;
+                j = jobs.front();
+                jobs.erase(jobs.begin());
+            }
+            cudaError_t r = cudaSuccess;
+            const size_t np = (j.p1 - j.p0) * sizeof(uint32_t), nt = (j.t1 - j.t0) * sizeof(uint32_t);
+            if (np && r == cudaSuccess)
+                r = cudaMemcpyAsync(S.tok_row + j.p0, H.tok_row.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
+            if (np && r == cudaSuccess)
+                r = cudaMemcpyAsync(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
+            if (nt && r == cudaSuccess)
+                r = cudaMemcpyAsync(S.doc_map + j.t0, H.doc_map.data() + j.t0, nt, cudaMemcpyHostToDevice, cs);
+            if (r == cudaSuccess) r = cudaStreamSynchronize(cs);
+            if (r != cudaSuccess && copy_err == cudaSuccess) copy_err = r;
+        }
+        if (cs) cudaStreamDestroy(cs);
+    });
+    auto on_final = [&](uint64_t p0, uint64_t p1, uint64_t t0, uint64_t t1) {
+        {
+            std::lock_guard<std::mutex> lk(mu);
+            jobs.push_back(Job{p0, p1, t0, t1});
+        }
+        cv.notify_one();
+    };
     std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
-                                      S.sweep_tile ? 2 : (S.sweep_quad ? 1 : 0), ctx->tail_per_tile, H);
+                                      S.sweep_tile ? 2 : (S.sweep_quad ? 1 : 0), ctx->tail_per_tile, H,
+                                      on_final);
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        jobs_done = true;
+    }
+    cv.notify_one();
+    copier.join();
     if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
+    if (copy_err != cudaSuccess) return fail(ctx, LDA_ECUDA, std::string("token table copy: ") + cudaGetErrorString(copy_err));
+    lda::tmark("layout done, token tables on the device");
 
     S.V = V;
     S.K = K;
@@ -394,10 +452,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.beta = ctx->beta;
     S.seed = seed;
 
-    DA(S.tok_row, Tg);
     DA(S.tok_z, Tg);
-    DA(S.doc_map, Tg);
-    DA(S.tok_crank, Tg);
     if (ctx->theta_mode == 1) DA(S.z_doc, Tg + 4);
     DA(S.doc_ptr32, Dg + 1);
     DA(S.row_off32, std::max<int64_t>(Dg, 1));
@@ -435,9 +490,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream) : cudaSuccess;
     };
     lda::tmark("device allocation");
-    CU(h2d(S.tok_row, H.tok_row.data(), sizeof(uint32_t) * Tg));
-    CU(h2d(S.doc_map, H.doc_map.data(), sizeof(uint32_t) * Tg));
-    CU(h2d(S.tok_crank, H.tok_crank.data(), sizeof(uint32_t) * Tg));
     CU(h2d(S.doc_ptr32, H.doc_ptr32.data(), sizeof(uint32_t) * (Dg + 1)));
     CU(h2d(S.row_off32, H.row_off32.data(), sizeof(uint32_t) * Dg));
     CU(h2d(S.segs, H.segs.data(), sizeof(lda::Seg) * H.segs.size()));
@@ -646,10 +698,17 @@ int lda_get_counts(lda_ctx *ctx, int32_t *n_wk, int32_t *n_k, int64_t *ndk_ptr, 
         }
         if (ndk_ptr) ndk_ptr[S.D] = pos;
     }
-    if (z) {
-        std::vector<uint16_t> zw(S.T);
-        if (S.T) CU(cudaMemcpy(zw.data(), S.tok_z, sizeof(uint16_t) * S.T, cudaMemcpyDeviceToHost));
-        for (int64_t i = 0; i < S.T; ++i) z[i] = zw[H.doc_map[i]];
+    if (z && S.T) {
+        // z into document order on the device (the θ rebuild's gather), then D2H
+        uint16_t *zd = S.z_doc;
+        if (!zd) CU(cudaMalloc(&zd, sizeof(uint16_t) * (S.T + 8)));
+        int r = lda::launch_gather_z(S, zd, ctx->stream);
+        cudaError_t ce = r == cudaSuccess ? cudaMemcpyAsync(z, zd, sizeof(uint16_t) * S.T, cudaMemcpyDeviceToHost,
+                                                            ctx->stream)
+                                          : static_cast<cudaError_t>(r);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(ctx->stream);
+        if (zd != S.z_doc) cudaFree(zd);
+        if (ce != cudaSuccess) return fail(ctx, LDA_ECUDA, std::string("z gather: ") + cudaGetErrorString(ce));
     }
     return LDA_OK;
 }
@@ -659,13 +718,19 @@ int lda_set_z(lda_ctx *ctx, const uint16_t *z) {
     if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
     const lda::DevState &S = ctx->S;
     if (!z && S.T) return fail(ctx, LDA_EINVAL, "null z");
-    std::vector<uint16_t> zw(S.T);
-    for (int64_t i = 0; i < S.T; ++i) {
+    for (int64_t i = 0; i < S.T; ++i)
         if (z[i] >= S.K) return fail(ctx, LDA_EINVAL, "topic id >= K");
-        zw[ctx->H.doc_map[i]] = z[i];
-    }
     CU(cudaSetDevice(ctx->device));
-    if (S.T) CU(cudaMemcpy(S.tok_z, zw.data(), sizeof(uint16_t) * S.T, cudaMemcpyHostToDevice));
+    if (S.T) {
+        // H2D in document order, scattered to word-major positions on the device
+        uint16_t *zd = nullptr;
+        CU(cudaMalloc(&zd, sizeof(uint16_t) * S.T));
+        cudaError_t ce = cudaMemcpyAsync(zd, z, sizeof(uint16_t) * S.T, cudaMemcpyHostToDevice, ctx->stream);
+        if (ce == cudaSuccess) ce = static_cast<cudaError_t>(lda::launch_scatter_z(S, zd, ctx->stream));
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(ctx->stream);
+        cudaFree(zd);
+        if (ce != cudaSuccess) return fail(ctx, LDA_ECUDA, std::string("z scatter: ") + cudaGetErrorString(ce));
+    }
     int launches = 0;
     int r = rebuild_counts(ctx, &launches);
     if (r != LDA_OK) return r;

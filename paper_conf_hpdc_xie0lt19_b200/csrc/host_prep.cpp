@@ -130,7 +130,8 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
-                         int sampler, int64_t tail_per_tile, HostLayout &L) {
+                         int sampler, int64_t tail_per_tile, HostLayout &L,
+                         const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final) {
     const bool build_pairs = sampler == 1;
     const int64_t T = doc_ptr[D];
     L.D = D;
@@ -229,6 +230,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 
     uint64_t pos = 0;  // start of the current tile's segment
     for (int b = 0; b < ndt; ++b) {
+        const uint64_t pos_tile = pos;
         const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
         // the tile's documents in nth contiguous parts (original order), balanced by tokens
         const int nth = (doc_ptr[d1] - doc_ptr[d0]) < (1 << 16) ? 1 : nthreads;
@@ -300,7 +302,10 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                 }
             }
         });
+        if (on_final)
+            on_final(pos_tile, pos, static_cast<uint64_t>(doc_ptr[d0]), static_cast<uint64_t>(doc_ptr[d1]));
     }
+    if (on_final && tail_tokens > 0) on_final(static_cast<uint64_t>(T - tail_tokens), static_cast<uint64_t>(T), 0, 0);
     if (pos != static_cast<uint64_t>(T - tail_tokens)) return "internal: token layout does not cover the corpus";
     ctmp.release();
     tmark("layout: tiles (count, ranks, scatter)");

@@ -1578,6 +1578,14 @@ __global__ void gather_z_kernel(const uint32_t *__restrict__ doc_map, const uint
     }
 }
 
+// z in document order -> word-major (lda_set_z): zw[doc_map[i]] = zd[i]
+__global__ void scatter_z_kernel(const uint32_t *__restrict__ doc_map, const uint16_t *__restrict__ zd,
+                                 uint16_t *__restrict__ zw, int64_t T) {
+    for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < T;
+         i += static_cast<int64_t>(gridDim.x) * blockDim.x)
+        zw[doc_map[i]] = zd[i];
+}
+
 // GATHERED = false: z through the doc-word map (fused); true: zd is z in
 // document order (phase B of the two-phase variant).
 template <bool GATHERED>
@@ -1872,6 +1880,20 @@ int launch_recount(const DevState &s, void *stream, int *launches) {
     recount_kernel<<<s.sweep_grid > 0 ? s.num_sms * 4 : 1, 256, 8 * s.K, st>>>(
         s.rchunks, s.n_rchunks, s.segs, s.K, s.tok_z, s.nwk, nk, s.counter + 1);
     ++*launches;
+    return cudaGetLastError();
+}
+
+int launch_gather_z(const DevState &s, uint16_t *zd, void *stream) {
+    const int64_t thr = (s.T + 7) / 8;
+    if (thr > 0)
+        gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, static_cast<cudaStream_t>(stream)>>>(
+            s.doc_map, s.tok_z, zd, s.T);
+    return cudaGetLastError();
+}
+
+int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream) {
+    if (s.T > 0)
+        scatter_z_kernel<<<4 * s.num_sms, 256, 0, static_cast<cudaStream_t>(stream)>>>(s.doc_map, zd, s.tok_z, s.T);
     return cudaGetLastError();
 }
 

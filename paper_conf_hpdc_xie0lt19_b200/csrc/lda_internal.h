@@ -3,6 +3,7 @@
 #pragma once
 
 #include <cstdint>
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -122,11 +123,17 @@ struct HostLayout {
 };
 
 // cbase[w] = canonical index of this rank's first token of word w.
+// on_final(pos_begin, pos_end, tok_begin, tok_end), if set, is called as soon
+// as tok_row / tok_crank over word-major positions [pos_begin, pos_end) and
+// doc_map over document-major tokens [tok_begin, tok_end) are final (after
+// each document tile, and for the tail region at the end) -- the caller can
+// start their host->device copies while the next tile is prepared.
 // Returns "" on success, else an error message.
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
-                         int sampler, int64_t tail_per_tile, HostLayout &out);
+                         int sampler, int64_t tail_per_tile, HostLayout &out,
+                         const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {});
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
@@ -210,6 +217,9 @@ int configure_kernels(DevState &s);
 int launch_init(const DevState &s, void *stream);
 int launch_recount(const DevState &s, void *stream, int *launches);
 int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches);
+// z in document order <-> word-major, through doc_map (device buffers of T entries; zd 16-byte aligned)
+int launch_gather_z(const DevState &s, uint16_t *zd, void *stream);
+int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream);
 int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event);
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches);
 
