@@ -1051,10 +1051,16 @@ __device__ __forceinline__ double i2d_pos(int n) {
 // Layout per word (wt_bytes, a multiple of 16): [Pc: NC+1 doubles, padded
 // to an even count][p32: K4 floats][L32: K4 floats].  One warp per word;
 // lane l holds k = 128c + 4l .. 4l+3 of chunk c.
+// L32 holds whole 128-topic chunks, groups of 4 entries swizzled by the chunk
+// index (k ^ ((c & 7) << 2)): the dense binary searches of lanes in different
+// chunks probe the same in-chunk offsets, which would otherwise all fall in
+// one shared-memory bank.
 __host__ __device__ constexpr int tab_nc2(int K) { return ((K + 127) / 128 + 2) / 2 * 2; }
 __host__ __device__ constexpr size_t tab_bytes(int K) {
-    return static_cast<size_t>(tab_nc2(K)) * 8 + static_cast<size_t>(8) * ((K + 3) & ~3);
+    return static_cast<size_t>(tab_nc2(K)) * 8 + static_cast<size_t>(4) * ((K + 3) & ~3) +
+           static_cast<size_t>(4) * 128 * ((K + 127) / 128);
 }
+__host__ __device__ constexpr int l32_idx(int k) { return k ^ (((k >> 7) & 7) << 2); }
 
 template <bool VEC>
 __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double *__restrict__ denom, int V, int K,
@@ -1108,12 +1114,12 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
             const float f0 = d2f_trunc(excl + l0), f1 = d2f_trunc(excl + l1);
             const float f2 = d2f_trunc(excl + l2), f3 = d2f_trunc(excl + l3);
             if (VEC) {
-                if (k < K) *reinterpret_cast<float4 *>(L32 + k) = make_float4(f0, f1, f2, f3);
+                if (k < K) *reinterpret_cast<float4 *>(L32 + l32_idx(k)) = make_float4(f0, f1, f2, f3);
             } else {
                 const float ff[4] = {f0, f1, f2, f3};
 #pragma unroll
                 for (int e = 0; e < 4; ++e)
-                    if (k + e < K) L32[k + e] = ff[e];
+                    if (k + e < K) L32[l32_idx(k + e)] = ff[e];
             }
             if (lane == 0) Pc[c] = carry;
             carry += __shfl_sync(kFull, incl, 31);
@@ -1121,10 +1127,8 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
         if (lane == 0) Pc[(K + 127) / 128] = carry;
         // zero the padding so that the table bytes are deterministic
         if (lane == 1 && tab_nc2(K) > (K + 127) / 128 + 1) Pc[tab_nc2(K) - 1] = 0.0;
-        for (int k = K + lane; k < K4; k += 32) {
-            p32[k] = 0.0f;
-            L32[k] = 0.0f;
-        }
+        for (int k = K + lane; k < K4; k += 32) p32[k] = 0.0f;
+        for (int k = K + lane; k < 128 * ((K + 127) / 128); k += 32) L32[l32_idx(k)] = 0.0f;
     }
 }
 
@@ -1178,7 +1182,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     double *Pc = reinterpret_cast<double *>(wb);
     float *p32 = reinterpret_cast<float *>(Pc + tab_nc2(K));
     float *L32 = p32 + K4;
-    float *blk = L32 + K4;                 // 4 block sums per line
+    float *blk = L32 + 128 * NC;           // 4 block sums per line
     float *lsm = blk + 4 * LM;             // line sums
     uint32_t *lrow = reinterpret_cast<uint32_t *>(lsm + LM);
     uint32_t *tcum = lrow + LM;
@@ -1214,6 +1218,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     // walk in flight.  Built for the next batch before the current batch's
     // draw, so that its loads overlap the draw.
     Blk8 ring[R];
+    bool hdr[R];  // the line in ring slot s2 is the first of its row (word 0 = nnz header)
     struct Head {
         bool take, dup;
         int nb;
@@ -1248,7 +1253,12 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
             const uint32_t L = q + 8u * s2;
 #pragma unroll
             for (int e = 0; e < 8; ++e) ring[s2].w[e] = 0u;
-            if (L < h.lsum) ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lrow[L] & 0x7FFFFFFFu) + sub) * 8);
+            hdr[s2] = false;
+            if (L < h.lsum) {
+                const uint32_t lr = lrow[L];
+                ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+                hdr[s2] = sub == 0 && (lr >> 31);
+            }
         }
         return h;
     };
@@ -1317,9 +1327,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
             float bs[R];
 #pragma unroll
             for (int s2 = 0; s2 < R; ++s2) {
-                const uint32_t L = base + 8u * s2 + q;
-                const uint32_t lr = lrow[min(L, static_cast<uint32_t>(LM) - 1u)];
-                const uint32_t w0 = (sub == 0 && (lr >> 31)) ? 0u : ring[s2].w[0];  // header word
+                const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
                 float s0 = count_f32(w0) * tab32(p32, w0);
                 float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
                 s0 = entry_mass32(ring[s2].w[2], p32, s0);
@@ -1333,7 +1341,11 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
 #pragma unroll
             for (int s2 = 0; s2 < R; ++s2) {
                 const uint32_t Ln = base + 8u * (s2 + R) + q;
-                if (Ln < lsum) ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lrow[Ln] & 0x7FFFFFFFu) + sub) * 8);
+                if (Ln < lsum) {
+                    const uint32_t lr = lrow[Ln];
+                    ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+                    hdr[s2] = sub == 0 && (lr >> 31);
+                }
             }
 #pragma unroll
             for (int s2 = 0; s2 < R; ++s2) {
@@ -1441,12 +1453,12 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
                 int k = 0;  // first k in the chunk with L32 > r (kn - 1 if none)
                 for (int n = kn; n > 1;) {
                     const int h = n >> 1;
-                    if (L32[kb + k + h - 1] <= r32) k += h;
+                    if (L32[l32_idx(kb + k + h - 1)] <= r32) k += h;
                     n -= h;
                 }
                 z = kb + k;
                 // certify the bracket: L[z-1] <= y < L[z] (Pc[c] when k = 0)
-                const float le = L32[z], lp = k > 0 ? L32[z - 1] : 0.0f;
+                const float le = L32[l32_idx(z)], lp = k > 0 ? L32[l32_idx(z - 1)] : 0.0f;
                 flag = (z < K - 1 && le - r32 <= fmaf(1.3e-7f * g32, le, eR)) ||
                        (k > 0 && r32 - lp <= fmaf(1.3e-7f * g32, lp, eR)) ||
                        (k == 0 && c > 0 && r <= ey);
