@@ -164,15 +164,18 @@ def lda_loglik(ctx) -> float:
     return v.value
 
 
-def lda_get_counts(ctx, n_wk=None, n_k=None, ndk_ptr=None, ndk_topic=None, ndk_count=None, z=None):
+def lda_get_counts(ctx, n_wk=None, n_k=None, ndk_ptr=None, ndk_topic=None, ndk_count=None, z=None,
+                   want_nnz=False):
     """Fills the given (preallocated, C-contiguous) numpy arrays; returns nnz."""
     nnz = _i64()
     cap = 0 if ndk_topic is None else len(ndk_topic)
     if ndk_count is not None:
         cap = len(ndk_count) if ndk_topic is None else min(cap, len(ndk_count))
+    # the θ rows are read back (and nnz counted) only when a θ array is requested
+    want = want_nnz or ndk_ptr is not None or ndk_topic is not None or ndk_count is not None
     _check(lib().lda_get_counts(ctx, _p(n_wk), _p(n_k), _p(ndk_ptr), _p(ndk_topic), _p(ndk_count), cap,
-                                ctypes.byref(nnz), _p(z)), ctx)
-    return nnz.value
+                                ctypes.byref(nnz) if want else None, _p(z)), ctx)
+    return nnz.value if want else None
 
 
 def lda_get_stats(ctx) -> dict:
@@ -269,7 +272,7 @@ class LDA:
         return a
 
     def theta_csr(self):
-        nnz = lda_get_counts(self.ctx)
+        nnz = lda_get_counts(self.ctx, want_nnz=True)
         Dg = self.doc_end - self.doc_begin
         ptr = np.empty(Dg + 1, np.int64)
         top = np.empty(nnz, np.uint16)
