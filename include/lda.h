@@ -98,7 +98,7 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *   "tile_tokens"   split the documents into tiles of about this many tokens
  *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
- *   "sampler"       -1 (default): 2 if K <= 4096, else 0.
+ *   "sampler"       -1 (default): 2 if K <= 4096, else 3.
  *                   2: tile sampler -- work items are the tokens
  *                   of one word inside one document tile, queued tile by
  *                   tile so the tiles' θ rows stay in L2; one warp per item,
@@ -110,6 +110,10 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   layout (else sampler 0); at K = 8192 its per-warp
  *                   tables leave too few warps per SM (measured slower
  *                   than sampler 0, hence the default).
+ *                   3: the tile sampler with the word table shared by the
+ *                   8 warps of a CTA (double-buffered) -- large K (at
+ *                   K = 8192: 1.7x the lane-per-token sampler); same draws
+ *                   as 2.  Falls back to 0 when its tables do not fit.
  *                   1: quad sampler over (word, document) pairs.
  *                   0: lane-per-token fp64 sampler (32-byte row blocks).
  *                   The samplers differ only in rounding at a CDF boundary

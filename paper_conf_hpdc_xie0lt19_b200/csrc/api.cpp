@@ -247,7 +247,7 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
         if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "filter32 must be 0 or 1");
         ctx->filter32 = static_cast<int>(value);
     } else if (k == "sampler") {
-        if (value < -1 || value > 2) return fail(ctx, LDA_EINVAL, "sampler must be -1 (auto), 0, 1 or 2");
+        if (value < -1 || value > 3) return fail(ctx, LDA_EINVAL, "sampler must be -1 (auto), 0, 1, 2 or 3");
         ctx->sampler = static_cast<int>(value);
     } else if (k == "tail_per_tile") {
         if (value < 0 || value > (int64_t(1) << 30)) return fail(ctx, LDA_EINVAL, "tail_per_tile out of range");
@@ -431,7 +431,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     };
     std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
-                                      S.sweep_tile ? 2 : (S.sweep_quad ? 1 : 0), ctx->tail_per_tile, H,
+                                      (S.sweep_tile || S.sweep_tile_cta) ? 2 : (S.sweep_quad ? 1 : 0),
+                                      ctx->tail_per_tile, H,
                                       on_final);
     {
         std::lock_guard<std::mutex> lk(mu);
@@ -469,7 +470,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         DA(S.pairs, H.pairs.size());
     }
     S.n_titems = static_cast<int64_t>(H.titems.size());
-    if (S.sweep_tile) {
+    if (S.sweep_tile || S.sweep_tile_cta) {
         DA(S.titems, H.titems.size());
         DA(S.cbase, V);
         DA(S.wtab, S.wt_bytes * static_cast<size_t>(V));
@@ -501,7 +502,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         CU(h2d(S.pchunks, H.pchunks.data(), sizeof(lda::PairChunk) * H.pchunks.size()));
         CU(h2d(S.pairs, H.pairs.data(), sizeof(lda::PairRec) * H.pairs.size()));
     }
-    if (S.sweep_tile) {
+    if (S.sweep_tile || S.sweep_tile_cta) {
         CU(h2d(S.titems, H.titems.data(), sizeof(lda::TileItem) * H.titems.size()));
         CU(h2d(S.cbase, cbase.data(), sizeof(uint64_t) * V));
     }

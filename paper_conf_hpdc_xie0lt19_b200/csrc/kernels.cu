@@ -1168,6 +1168,254 @@ __host__ __device__ constexpr size_t tile_warp_bytes(int K, int lmax) {
     return tab_bytes(K) + static_cast<size_t>(lmax) * (16 + 4 + 4) + 32 * 4 + 16;
 }
 
+// Batch head of the tile sampler: up to 32 tokens whose θ rows have at most
+// LM lines in total; consecutive tokens of one document -- a (word, doc)
+// pair -- share the walk of its row.  Writes the line table (bits 0-30: θ
+// row offset of the line in 32-byte units, bit 31: first line of its row) and
+// puts the first R lines of the walk in flight.
+struct TileHead {
+    bool take, dup;
+    int nb;
+    uint32_t lsum, c0, nl;
+};
+template <int R>
+__device__ __forceinline__ TileHead tile_head(const TileArgs &a, uint32_t row, uint32_t nnz, bool valid, int LM,
+                                              uint32_t *lrow, Blk8 (&ring)[R], bool (&hdr)[R]) {
+    const int lane = threadIdx.x & 31, q = lane >> 2, sub = lane & 3;
+    TileHead h;
+    const uint32_t prow = __shfl_up_sync(kFull, row, 1);
+    h.dup = valid && lane > 0 && prow == row;
+    h.nl = valid ? (nnz + 32u) >> 5 : 0u;  // 128-byte lines holding words 0..nnz
+    const uint32_t nlw = h.dup ? 0u : h.nl;
+    uint32_t incl = nlw;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+    }
+    h.take = valid && (incl <= static_cast<uint32_t>(LM) || lane == 0);
+    h.nb = __popc(__ballot_sync(kFull, h.take));
+    const uint32_t ls = __shfl_sync(kFull, incl, h.nb > 0 ? h.nb - 1 : 0);
+    h.lsum = h.nb > 0 ? ls : 0u;
+    const uint32_t c0 = incl - nlw;
+    // a duplicate's lines are those of the last non-duplicate lane before it
+    const unsigned heads = __ballot_sync(kFull, !h.dup);
+    const int hl = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));
+    h.c0 = __shfl_sync(kFull, c0, hl);
+    if (h.take && !h.dup)
+        for (uint32_t i = 0; i < h.nl; ++i) lrow[h.c0 + i] = (row + 4u * i) | (i == 0 ? 0x80000000u : 0u);
+    __syncwarp();
+#pragma unroll
+    for (int s2 = 0; s2 < R; ++s2) {
+        const uint32_t L = q + 8u * s2;
+#pragma unroll
+        for (int e = 0; e < 8; ++e) ring[s2].w[e] = 0u;
+        hdr[s2] = false;
+        if (L < h.lsum) {
+            const uint32_t lr = lrow[L];
+            ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+            hdr[s2] = sub == 0 && (lr >> 31);
+        }
+    }
+    return h;
+}
+
+// The walk (p1 of Eq. 6): quad q takes lines q, q+8, ... of the batch; lane
+// `sub` sums entries 8·sub .. 8·sub+7 of the line (two FFMA chains); the
+// quad's line sum by two xor-shuffles.  Branch-free over the R lines in
+// flight (a lane past the end sums stale entries and discards them).
+// at_step2() runs once, after the first step (the caller's prefetch hook).
+template <int R, class F>
+__device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, const uint32_t *lrow, Blk8 (&ring)[R],
+                                          bool (&hdr)[R], const float *p32, float *blk, float *lsm, F &&at_step2) {
+    const int lane = threadIdx.x & 31, q = lane >> 2, sub = lane & 3;
+    bool hooked = false;
+    for (uint32_t base = 0; base < lsum; base += 8u * R) {
+        if (base == 8u * R) {
+            at_step2();
+            hooked = true;
+        }
+        float bs[R];
+#pragma unroll
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
+            float s0 = count_f32(w0) * tab32(p32, w0);
+            float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
+            s0 = entry_mass32(ring[s2].w[2], p32, s0);
+            s1 = entry_mass32(ring[s2].w[3], p32, s1);
+            s0 = entry_mass32(ring[s2].w[4], p32, s0);
+            s1 = entry_mass32(ring[s2].w[5], p32, s1);
+            s0 = entry_mass32(ring[s2].w[6], p32, s0);
+            s1 = entry_mass32(ring[s2].w[7], p32, s1);
+            bs[s2] = s0 + s1;
+        }
+#pragma unroll
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t Ln = base + 8u * (s2 + R) + q;
+            if (Ln < lsum) {
+                const uint32_t lr = lrow[Ln];
+                ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+                hdr[s2] = sub == 0 && (lr >> 31);
+            }
+        }
+#pragma unroll
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t L = base + 8u * s2 + q;
+            float ls = bs[s2] + __shfl_xor_sync(kFull, bs[s2], 1);
+            ls += __shfl_xor_sync(kFull, ls, 2);
+            if (L < lsum) {
+                blk[4 * L + sub] = bs[s2];
+                if (sub == 0) lsm[L] = ls;
+            }
+        }
+    }
+    if (!hooked) at_step2();
+}
+
+// Draw of one token of a tile-sampler batch (lane per token, `take` lanes):
+// Every search runs on the approximate (monotone) prefixes with plain
+// comparisons; the draw is then certified by the margins of the two prefixes
+// that bracket x, each against a rigorous bound on its error (the other
+// prefixes are farther from x by monotonicity); uncertain -> flag.
+__device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t c0, uint32_t nl, uint32_t row,
+                                          uint32_t crank, uint64_t cb, double Q64, double gS, const float *lsm,
+                                          const float *blk, const float *p32, const float *L32, const double *Pc,
+                                          int NC, int &z, bool &flag, uint32_t &x0) {
+    const int K = a.K;
+    const double u = 5.9604644775390625e-08;  // fp32 unit roundoff 2^-24
+    z = 0;
+    flag = false;
+    x0 = 0;
+    if (take) {
+        const float *ln = lsm + c0;
+        double S = 0.0;
+        for (uint32_t i = 0; i < nl; ++i) S += f2d_pos(ln[i]);
+        x0 = philox_x0_sched(cb + crank, a.t, a.key0, a.key1);
+        const double U = (__hiloint2double(0x43300000, static_cast<int>(x0)) - 4503599627370496.0) *
+                         2.3283064365386962890625e-10;  // x0·2^-32, exact
+        const double tot = S + Q64;
+        const double x = U * tot;
+        const double eps = 1.0e-13 * tot * a.slack;  // fp64 roundings of this path
+        const double eX = U * gS * S + eps;          // |x' - x|
+        const double d = S - x;                       // sparse iff > 0
+        const float g32 = static_cast<float>(a.slack);
+        if (fabs(d) <= (1.0 - U) * gS * S + eps) {
+            flag = true;
+        } else if (d > 0.0) {
+            // sparse bucket: the line, then the block, whose end prefix first exceeds x
+            double C = 0.0, Cn = 0.0;
+            uint32_t i = 0;
+            for (;; ++i) {
+                Cn = C + f2d_pos(ln[i]);
+                if (Cn > x || i + 1 >= nl) break;
+                C = Cn;
+            }
+            const float *bk = blk + 4 * (c0 + i);
+            uint32_t b = 0;
+            for (; b < 3; ++b) {
+                const double Cb = C + f2d_pos(bk[b]);
+                if (Cb > x) {
+                    Cn = Cb;
+                    break;
+                }
+                C = Cb;
+            }
+            // certify: C <= x < Cn with margins (C = 0 needs none)
+            flag = (x - C <= gS * C + eX && C > 0.0) || (Cn - x <= gS * Cn + eX);
+            b += 4 * i;
+            // the block's entries in order, relative to r = x - C (fp32):
+            // first e with local prefix s_e > r; certify s_{e-1}, s_e
+            const float r32 = static_cast<float>(x - C);
+            const float eR = static_cast<float>((eX + gS * C + u * (x - C)) * 1.0001 + 1e-30);
+            Blk8 w = ld_nc_v8(a.rows + (static_cast<size_t>(row) + b) * 8);
+            if (b == 0) w.w[0] = 0u;
+            float sl = 0.0f, sp = 0.0f, se = 0.0f;
+            int ez = -1;
+            uint32_t we = 0;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+                const float sn = entry_mass32(w.w[e], p32, sl);
+                if (ez < 0 && sn > r32) {
+                    ez = e;
+                    sp = sl;
+                    se = sn;
+                    we = w.w[e];
+                }
+                sl = sn;
+            }
+            if (ez < 0) {
+                flag = true;
+            } else {
+                flag = flag || (se - r32 <= fmaf(6.2e-7f * g32, se, eR)) ||
+                       (sp > 0.0f && r32 - sp <= fmaf(6.2e-7f * g32, sp, eR));   // (2u + 8u)·s
+                z = static_cast<int>(we >> kTS);
+            }
+        } else {
+            // dense bucket: first k with P[k] > y = x - S = U·Q - (1-U)·S;
+            // chunk by the fp64 bases Pc, then inside the chunk by L32
+            const double y = U * Q64 - (1.0 - U) * S;
+            const double ey = (1.0 - U) * gS * S + eps;
+            int c = 0;
+            for (int n = NC; n > 1;) {  // last chunk c with Pc[c] <= y
+                const int h = n >> 1;
+                if (Pc[c + h] <= y) c += h;
+                n -= h;
+            }
+            const double r = y - Pc[c];
+            const float r32 = static_cast<float>(r);
+            const float eR = static_cast<float>((ey + u * fabs(r)) * 1.0001 + 1e-30);
+            const int kb = 128 * c, kn = min(K, kb + 128) - kb;
+            int k = 0;  // first k in the chunk with L32 > r (kn - 1 if none)
+            for (int n = kn; n > 1;) {
+                const int h = n >> 1;
+                if (L32[l32_idx(kb + k + h - 1)] <= r32) k += h;
+                n -= h;
+            }
+            z = kb + k;
+            // certify the bracket: L[z-1] <= y < L[z] (Pc[c] when k = 0)
+            const float le = L32[l32_idx(z)], lp = k > 0 ? L32[l32_idx(z - 1)] : 0.0f;
+            flag = (z < K - 1 && le - r32 <= fmaf(1.3e-7f * g32, le, eR)) ||
+                   (k > 0 && r32 - lp <= fmaf(1.3e-7f * g32, lp, eR)) ||
+                   (k == 0 && c > 0 && r <= ey);
+        }
+    }
+}
+
+// Exact fp64 redraw of a batch's uncertain tokens (one at a time by the
+// warp), then z and the fused recount (ϕ update, L1273-1285).
+__device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool flag, int z, uint32_t row,
+                                            uint32_t nnz, uint32_t x0, uint32_t p, const int32_t *nwk_row,
+                                            int32_t *row_next, int *nkh, double *q64x, int *have_q,
+                                            unsigned &n_exact) {
+    const int lane = threadIdx.x & 31;
+    const int K = a.K;
+    // ---- exact fp64 redraw of the uncertain tokens, one at a time by the warp
+    unsigned fl = __ballot_sync(kFull, flag);
+    while (fl) {
+        const int f = __ffs(fl) - 1;
+        fl &= fl - 1;
+        const uint32_t rf = __shfl_sync(kFull, row, f);
+        const uint32_t nf = __shfl_sync(kFull, nnz, f);
+        const uint32_t xf = __shfl_sync(kFull, x0, f);
+        const int zf = draw_exact_warp(nwk_row, a.denom, a.rows + static_cast<size_t>(rf) * 8, nf, xf, K,
+                                       a.alpha, a.beta, q64x, have_q);
+        if (lane == f) z = zf;
+        ++n_exact;
+    }
+    // ---- z and the fused recount
+    if (take) {
+        a.z[p] = static_cast<uint16_t>(z);
+        const unsigned act = __activemask();
+        const unsigned peers = __match_any_sync(act, z);
+        if (lane == __ffs(peers) - 1) {
+            const int c = __popc(peers);
+            atomicAdd(row_next + z, c);
+            atomicAdd(&nkh[z], c);
+        }
+    }
+    __syncwarp();
+}
+
 template <int R>
 __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     extern __shared__ double smem_dd[];
@@ -1219,48 +1467,8 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     // draw, so that its loads overlap the draw.
     Blk8 ring[R];
     bool hdr[R];  // the line in ring slot s2 is the first of its row (word 0 = nnz header)
-    struct Head {
-        bool take, dup;
-        int nb;
-        uint32_t lsum, c0, nl;
-    };
     auto head = [&](uint32_t row, uint32_t nnz, bool valid) {
-        Head h;
-        const uint32_t prow = __shfl_up_sync(kFull, row, 1);
-        h.dup = valid && lane > 0 && prow == row;
-        h.nl = valid ? (nnz + 32u) >> 5 : 0u;  // 128-byte lines holding words 0..nnz
-        const uint32_t nlw = h.dup ? 0u : h.nl;
-        uint32_t incl = nlw;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const uint32_t y = __shfl_up_sync(kFull, incl, o);
-            if (lane >= o) incl += y;
-        }
-        h.take = valid && (incl <= static_cast<uint32_t>(LM) || lane == 0);
-        h.nb = __popc(__ballot_sync(kFull, h.take));
-        const uint32_t ls = __shfl_sync(kFull, incl, h.nb > 0 ? h.nb - 1 : 0);
-        h.lsum = h.nb > 0 ? ls : 0u;
-        uint32_t c0 = incl - nlw;
-        // a duplicate's lines are those of the last non-duplicate lane before it
-        const unsigned heads = __ballot_sync(kFull, !h.dup);
-        const int hl = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));
-        h.c0 = __shfl_sync(kFull, c0, hl);
-        if (h.take && !h.dup)
-            for (uint32_t i = 0; i < h.nl; ++i) lrow[h.c0 + i] = (row + 4u * i) | (i == 0 ? 0x80000000u : 0u);
-        __syncwarp();
-#pragma unroll
-        for (int s2 = 0; s2 < R; ++s2) {
-            const uint32_t L = q + 8u * s2;
-#pragma unroll
-            for (int e = 0; e < 8; ++e) ring[s2].w[e] = 0u;
-            hdr[s2] = false;
-            if (L < h.lsum) {
-                const uint32_t lr = lrow[L];
-                ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
-                hdr[s2] = sub == 0 && (lr >> 31);
-            }
-        }
-        return h;
+        return tile_head<R>(a, row, nnz, valid, LM, lrow, ring, hdr);
     };
     // the first batch
     uint32_t row = 0, crank = 0, nnz = 0;
@@ -1269,7 +1477,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
         crank = __ldg(a.tok_crank + it.pos + lane);
         nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
     }
-    Head hd = head(row, nnz, static_cast<uint32_t>(lane) < it.n);
+    TileHead hd = head(row, nnz, static_cast<uint32_t>(lane) < it.n);
     uint32_t b0 = 0;
     bool new_item = true;
     const int32_t *nwk_row = nullptr;
@@ -1314,181 +1522,24 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
             n_row = __ldg(a.tok_row + nxt_pos + lane);
             n_crank = __ldg(a.tok_crank + nxt_pos + lane);
         }
-        bool nnz_issued = false;
-        // ---- walk: quad q takes lines q, q+8, ... of the batch; lane `sub`
-        // sums entries 8·sub .. 8·sub+7 of the line (two FFMA chains); the
-        // quad's line sum by two xor-shuffles.  Branch-free over the R lines
-        // in flight (a lane past the end sums stale entries and discards them).
-        for (uint32_t base = 0; base < lsum; base += 8u * R) {
-            if (base == 8u * R) {  // the next batch's row headers, once its rows have arrived
-                if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
-                nnz_issued = true;
-            }
-            float bs[R];
-#pragma unroll
-            for (int s2 = 0; s2 < R; ++s2) {
-                const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
-                float s0 = count_f32(w0) * tab32(p32, w0);
-                float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
-                s0 = entry_mass32(ring[s2].w[2], p32, s0);
-                s1 = entry_mass32(ring[s2].w[3], p32, s1);
-                s0 = entry_mass32(ring[s2].w[4], p32, s0);
-                s1 = entry_mass32(ring[s2].w[5], p32, s1);
-                s0 = entry_mass32(ring[s2].w[6], p32, s0);
-                s1 = entry_mass32(ring[s2].w[7], p32, s1);
-                bs[s2] = s0 + s1;
-            }
-#pragma unroll
-            for (int s2 = 0; s2 < R; ++s2) {
-                const uint32_t Ln = base + 8u * (s2 + R) + q;
-                if (Ln < lsum) {
-                    const uint32_t lr = lrow[Ln];
-                    ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
-                    hdr[s2] = sub == 0 && (lr >> 31);
-                }
-            }
-#pragma unroll
-            for (int s2 = 0; s2 < R; ++s2) {
-                const uint32_t L = base + 8u * s2 + q;
-                float ls = bs[s2] + __shfl_xor_sync(kFull, bs[s2], 1);
-                ls += __shfl_xor_sync(kFull, ls, 2);
-                if (L < lsum) {
-                    blk[4 * L + sub] = bs[s2];
-                    if (sub == 0) lsm[L] = ls;
-                }
-            }
-        }
-        if (!nnz_issued && nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+        // ---- walk (the next batch's row headers issued after its first step)
+        tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, lsm, [&] {
+            if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+        });
         __syncwarp();
         // ---- the next batch's head: its line table and first lines, in flight during this draw
-        const Head hn = head(n_row, n_nnz, nxt_valid);
+        const TileHead hn = head(n_row, n_nnz, nxt_valid);
 
         // ---- draw: lane per token (lanes < nb).  Every search below runs on
         // the approximate (monotone) prefixes with plain comparisons; the
         // draw is then certified by the margins of the two prefixes that
         // bracket x, each against a rigorous bound on its error (the other
         // prefixes are farther from x by monotonicity); uncertain -> flag.
-        int z = 0;
-        bool flag = false;
-        uint32_t x0 = 0;
-        if (take) {
-            const float *ln = lsm + c0;
-            double S = 0.0;
-            for (uint32_t i = 0; i < nl; ++i) S += f2d_pos(ln[i]);
-            x0 = philox_x0_sched(cb + crank, a.t, a.key0, a.key1);
-            const double U = (__hiloint2double(0x43300000, static_cast<int>(x0)) - 4503599627370496.0) *
-                             2.3283064365386962890625e-10;  // x0·2^-32, exact
-            const double tot = S + Q64;
-            const double x = U * tot;
-            const double eps = 1.0e-13 * tot * a.slack;  // fp64 roundings of this path
-            const double eX = U * gS * S + eps;          // |x' - x|
-            const double d = S - x;                       // sparse iff > 0
-            const float g32 = static_cast<float>(a.slack);
-            if (fabs(d) <= (1.0 - U) * gS * S + eps) {
-                flag = true;
-            } else if (d > 0.0) {
-                // sparse bucket: the line, then the block, whose end prefix first exceeds x
-                double C = 0.0, Cn = 0.0;
-                uint32_t i = 0;
-                for (;; ++i) {
-                    Cn = C + f2d_pos(ln[i]);
-                    if (Cn > x || i + 1 >= nl) break;
-                    C = Cn;
-                }
-                const float *bk = blk + 4 * (c0 + i);
-                uint32_t b = 0;
-                for (; b < 3; ++b) {
-                    const double Cb = C + f2d_pos(bk[b]);
-                    if (Cb > x) {
-                        Cn = Cb;
-                        break;
-                    }
-                    C = Cb;
-                }
-                // certify: C <= x < Cn with margins (C = 0 needs none)
-                flag = (x - C <= gS * C + eX && C > 0.0) || (Cn - x <= gS * Cn + eX);
-                b += 4 * i;
-                // the block's entries in order, relative to r = x - C (fp32):
-                // first e with local prefix s_e > r; certify s_{e-1}, s_e
-                const float r32 = static_cast<float>(x - C);
-                const float eR = static_cast<float>((eX + gS * C + u * (x - C)) * 1.0001 + 1e-30);
-                Blk8 w = ld_nc_v8(a.rows + (static_cast<size_t>(row) + b) * 8);
-                if (b == 0) w.w[0] = 0u;
-                float sl = 0.0f, sp = 0.0f, se = 0.0f;
-                int ez = -1;
-                uint32_t we = 0;
-#pragma unroll
-                for (int e = 0; e < 8; ++e) {
-                    const float sn = entry_mass32(w.w[e], p32, sl);
-                    if (ez < 0 && sn > r32) {
-                        ez = e;
-                        sp = sl;
-                        se = sn;
-                        we = w.w[e];
-                    }
-                    sl = sn;
-                }
-                if (ez < 0) {
-                    flag = true;
-                } else {
-                    flag = flag || (se - r32 <= fmaf(6.2e-7f * g32, se, eR)) ||
-                           (sp > 0.0f && r32 - sp <= fmaf(6.2e-7f * g32, sp, eR));   // (2u + 8u)·s
-                    z = static_cast<int>(we >> kTS);
-                }
-            } else {
-                // dense bucket: first k with P[k] > y = x - S = U·Q - (1-U)·S;
-                // chunk by the fp64 bases Pc, then inside the chunk by L32
-                const double y = U * Q64 - (1.0 - U) * S;
-                const double ey = (1.0 - U) * gS * S + eps;
-                int c = 0;
-                for (int n = NC; n > 1;) {  // last chunk c with Pc[c] <= y
-                    const int h = n >> 1;
-                    if (Pc[c + h] <= y) c += h;
-                    n -= h;
-                }
-                const double r = y - Pc[c];
-                const float r32 = static_cast<float>(r);
-                const float eR = static_cast<float>((ey + u * fabs(r)) * 1.0001 + 1e-30);
-                const int kb = 128 * c, kn = min(K, kb + 128) - kb;
-                int k = 0;  // first k in the chunk with L32 > r (kn - 1 if none)
-                for (int n = kn; n > 1;) {
-                    const int h = n >> 1;
-                    if (L32[l32_idx(kb + k + h - 1)] <= r32) k += h;
-                    n -= h;
-                }
-                z = kb + k;
-                // certify the bracket: L[z-1] <= y < L[z] (Pc[c] when k = 0)
-                const float le = L32[l32_idx(z)], lp = k > 0 ? L32[l32_idx(z - 1)] : 0.0f;
-                flag = (z < K - 1 && le - r32 <= fmaf(1.3e-7f * g32, le, eR)) ||
-                       (k > 0 && r32 - lp <= fmaf(1.3e-7f * g32, lp, eR)) ||
-                       (k == 0 && c > 0 && r <= ey);
-            }
-        }
-        // ---- exact fp64 redraw of the uncertain tokens, one at a time by the warp
-        unsigned fl = __ballot_sync(kFull, flag);
-        while (fl) {
-            const int f = __ffs(fl) - 1;
-            fl &= fl - 1;
-            const uint32_t rf = __shfl_sync(kFull, row, f);
-            const uint32_t nf = __shfl_sync(kFull, nnz, f);
-            const uint32_t xf = __shfl_sync(kFull, x0, f);
-            const int zf = draw_exact_warp(nwk_row, a.denom, a.rows + static_cast<size_t>(rf) * 8, nf, xf, K,
-                                           a.alpha, a.beta, &q64x, &have_q);
-            if (lane == f) z = zf;
-            ++n_exact;
-        }
-        // ---- z and the fused recount
-        if (take) {
-            a.z[p] = static_cast<uint16_t>(z);
-            const unsigned act = __activemask();
-            const unsigned peers = __match_any_sync(act, z);
-            if (lane == __ffs(peers) - 1) {
-                const int c = __popc(peers);
-                atomicAdd(row_next + z, c);
-                atomicAdd(&nkh[z], c);
-            }
-        }
-        __syncwarp();
+        int z;
+        bool flag;
+        uint32_t x0;
+        tile_draw(a, take, c0, nl, row, crank, cb, Q64, gS, lsm, blk, p32, L32, Pc, NC, z, flag, x0);
+        tile_finish(a, take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q, n_exact);
         // ---- advance
         row = n_row;
         crank = n_crank;
@@ -1506,6 +1557,140 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
             itn = cn < a.n_items ? a.items[cn] : none;
             if (lane == 0 && cn < a.n_items && itn.word != it.word)
                 prefetch_l2_bulk(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
+        }
+    }
+    __syncthreads();
+    for (int k = threadIdx.x; k < K; k += blockDim.x)
+        if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
+    if (a.n_exact && lane == 0 && n_exact) atomicAdd(a.n_exact, static_cast<unsigned long long>(n_exact));
+}
+
+
+// ---------------------------------------------------------------------------
+// a3 + a4, tile sampler for large K (sampler 3): the 8 warps of a CTA share
+// the word table, double-buffered in shared memory -- at K = 8192 a per-warp
+// table (66 KB) would leave 2-3 warps per SM.  The CTA takes the work items
+// in queue order; its warps claim 32-token slots of the current item and walk
+// / draw them exactly as sweep_tile_kernel does (same helpers, same
+// certification); the last warp to leave an item refills that buffer with
+// the CTA's next item (bulk copy), while the other warps already work on the
+// item in the other buffer.
+// ---------------------------------------------------------------------------
+__host__ __device__ constexpr size_t tile_cta_warp_bytes(int lmax) {
+    return static_cast<size_t>(lmax) * (16 + 4 + 4) + 32 * 4 + 16;
+}
+__host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps) {
+    return static_cast<size_t>(4) * ((K + 3) & ~3) + 2 * tab_bytes(K) + nwarps * tile_cta_warp_bytes(lmax) + 64;
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+template <int R>
+__global__ void __launch_bounds__(256, 2) sweep_tile_cta_kernel(TileArgs a) {
+    extern __shared__ double smem_dd[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
+    const int K = a.K;
+    const int K4 = (K + 3) & ~3;
+    const int NC = (K + 127) / 128;
+    const int LM = a.lmax;
+    const size_t wt = a.wt_bytes;
+    int *nkh = reinterpret_cast<int *>(smem_dd);
+    char *tabs = reinterpret_cast<char *>(nkh + K4);
+    char *wb = tabs + 2 * wt + static_cast<size_t>(warp) * tile_cta_warp_bytes(LM);
+    float *blk = reinterpret_cast<float *>(wb);
+    float *lsm = blk + 4 * LM;
+    uint32_t *lrow = reinterpret_cast<uint32_t *>(lsm + LM);
+    char *ctrl = tabs + 2 * wt + static_cast<size_t>(nwarps) * tile_cta_warp_bytes(LM);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(ctrl);         // [2]
+    TileItem *items = reinterpret_cast<TileItem *>(ctrl + 16);  // [2]
+    uint32_t *slot = reinterpret_cast<uint32_t *>(ctrl + 48);   // [2]
+    uint32_t *left = slot + 2;                                  // [2]
+    const double gS = 9.5 * 5.9604644775390625e-08 * a.slack;
+
+    // buffer b <- the CTA's next work item (its table by bulk copy); the end
+    // of the queue is an item with n = 0
+    auto load = [&](int b) {
+        const uint32_t ci = atomicAdd(a.counter, 1u);
+        TileItem it = {0u, 0u, 0u, 0u};
+        if (ci < a.n_items) it = a.items[ci];
+        items[b] = it;
+        slot[b] = 0u;
+        left[b] = static_cast<uint32_t>(nwarps);
+        if (it.n) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive_expect_tx(bar + b, a.wt_bytes);
+            bulk_g2s(tabs + b * wt, a.wtab + static_cast<size_t>(it.word) * a.wt_bytes, a.wt_bytes, bar + b);
+        } else {
+            mbar_arrive(bar + b);
+        }
+    };
+    for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
+    if (threadIdx.x == 0) {
+        mbar_init(bar, 1);
+        mbar_init(bar + 1, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        load(0);
+        load(1);
+    }
+    __syncthreads();
+
+    unsigned n_exact = 0;
+    uint32_t ph[2] = {0u, 0u};
+    Blk8 ring[R];
+    bool hdr[R];
+    for (int b = 0;; b ^= 1) {
+        mbar_wait(bar + b, ph[b]);
+        ph[b] ^= 1u;
+        const TileItem it = items[b];
+        if (it.n == 0) break;
+        const double *Pc = reinterpret_cast<const double *>(tabs + b * wt);
+        const float *p32 = reinterpret_cast<const float *>(Pc + tab_nc2(K));
+        const float *L32 = p32 + K4;
+        const double Q64 = Pc[NC];
+        const uint64_t cb = __ldg(a.cbase + it.word);
+        const int32_t *nwk_row = a.nwk + static_cast<size_t>(it.word) * K;
+        int32_t *row_next = a.nwk_next + static_cast<size_t>(it.word) * K;
+        double q64x = 0.0;
+        int have_q = 0;
+        for (;;) {
+            uint32_t sl = 0;
+            if (lane == 0) sl = atomicAdd(slot + b, 1u);
+            sl = __shfl_sync(kFull, sl, 0);
+            if (32u * sl >= it.n) break;
+            const uint32_t t1 = min(it.n, 32u * sl + 32u);
+            for (uint32_t b0 = 32u * sl; b0 < t1;) {
+                const bool valid = b0 + lane < t1;
+                const uint32_t p = it.pos + b0 + lane;
+                uint32_t row = 0, crank = 0, nnz = 0;
+                if (valid) {
+                    row = __ldg(a.tok_row + p);
+                    crank = __ldg(a.tok_crank + p);
+                    nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
+                }
+                const TileHead hd = tile_head<R>(a, row, nnz, valid, LM, lrow, ring, hdr);
+                tile_walk<R>(a, hd.lsum, lrow, ring, hdr, p32, blk, lsm, [] {});
+                __syncwarp();
+                int z;
+                bool flag;
+                uint32_t x0;
+                tile_draw(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, lsm, blk, p32, L32, Pc, NC, z, flag,
+                          x0);
+                tile_finish(a, hd.take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q,
+                            n_exact);
+                b0 += static_cast<uint32_t>(hd.nb);
+            }
+        }
+        // leave the item; the last warp out refills the buffer
+        __syncwarp();
+        __threadfence_block();
+        uint32_t was = 0;
+        if (lane == 0) was = atomicSub(left + b, 1u);
+        was = __shfl_sync(kFull, was, 0);
+        if (was == 1u && lane == 0) {
+            __threadfence_block();
+            load(b);
         }
     }
     __syncthreads();
@@ -1820,9 +2005,34 @@ int configure_kernels(DevState &s) {
         // sampler -1 (auto): the tile sampler up to K = kTileMaxK; at large K its
         // per-warp tables of 8·K bytes leave too few warps per SM (measured at
         // K = 8192 on the NYTimes shape: sampler 0 is faster)
-        if (s.sampler < 0) s.sampler = s.K <= kTileMaxK ? 2 : 0;
+        if (s.sampler < 0) s.sampler = s.K <= kTileMaxK ? 2 : 3;
         s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1;
+        // large K: CTA-shared double-buffered tables (sweep_tile_cta_kernel)
+        const size_t cta_bytes = tile_cta_bytes(s.K, s.tile_lmax, 8);
+        s.sweep_tile_cta = s.sampler == 3 && !s.exclude_self && LDA_FUSE &&
+                           cta_bytes + 1024 <= static_cast<size_t>(max_optin);
+        if (s.sampler == 3 && !s.sweep_tile_cta) s.sampler = 0;
+        if (s.sweep_tile_cta) {
+            const void *fn = reinterpret_cast<const void *>(&sweep_tile_cta_kernel<LDA_TRING>);
+            s.tile_block = 256;
+            s.tile_smem = cta_bytes;
+            if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          static_cast<int>(s.tile_smem))) != cudaSuccess)
+                return e;
+            int bps = 1;
+            if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, s.tile_block, s.tile_smem)) !=
+                cudaSuccess)
+                return e;
+            s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
+            s.sweep_fused = true;
+        }
         s.wt_bytes = tab_bytes(s.K);
+        if (s.sweep_tile || s.sweep_tile_cta)
+            for (const void *f : {reinterpret_cast<const void *>(&word_table_kernel<true>),
+                                  reinterpret_cast<const void *>(&word_table_kernel<false>)})
+                if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) !=
+                    cudaSuccess)
+                    return e;
         if (s.sweep_tile) {
             const void *fn = reinterpret_cast<const void *>(&sweep_tile_kernel<LDA_TRING>);
             s.tile_block = 32 * wpc;
@@ -1836,11 +2046,6 @@ int configure_kernels(DevState &s) {
                 return e;
             s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
             s.sweep_fused = true;
-            for (const void *f : {reinterpret_cast<const void *>(&word_table_kernel<true>),
-                                  reinterpret_cast<const void *>(&word_table_kernel<false>)})
-                if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) !=
-                    cudaSuccess)
-                    return e;
         }
     }
     // recount
@@ -1934,7 +2139,7 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
     const int32_t *nk = s.nwk + static_cast<size_t>(s.V) * s.K;
     prologue_kernel<<<(s.K + 255) / 256, 256, 0, st>>>(nk, s.K, Vbeta, s.denom);
     ++*launches;
-    if (!s.sweep_tile && table_done_event &&
+    if (!s.sweep_tile && !s.sweep_tile_cta && table_done_event &&
         (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
         return e;
     if ((e = cudaMemsetAsync(s.counter, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
@@ -1953,7 +2158,7 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         a.nwk_next = nullptr;
         a.nk_next = nullptr;
     }
-    if (s.sweep_tile) {
+    if (s.sweep_tile || s.sweep_tile_cta) {
         // every row of the next n_wk is accumulated (words span tiles)
         if ((e = cudaMemsetAsync(s.nwk_alt, 0, sizeof(int32_t) * (static_cast<size_t>(s.V) * s.K + s.K), st)) !=
             cudaSuccess)
@@ -1995,7 +2200,10 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
             k0 += 0x9E3779B9u;
             k1 += 0xBB67AE85u;
         }
-        sweep_tile_kernel<LDA_TRING><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
+        if (s.sweep_tile_cta)
+            sweep_tile_cta_kernel<LDA_TRING><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
+        else
+            sweep_tile_kernel<LDA_TRING><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
         ++*launches;
         return cudaGetLastError();
     }

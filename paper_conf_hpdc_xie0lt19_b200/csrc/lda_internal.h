@@ -193,6 +193,7 @@ struct DevState {
     size_t quad_smem = 0;
     int quad_grid = 0;
     bool sweep_tile = false;        // the tile sampler is used (sampler 2, fits in smem, no exclude_self)
+    bool sweep_tile_cta = false;    // its large-K form with CTA-shared tables (sampler 3)
     size_t tile_smem = 0;
     int tile_grid = 0, tile_block = 0, tile_lmax = 160;
     char *wtab = nullptr;           // tile sampler: per-word tables (p32, dense prefix), rebuilt every sweep

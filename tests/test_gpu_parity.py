@@ -74,11 +74,12 @@ def test_tiny_config_free_running_ll_after_100():
     assert np.mean(g.z() != o.z) < 1e-3
 
 
-@pytest.mark.parametrize("sampler", [2, 1, 0])
+@pytest.mark.parametrize("sampler", [2, 3, 1, 0])
 @pytest.mark.parametrize("K", [1, 2, 37, 128, 1024])
 def test_k_variants_lockstep(K, sampler):
-    """Every sampler (2 = tile sampler, the default; 1 = quad per (word, doc)
-    pair; 0 = lane per token) against the oracle."""
+    """Every sampler (2 = tile sampler, the default; 3 = its CTA-shared-table
+    form for large K; 1 = quad per (word, doc) pair; 0 = lane per token)
+    against the oracle."""
     doc_ptr, words = _corpus(600, 700, 60_000, 0.7, 16, 11)
     a, b = 50.0 / K, 0.01
     o = U.oracle_for(600, 700, K, a, b, doc_ptr, words, 5)
@@ -90,9 +91,10 @@ def test_k_variants_lockstep(K, sampler):
     assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
 
 
-@pytest.mark.parametrize("sampler", [-1, 2])
+@pytest.mark.parametrize("sampler", [-1, 2, 0])
 def test_k8192_small(sampler):
-    """K = 8192: the default (auto -> sampler 0) and the tile sampler forced."""
+    """K = 8192: the default (auto -> the CTA tile sampler), the per-warp tile
+    sampler and the lane-per-token sampler forced."""
     doc_ptr, words = _corpus(300, 400, 40_000, 0.7, 64, 12)
     K = 8192
     o = U.oracle_for(300, 400, K, 50.0 / K, 0.01, doc_ptr, words, 9)
@@ -137,7 +139,7 @@ def test_exclude_self_lockstep():
     assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
-@pytest.mark.parametrize("sampler", [2, 1, 0])
+@pytest.mark.parametrize("sampler", [2, 3, 1, 0])
 def test_edge_cases(sampler):
     rng = np.random.default_rng(4)
     # empty docs, single-token docs, a 65535-token doc, absent words, D=1
@@ -171,15 +173,19 @@ def test_tile_sampler_decomposition_and_fallback_rate():
     ga = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=100_000)
     gb = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=0,
                      chunk_tokens=77)
+    gc = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=300_000,
+                     sampler=3)     # CTA-shared tables: same arithmetic, other batches
     g0 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, sampler=0)
     n_exact = 0
     for _ in range(6):
         ga.iterate(1)
         n_exact += ga.stats()["n_exact_redraws"]
         gb.iterate(1)
+        gc.iterate(1)
         g0.iterate(1)
         za = ga.z()
         assert np.array_equal(za, gb.z())
+        assert np.array_equal(za, gc.z())
         diff = np.count_nonzero(za != g0.z())
         assert diff <= 1e-6 * cfg.T + 2
         if diff:                       # keep the chains in lock step
@@ -187,8 +193,9 @@ def test_tile_sampler_decomposition_and_fallback_rate():
     assert n_exact <= 2e-3 * cfg.T * 6, n_exact
 
 
+@pytest.mark.parametrize("sampler", [2, 3])
 @pytest.mark.parametrize("K", [37, 1024])
-def test_tile_sampler_exact_redraw_path(K):
+def test_tile_sampler_exact_redraw_path(K, sampler):
     """Inflating the tile sampler's certification bounds (certify_slack) sends
     most tokens through the warp-collective fp64 redraw; the chains must still
     match the oracle in lock step (the redraw is the exact path, not a
@@ -196,8 +203,9 @@ def test_tile_sampler_exact_redraw_path(K):
     doc_ptr, words = _corpus(800, 900, 80_000, 0.7, 16, 31)
     a, b = 50.0 / K, 0.01
     o = U.oracle_for(800, 900, K, a, b, doc_ptr, words, 6)
-    g = U.gpu_model(800, 900, K, a, b, doc_ptr, words, 6, certify_slack=1 << 20, tile_tokens=20_000)
-    h = U.gpu_model(800, 900, K, a, b, doc_ptr, words, 6, tile_tokens=20_000)
+    g = U.gpu_model(800, 900, K, a, b, doc_ptr, words, 6, certify_slack=1 << 20, tile_tokens=20_000,
+                    sampler=sampler)
+    h = U.gpu_model(800, 900, K, a, b, doc_ptr, words, 6, tile_tokens=20_000, sampler=sampler)
     n_exact = 0
     for _ in range(3):
         margins = o.iterate(1, margins=True)
