@@ -386,7 +386,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // thread while the host prepares the next tile
     DA(S.tok_row, Tg);
     DA(S.doc_map, Tg);
-    DA(S.tok_crank, Tg);
+    const bool tile_layout = S.sweep_tile || S.sweep_tile_cta;
+    if (!tile_layout) DA(S.tok_crank, Tg);  // the tile samplers take ranks from their items
     lda::tmark("histogram, streams, configure");
     struct Job {
         uint64_t p0, p1, t0, t1;
@@ -413,7 +414,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             const size_t np = (j.p1 - j.p0) * sizeof(uint32_t), nt = (j.t1 - j.t0) * sizeof(uint32_t);
             if (np && r == cudaSuccess)
                 r = cudaMemcpyAsync(S.tok_row + j.p0, H.tok_row.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
-            if (np && r == cudaSuccess)
+            if (np && r == cudaSuccess && S.tok_crank)
                 r = cudaMemcpyAsync(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
             if (nt && r == cudaSuccess)
                 r = cudaMemcpyAsync(S.doc_map + j.t0, H.doc_map.data() + j.t0, nt, cudaMemcpyHostToDevice, cs);
@@ -431,7 +432,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     };
     std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens,
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
-                                      (S.sweep_tile || S.sweep_tile_cta) ? 2 : (S.sweep_quad ? 1 : 0),
+                                      tile_layout ? 2 : (S.sweep_quad ? 1 : 0),
                                       ctx->tail_per_tile, H,
                                       on_final);
     {

@@ -193,16 +193,24 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     const int nt = ndt + (any_tail ? 1 : 0);
     L.ntiles = nt;
 
-    if (!L.tok_row.allocate(T) || !L.doc_map.allocate(T) || !L.tok_crank.allocate(T))
+    // Tile samplers: documents keep their order inside each tile part, so a
+    // word's run holds its tokens in canonical order and a token's rank is
+    // its item's base + offset (no per-token rank table).  Samplers 0 / 1:
+    // documents by decreasing length inside a part (similar θ row lengths in
+    // a warp), ranks stored per token.
+    const bool tile_layout = sampler == 2;
+    if (!L.tok_row.allocate(T) || !L.doc_map.allocate(T) || (!tile_layout && !L.tok_crank.allocate(T)))
         return "host allocation of the token tables failed";
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
-    if (!ctmp.allocate(T)) return "host allocation of the token tables failed";
+    if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";
     // first touch in parallel (every entry is written below)
     parallel_for(nthreads, T, [&](int, int64_t b, int64_t e) {
         std::fill(L.tok_row.data() + b, L.tok_row.data() + e, 0u);
         std::fill(L.doc_map.data() + b, L.doc_map.data() + e, 0u);
-        std::fill(L.tok_crank.data() + b, L.tok_crank.data() + e, 0u);
-        std::fill(ctmp.data() + b, ctmp.data() + e, 0u);
+        if (!tile_layout) {
+            std::fill(L.tok_crank.data() + b, L.tok_crank.data() + e, 0u);
+            std::fill(ctmp.data() + b, ctmp.data() + e, 0u);
+        }
     });
     tmark("layout: host tables");
     std::vector<uint32_t> tseg(static_cast<size_t>(nt) * V, 0);  // run start of (tile, word)
@@ -224,6 +232,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             }
     }
     std::vector<uint32_t> crank_run(V, 0);   // tokens of each word in earlier tiles (canonical order)
+    std::vector<uint32_t> tcrank(static_cast<size_t>(nt) * V, 0);  // rank of a (tile, word) run's first token
     std::vector<std::vector<uint32_t>> cnt(nthreads, std::vector<uint32_t>(V));
     std::vector<std::vector<uint32_t>> pnext(nthreads, std::vector<uint32_t>(V));
     std::vector<std::vector<uint32_t>> cnext(nthreads, std::vector<uint32_t>(V));
@@ -260,6 +269,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         for (int32_t w = 0; w < V; ++w) {
             uint32_t run_p = tail[w] ? tail_next[w] : static_cast<uint32_t>(pos);
             uint32_t run_c = crank_run[w];
+            tcrank[static_cast<size_t>(b) * V + w] = run_c;
             if (!tail[w]) tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
             for (int t = 0; t < nth; ++t) {
                 const uint32_t h = cnt[t][w];
@@ -284,6 +294,18 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         // (The Philox counter does not depend on this order: each token
         // carries its canonical rank.)
         run_parts([&](int t) {
+            auto &next = pnext[t];
+            if (tile_layout) {
+                for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
+                    const uint32_t row = L.row_off32[d];
+                    for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
+                        const uint32_t p = next[words[i]]++;
+                        L.doc_map[i] = p;
+                        L.tok_row[p] = row;
+                    }
+                }
+                return;
+            }
             auto &cn = cnext[t];
             for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) ctmp[i] = cn[words[i]]++;
             std::vector<int64_t> ord(tdoc[t + 1] - tdoc[t]);
@@ -291,7 +313,6 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
             std::stable_sort(ord.begin(), ord.end(), [&](int64_t x, int64_t y) {
                 return doc_ptr[x + 1] - doc_ptr[x] > doc_ptr[y + 1] - doc_ptr[y];
             });
-            auto &next = pnext[t];
             for (const int64_t d : ord) {
                 const uint32_t row = L.row_off32[d];
                 for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
@@ -324,7 +345,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                 for (int64_t q = 0; q < pieces; ++q) {
                     const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
                     L.titems.push_back(TileItem{static_cast<uint32_t>(w), pos + static_cast<uint32_t>(vb),
-                                                static_cast<uint32_t>(ve - vb), static_cast<uint32_t>(b)});
+                                                static_cast<uint32_t>(ve - vb),
+                                                tcrank[static_cast<size_t>(b) * V + w] + static_cast<uint32_t>(vb)});
                 }
             }
             std::stable_sort(L.titems.begin() + first, L.titems.end(),

@@ -126,6 +126,21 @@ __global__ void init_kernel(const SampleChunk *__restrict__ chunks, int64_t n_ch
     }
 }
 
+// The same draw for the tile samplers' layout: token pos + j of an item has
+// canonical rank crank0 + j.
+__global__ void init_tile_kernel(const TileItem *__restrict__ items, int64_t n_items,
+                                 const uint64_t *__restrict__ cbase, uint16_t *__restrict__ z, uint32_t K,
+                                 uint32_t k0, uint32_t k1) {
+    for (int64_t ci = blockIdx.x; ci < n_items; ci += gridDim.x) {
+        const TileItem it = items[ci];
+        const uint64_t c0 = cbase[it.word] + it.crank0;
+        for (uint32_t j = threadIdx.x; j < it.n; j += blockDim.x) {
+            const uint32_t x0 = philox_x0(c0 + j, 0u, k0, k1);
+            z[it.pos + j] = static_cast<uint16_t>((static_cast<uint64_t>(x0) * K) >> 32);
+        }
+    }
+}
+
 // ---------------------------------------------------------------------------
 // a2: sweep prologue, denom[k] = n_k + Vβ  (fp64, Eq. 1 / Eq. 8 denominator).
 // ---------------------------------------------------------------------------
@@ -937,7 +952,6 @@ struct TileArgs {
     int64_t n_items;
     const uint64_t *cbase;     // V: canonical index of the rank's first token of each word
     const uint32_t *tok_row;   // word-major: θ row of the token's doc (32-byte units, 128-byte aligned)
-    const uint32_t *tok_crank; // word-major: canonical rank within the word
     uint16_t *z;
     const uint32_t *rows;
     const int32_t *nwk;        // frozen counts (V*K, n_k after)
@@ -1474,7 +1488,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     uint32_t row = 0, crank = 0, nnz = 0;
     if (lane < it.n) {
         row = __ldg(a.tok_row + it.pos + lane);
-        crank = __ldg(a.tok_crank + it.pos + lane);
+        crank = it.crank0 + lane;
         nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
     }
     TileHead hd = head(row, nnz, static_cast<uint32_t>(lane) < it.n);
@@ -1517,11 +1531,9 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
         const uint32_t nxt_pos = more ? it.pos + b1 : itn.pos;
         const uint32_t nxt_n = more ? it.n - b1 : (cn < a.n_items ? itn.n : 0u);
         const bool nxt_valid = static_cast<uint32_t>(lane) < nxt_n;
-        uint32_t n_row = 0, n_crank = 0, n_nnz = 0;
-        if (nxt_valid) {
-            n_row = __ldg(a.tok_row + nxt_pos + lane);
-            n_crank = __ldg(a.tok_crank + nxt_pos + lane);
-        }
+        uint32_t n_row = 0, n_nnz = 0;
+        const uint32_t n_crank = (more ? it.crank0 + b1 : itn.crank0) + lane;
+        if (nxt_valid) n_row = __ldg(a.tok_row + nxt_pos + lane);
         // ---- walk (the next batch's row headers issued after its first step)
         tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, lsm, [&] {
             if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
@@ -1666,7 +1678,7 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_cta_kernel(TileArgs a) {
                 uint32_t row = 0, crank = 0, nnz = 0;
                 if (valid) {
                     row = __ldg(a.tok_row + p);
-                    crank = __ldg(a.tok_crank + p);
+                    crank = it.crank0 + b0 + lane;
                     nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
                 }
                 const TileHead hd = tile_head<R>(a, row, nnz, valid, LM, lrow, ring, hdr);
@@ -2077,6 +2089,12 @@ int configure_kernels(DevState &s) {
 
 int launch_init(const DevState &s, void *stream) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (!s.tok_crank) {  // tile samplers' layout
+        const int g = static_cast<int>(std::min<int64_t>(s.n_titems > 0 ? s.n_titems : 1, 65535));
+        init_tile_kernel<<<g, 256, 0, st>>>(s.titems, s.n_titems, s.cbase, s.tok_z, static_cast<uint32_t>(s.K),
+                                            static_cast<uint32_t>(s.seed), static_cast<uint32_t>(s.seed >> 32));
+        return cudaGetLastError();
+    }
     const int grid = static_cast<int>(std::min<int64_t>(s.n_chunks > 0 ? s.n_chunks : 1, 65535));
     init_kernel<<<grid, 256, 0, st>>>(s.chunks, s.n_chunks, s.segs, s.tok_crank, s.tok_z, static_cast<uint32_t>(s.K),
                                       static_cast<uint32_t>(s.seed), static_cast<uint32_t>(s.seed >> 32));
@@ -2176,7 +2194,6 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.n_items = s.n_titems;
         ta.cbase = s.cbase;
         ta.tok_row = s.tok_row;
-        ta.tok_crank = s.tok_crank;
         ta.z = s.tok_z;
         ta.rows = s.rows;
         ta.nwk = s.nwk;

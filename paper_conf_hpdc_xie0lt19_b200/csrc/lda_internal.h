@@ -97,7 +97,8 @@ struct TileItem {
     uint32_t word;
     uint32_t pos;
     uint32_t n;
-    uint32_t tile;
+    uint32_t crank0;  // canonical rank (within the word, this rank) of the item's first token;
+                      // the run holds the word's tokens in canonical order: token pos + j has crank0 + j
 };
 
 // Host-side layout of one rank's shard (built by build_layout).
@@ -163,7 +164,7 @@ struct DevState {
     uint32_t *tok_row = nullptr;    // T
     uint16_t *tok_z = nullptr;      // T (word-major)
     uint32_t *doc_map = nullptr;    // T
-    uint32_t *tok_crank = nullptr;  // T (word-major)
+    uint32_t *tok_crank = nullptr;  // T (word-major); null for the tile samplers (ranks from the items)
     uint16_t *z_doc = nullptr;      // T, z in document order (two-phase θ rebuild only)
     uint32_t *doc_ptr32 = nullptr;  // D+1
     uint32_t *row_off32 = nullptr;  // D
