@@ -1401,6 +1401,8 @@ __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool f
                                             uint32_t nnz, uint32_t x0, uint32_t p, const int32_t *nwk_row,
                                             int32_t *row_next, int *nkh, double *q64x, int *have_q,
                                             unsigned &n_exact) {
+    // nkh: the n_k histogram -- the CTA's in shared memory, or the global
+    // next n_k (the large-K kernel keeps its shared memory for warps)
     const int lane = threadIdx.x & 31;
     const int K = a.K;
     // ---- exact fp64 redraw of the uncertain tokens, one at a time by the warp
@@ -1591,16 +1593,20 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
 __host__ __device__ constexpr size_t tile_cta_warp_bytes(int lmax) {
     return static_cast<size_t>(lmax) * (16 + 4 + 4) + 32 * 4 + 16;
 }
-__host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps) {
-    return static_cast<size_t>(4) * ((K + 3) & ~3) + 2 * tab_bytes(K) + nwarps * tile_cta_warp_bytes(lmax) + 64;
+__host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps, bool gnk) {
+    return (gnk ? 0 : static_cast<size_t>(4) * ((K + 3) & ~3)) + 2 * tab_bytes(K) + nwarps * tile_cta_warp_bytes(lmax) +
+           64;
 }
 
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-template <int R>
-__global__ void __launch_bounds__(256, 2) sweep_tile_cta_kernel(TileArgs a) {
+// GNK: n_k by warp-aggregated global reductions (large K: the shared memory
+// goes to warps); else a per-CTA shared histogram (global reductions on few
+// addresses contend at small K).
+template <int R, bool GNK>
+__global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     extern __shared__ double smem_dd[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     const int K = a.K;
@@ -1608,8 +1614,8 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_cta_kernel(TileArgs a) {
     const int NC = (K + 127) / 128;
     const int LM = a.lmax;
     const size_t wt = a.wt_bytes;
-    int *nkh = reinterpret_cast<int *>(smem_dd);
-    char *tabs = reinterpret_cast<char *>(nkh + K4);
+    int *nkh = GNK ? a.nk_next : reinterpret_cast<int *>(smem_dd);
+    char *tabs = reinterpret_cast<char *>(smem_dd) + (GNK ? 0 : 4 * K4);
     char *wb = tabs + 2 * wt + static_cast<size_t>(warp) * tile_cta_warp_bytes(LM);
     float *blk = reinterpret_cast<float *>(wb);
     float *lsm = blk + 4 * LM;
@@ -1638,7 +1644,8 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_cta_kernel(TileArgs a) {
             mbar_arrive(bar + b);
         }
     };
-    for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
+    if (!GNK)
+        for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
     if (threadIdx.x == 0) {
         mbar_init(bar, 1);
         mbar_init(bar + 1, 1);
@@ -1705,9 +1712,11 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_cta_kernel(TileArgs a) {
             load(b);
         }
     }
-    __syncthreads();
-    for (int k = threadIdx.x; k < K; k += blockDim.x)
-        if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
+    if (!GNK) {
+        __syncthreads();
+        for (int k = threadIdx.x; k < K; k += blockDim.x)
+            if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
+    }
     if (a.n_exact && lane == 0 && n_exact) atomicAdd(a.n_exact, static_cast<unsigned long long>(n_exact));
 }
 
@@ -2020,13 +2029,21 @@ int configure_kernels(DevState &s) {
         if (s.sampler < 0) s.sampler = s.K <= kTileMaxK ? 2 : 3;
         s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1;
         // large K: CTA-shared double-buffered tables (sweep_tile_cta_kernel)
-        const size_t cta_bytes = tile_cta_bytes(s.K, s.tile_lmax, 8);
-        s.sweep_tile_cta = s.sampler == 3 && !s.exclude_self && LDA_FUSE &&
-                           cta_bytes + 1024 <= static_cast<size_t>(max_optin);
+        s.tile_cta_gnk = s.K > kTileMaxK;
+        // as many warps as the shared memory holds: <= 16 at large K (one CTA per
+        // SM), <= 8 otherwise (two CTAs per SM: more items in flight)
+        const int cmax = s.tile_cta_gnk ? 16 : 8;
+        int cwarps = 0;
+        while (cwarps < cmax && tile_cta_bytes(s.K, s.tile_lmax, cwarps + 1, s.tile_cta_gnk) + 1024 <=
+                                  static_cast<size_t>(max_optin))
+            ++cwarps;
+        const size_t cta_bytes = tile_cta_bytes(s.K, s.tile_lmax, cwarps, s.tile_cta_gnk);
+        s.sweep_tile_cta = s.sampler == 3 && !s.exclude_self && LDA_FUSE && cwarps >= 2;
         if (s.sampler == 3 && !s.sweep_tile_cta) s.sampler = 0;
         if (s.sweep_tile_cta) {
-            const void *fn = reinterpret_cast<const void *>(&sweep_tile_cta_kernel<LDA_TRING>);
-            s.tile_block = 256;
+            const void *fn = s.tile_cta_gnk ? reinterpret_cast<const void *>(&sweep_tile_cta_kernel<LDA_TRING, true>)
+                                            : reinterpret_cast<const void *>(&sweep_tile_cta_kernel<LDA_TRING, false>);
+            s.tile_block = 32 * cwarps;
             s.tile_smem = cta_bytes;
             if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                           static_cast<int>(s.tile_smem))) != cudaSuccess)
@@ -2217,8 +2234,10 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
             k0 += 0x9E3779B9u;
             k1 += 0xBB67AE85u;
         }
-        if (s.sweep_tile_cta)
-            sweep_tile_cta_kernel<LDA_TRING><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
+        if (s.sweep_tile_cta && s.tile_cta_gnk)
+            sweep_tile_cta_kernel<LDA_TRING, true><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
+        else if (s.sweep_tile_cta)
+            sweep_tile_cta_kernel<LDA_TRING, false><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
         else
             sweep_tile_kernel<LDA_TRING><<<s.tile_grid, s.tile_block, s.tile_smem, st>>>(ta);
         ++*launches;
