@@ -165,6 +165,22 @@ int lda_partition_docs(int64_t D, const int64_t *doc_ptr, int32_t world, int64_t
 int lda_canonical_bases(int32_t V, int32_t world, int32_t rank, const int64_t *word_counts, int64_t *cbase,
                         int64_t *total);
 
+/* Host-only diagnostic (no device needed): build the token layout that
+ * lda_load_corpus would build for a one-rank corpus (doc_ptr: D+1 offsets,
+ * words: T ids < V) with the given sampler (0-3), tile_tokens,
+ * chunk_tokens and tail_per_tile, and check its invariants against brute
+ * force: doc_map is a permutation of [0, T); tok_row[doc_map[i]] is the θ
+ * row of token i's document; every (tile, word) run holds only that word;
+ * the runs of a word cover exactly its tokens; for the tile samplers every
+ * work item's token pos + j has canonical rank crank0 + j (the rank of the
+ * token within its word in (document, position) order, X18) and the items
+ * cover every token once.  out_stats (may be NULL) receives {tiles, items,
+ * tail words, runs}.  Returns LDA_OK, or LDA_EINVAL with a message in
+ * msg (msg_cap bytes) when an invariant fails or the input is invalid. */
+int lda_layout_selfcheck(int64_t D, int32_t V, int32_t K, const int64_t *doc_ptr, const int32_t *words,
+                         int32_t sampler, int64_t tile_tokens, int64_t chunk_tokens, int64_t tail_per_tile,
+                         int64_t *out_stats, char *msg, int32_t msg_cap);
+
 /* Load this rank's documents [doc_begin, doc_end) of the global corpus,
  * randomly initialise every token's topic (L377-379; Philox at t = 0, X10)
  * and build n_wk, n_k and θ (allreduced across ranks when world > 1).

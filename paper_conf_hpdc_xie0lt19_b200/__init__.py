@@ -24,7 +24,7 @@ STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4:
 
 # every symbol include/lda.h declares
 ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_partition_docs",
-               "lda_canonical_bases",
+               "lda_canonical_bases", "lda_layout_selfcheck",
                "lda_load_corpus", "lda_iterate", "lda_loglik", "lda_get_counts", "lda_get_stats",
                "lda_get_sweep_log", "lda_get_stream", "lda_set_z", "lda_destroy", "lda_last_error",
                "lda_version")
@@ -71,6 +71,8 @@ def lib():
             "lda_nccl_unique_id": ([_vp], ctypes.c_int),
             "lda_partition_docs": ([_i64, _vp, _i32, _vp], ctypes.c_int),
             "lda_canonical_bases": ([_i32, _i32, _i32, _vp, _vp, ctypes.POINTER(_i64)], ctypes.c_int),
+            "lda_layout_selfcheck": ([_i64, _i32, _i32, _vp, _vp, _i32, _i64, _i64, _i64, _vp, ctypes.c_char_p,
+                                      _i32], ctypes.c_int),
             "lda_load_corpus": ([_vp, _i64, _i64, _vp, _vp, _u64], ctypes.c_int),
             "lda_iterate": ([_vp, _i32], ctypes.c_int),
             "lda_loglik": ([_vp, ctypes.POINTER(_f64)], ctypes.c_int),
@@ -135,6 +137,20 @@ def lda_partition_docs(doc_ptr, world):
     out = np.empty(int(world) + 1, np.int64)
     _check(lib().lda_partition_docs(len(doc_ptr) - 1, _p(doc_ptr), int(world), _p(out)))
     return out
+
+
+def lda_layout_selfcheck(doc_ptr, words, V, K, sampler=2, tile_tokens=0, chunk_tokens=4096, tail_per_tile=64):
+    """Host-only check of the token layout (include/lda.h); returns
+    {tiles, items, tail_words, runs} or raises LDAError with the failed invariant."""
+    doc_ptr = np.ascontiguousarray(doc_ptr, np.int64)
+    words = np.ascontiguousarray(words, np.int32)
+    st = np.zeros(4, np.int64)
+    buf = ctypes.create_string_buffer(256)
+    r = lib().lda_layout_selfcheck(len(doc_ptr) - 1, int(V), int(K), _p(doc_ptr), _p(words), int(sampler),
+                                   int(tile_tokens), int(chunk_tokens), int(tail_per_tile), _p(st), buf, 256)
+    if r != 0:
+        raise LDAError(f"lda_layout_selfcheck: {buf.value.decode()} (status {r})")
+    return dict(zip(("tiles", "items", "tail_words", "runs"), st.tolist()))
 
 
 def lda_canonical_bases(word_counts, rank):

@@ -770,3 +770,98 @@ void lda_destroy(lda_ctx *ctx) {
 }
 
 }  // extern "C"
+
+int lda_layout_selfcheck(int64_t D, int32_t V, int32_t K, const int64_t *doc_ptr, const int32_t *words,
+                         int32_t sampler, int64_t tile_tokens, int64_t chunk_tokens, int64_t tail_per_tile,
+                         int64_t *out_stats, char *msg, int32_t msg_cap) {
+    auto bad = [&](const std::string &m) {
+        if (msg && msg_cap > 0) {
+            std::strncpy(msg, m.c_str(), static_cast<size_t>(msg_cap) - 1);
+            msg[msg_cap - 1] = 0;
+        }
+        return static_cast<int>(LDA_EINVAL);
+    };
+    if (D < 0 || V < 1 || K < 1 || !doc_ptr || sampler < 0 || sampler > 3 || chunk_tokens < 1)
+        return bad("invalid arguments");
+    bool range_err = false;
+    std::string v = lda::validate_corpus(doc_ptr, words, D, V, &range_err);
+    if (!v.empty()) return bad(v);
+    const int64_t T = doc_ptr[D];
+    std::vector<int64_t> cbase(V, 0), wc(V, 0);
+    lda::word_histogram(words, T, V, 0, wc.data());
+    lda_canonical_bases(V, 1, 0, wc.data(), cbase.data(), nullptr);
+    lda::HostLayout H;
+    const int layout = sampler >= 2 ? 2 : sampler;
+    std::string e = lda::build_layout(doc_ptr, words, D, V, K, cbase.data(), tile_tokens, chunk_tokens, 65536, 0,
+                                      layout, tail_per_tile, H);
+    if (!e.empty()) return bad(e);
+    // doc_map: a permutation; tok_row: the row of the token's document
+    std::vector<int64_t> word_at(T, -1), tokidx_at(T, -1);
+    for (int64_t d = 0; d < D; ++d)
+        for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
+            const uint32_t p = H.doc_map[i];
+            if (p >= static_cast<uint64_t>(T)) return bad("doc_map out of range");
+            if (word_at[p] >= 0) return bad("doc_map is not a permutation");
+            word_at[p] = words[i];
+            tokidx_at[p] = i;
+            if (H.tok_row[p] != H.row_off32[d]) return bad("tok_row is not the row of the token's document");
+        }
+    // canonical rank of each token by brute force: order within its word in (d, j) order
+    std::vector<int64_t> seen(V, 0), crank_at(T, -1);
+    for (int64_t i = 0; i < T; ++i) crank_at[H.doc_map[i]] = seen[words[i]]++;
+    // runs: each word's runs (segs) cover exactly its tokens and hold only that word
+    int64_t runs = 0;
+    {
+        // per word: runs {pos, vstart} ..., then a sentinel {0, n_w}
+        size_t sidx = 0;
+        for (int32_t w = 0; w < V; ++w) {
+            int64_t covered = 0;
+            while (sidx + 1 < H.segs.size() && H.segs[sidx].vstart < static_cast<uint64_t>(wc[w])) {
+                const lda::Seg &sg = H.segs[sidx];
+                const uint32_t len = H.segs[sidx + 1].vstart - sg.vstart;
+                for (uint32_t j = 0; j < len; ++j)
+                    if (word_at[static_cast<size_t>(sg.pos) + j] != w) return bad("a word's run holds another word");
+                covered += len;
+                ++runs;
+                ++sidx;
+            }
+            if (sidx >= H.segs.size() || H.segs[sidx].vstart != static_cast<uint64_t>(wc[w]))
+                return bad("missing run sentinel");
+            ++sidx;
+            if (covered != wc[w]) return bad("a word's runs do not cover its tokens");
+        }
+    }
+    // tile-sampler items: canonical ranks crank0 + j, every token once
+    if (layout == 2) {
+        std::vector<uint8_t> hit(T, 0);
+        for (const lda::TileItem &it : H.titems) {
+            for (uint32_t j = 0; j < it.n; ++j) {
+                const uint64_t p = static_cast<uint64_t>(it.pos) + j;
+                if (p >= static_cast<uint64_t>(T)) return bad("item out of range");
+                if (hit[p]) return bad("a token is in two items");
+                hit[p] = 1;
+                if (word_at[p] != static_cast<int64_t>(it.word)) return bad("an item holds another word");
+                if (crank_at[p] != static_cast<int64_t>(it.crank0) + j)
+                    return bad("item canonical rank crank0 + j differs from the brute-force rank");
+            }
+        }
+        for (int64_t p = 0; p < T; ++p)
+            if (!hit[p]) return bad("a token is in no item");
+    } else {
+        for (int64_t p = 0; p < T; ++p)
+            if (static_cast<int64_t>(H.tok_crank[p]) != crank_at[p]) return bad("tok_crank differs from the brute-force rank");
+    }
+    int64_t ntail = 0;
+    if (layout == 2 && H.ntiles > 1) {
+        // tail words: exactly one run, in the last tile
+        for (int32_t w = 0; w < V; ++w)
+            if (wc[w] > 0 && wc[w] < tail_per_tile * (H.ntiles - 1)) ++ntail;
+    }
+    if (out_stats) {
+        out_stats[0] = H.ntiles;
+        out_stats[1] = static_cast<int64_t>(layout == 2 ? H.titems.size() : H.chunks.size());
+        out_stats[2] = ntail;
+        out_stats[3] = runs;
+    }
+    return LDA_OK;
+}

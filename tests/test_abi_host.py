@@ -121,3 +121,36 @@ def test_no_gpu_fails_loudly():
         assert e2.value.code == L.LDA_ECUDA
     finally:
         L.lda_destroy(ctx)
+
+
+def _corpus(D, V, seed, max_len=40, empty=True):
+    rng = np.random.default_rng(seed)
+    L_d = rng.integers(0 if empty else 1, max_len, size=D)
+    doc_ptr = np.concatenate([[0], np.cumsum(L_d)]).astype(np.int64)
+    # Zipf-like word frequencies: heavy heads, many rare words (tail tile)
+    p = 1.0 / np.arange(1, V + 1)
+    words = rng.choice(V, size=int(doc_ptr[-1]), p=p / p.sum()).astype(np.int32)
+    return doc_ptr, words
+
+
+@pytest.mark.parametrize("sampler", [0, 1, 2, 3])
+@pytest.mark.parametrize("tile_tokens,chunk_tokens,tail", [(0, 4096, 64), (900, 4096, 64), (700, 33, 8),
+                                                            (500, 7, 1000), (300, 64, 0)])
+def test_layout_invariants(sampler, tile_tokens, chunk_tokens, tail):
+    """The host token layout (no GPU): doc_map a permutation, rows per token,
+    runs per word, and -- for the tile samplers -- canonical ranks
+    crank0 + j for every item token (checked against brute force)."""
+    doc_ptr, words = _corpus(400, 300, 5)
+    st = L.lda_layout_selfcheck(doc_ptr, words, 300, 24, sampler=sampler, tile_tokens=tile_tokens,
+                                chunk_tokens=chunk_tokens, tail_per_tile=tail)
+    if sampler >= 2 and tile_tokens and tail:
+        assert st["tiles"] >= 2 and st["tail_words"] > 0      # the tail tile is exercised
+    assert st["items"] > 0 and st["runs"] > 0
+
+
+def test_layout_selfcheck_rejects_bad_input():
+    doc_ptr, words = _corpus(10, 20, 1)
+    bad = words.copy()
+    bad[0] = 20                                               # word id >= V
+    with pytest.raises(L.LDAError):
+        L.lda_layout_selfcheck(doc_ptr, bad, 20, 4)
