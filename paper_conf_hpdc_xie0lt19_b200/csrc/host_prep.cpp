@@ -154,6 +154,9 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         L.row_off32[d] = static_cast<uint32_t>(off32);
         off32 += 4 * static_cast<uint64_t>((cap + 1 + 31) / 32);
         if (off32 >= (uint64_t(1) << 32) - 64) return "θ row storage exceeds 2^32 x 32 bytes";
+        // the tile samplers' line tables flag a row's first line in bit 31
+        if (sampler == 2 && off32 >= (uint64_t(1) << 31) - 64)
+            return "θ row storage exceeds 2^31 x 32 bytes (64 GB) on one rank: use more ranks or sampler 0";
     }
     L.doc_ptr32[D] = static_cast<uint32_t>(T);
     L.rows32 = off32 + 4;  // tail pad
