@@ -531,7 +531,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     ctx->stats.local_docs = Dg;
     ctx->stats.global_tokens = ctx->T_global;
     ctx->stats.world = ctx->world;
-    ctx->stats.n_sample_chunks = S.n_chunks;
+    ctx->stats.n_sample_chunks = (S.sweep_tile || S.sweep_tile_cta) ? S.n_titems : S.n_chunks;
     ctx->stats.sum_nnz_doc = ctx->cur_nnz;
     return LDA_OK;
 }

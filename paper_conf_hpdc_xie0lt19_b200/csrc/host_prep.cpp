@@ -387,26 +387,28 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // canonical index continues word w's run on this rank (cbase[w] + v).
     L.chunks.clear();
     L.zero_words.clear();
-    for (int32_t w = 0; w < V; ++w) {
-        const int64_t n = L.word_count[w];
-        const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
-        if (pieces != 1) L.zero_words.push_back(w);
-        if (n == 0) continue;
-        for (int64_t q = 0; q < pieces; ++q) {
-            const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
-            SampleChunk c;
-            c.word = static_cast<uint32_t>(w);
-            c.vbegin = static_cast<uint32_t>(vb);
-            c.count = static_cast<uint32_t>(ve - vb);
-            c.seg0 = seg_of(w, static_cast<uint32_t>(vb));
-            c.segN = static_cast<uint32_t>(wseg0[w + 1] - 1);
-            c.pad = pieces > 1 ? 1u : 0u;  // bit 0: the word is split over chunks
-            c.c_base = static_cast<uint64_t>(cbase[w]);
-            L.chunks.push_back(c);
+    if (sampler != 2) {  // samplers 0 / 1 only (the tile samplers use their own items)
+        for (int32_t w = 0; w < V; ++w) {
+            const int64_t n = L.word_count[w];
+            const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
+            if (pieces != 1) L.zero_words.push_back(w);
+            if (n == 0) continue;
+            for (int64_t q = 0; q < pieces; ++q) {
+                const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
+                SampleChunk c;
+                c.word = static_cast<uint32_t>(w);
+                c.vbegin = static_cast<uint32_t>(vb);
+                c.count = static_cast<uint32_t>(ve - vb);
+                c.seg0 = seg_of(w, static_cast<uint32_t>(vb));
+                c.segN = static_cast<uint32_t>(wseg0[w + 1] - 1);
+                c.pad = pieces > 1 ? 1u : 0u;  // bit 0: the word is split over chunks
+                c.c_base = static_cast<uint64_t>(cbase[w]);
+                L.chunks.push_back(c);
+            }
         }
+        std::stable_sort(L.chunks.begin(), L.chunks.end(),
+                         [](const SampleChunk &a, const SampleChunk &b) { return a.count > b.count; });
     }
-    std::stable_sort(L.chunks.begin(), L.chunks.end(),
-                     [](const SampleChunk &a, const SampleChunk &b) { return a.count > b.count; });
 
     tmark("layout: runs + sampler chunks");
     // Quad-sampler items: the same word chunks, their tokens (virtual order:
