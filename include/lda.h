@@ -118,9 +118,11 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   0: lane-per-token fp64 sampler (32-byte row blocks).
  *                   The samplers differ only in rounding at a CDF boundary
  *                   (draws differ only within fp64 rounding of it).
- *   "tail_per_tile" sampler 2: words with fewer than this many tokens per
- *                   document tile on average are sampled as one corpus-wide
- *                   item each (default 64; 0 = off)
+ *   "tail_per_tile" samplers 2, 3: words with fewer than this many tokens
+ *                   per document tile on average are sampled as one
+ *                   corpus-wide item each (default 64; 0 = off).  Sampler 3
+ *                   scales it and tile_tokens by K/1024 (its per-item table
+ *                   copy grows with K).
  *   "certify_slack" sampler 2, tests only: multiply every certification
  *                   bound by this factor (default 1) -- more tokens take the
  *                   exact fp64 redraw; the draws must not change
