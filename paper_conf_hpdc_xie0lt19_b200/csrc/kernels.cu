@@ -966,6 +966,7 @@ struct TileArgs {
     double slack;              // multiplier of every certification bound (1; > 1 only in tests)
     const char *wtab;          // word tables (word_table_kernel), wt_bytes per word
     uint32_t wt_bytes;
+    int nbuf;                  // sweep_tile_cta_kernel: table buffers per CTA
     uint32_t t;
     uint32_t key0[10], key1[10];
 };
@@ -1075,8 +1076,16 @@ __host__ __device__ constexpr size_t tab_bytes(int K) {
            static_cast<size_t>(4) * 128 * ((K + 127) / 128);
 }
 __host__ __device__ constexpr int l32_idx(int k) { return k ^ (((k >> 7) & 7) << 2); }
+// Compact layout (the large-K CTA sampler, which keeps several tables per
+// CTA): [Pg: fp64 prefix of α·p* at the start of every 32-topic group, then
+// Pg[G] = Q, padded to an even count][p32: K4 floats] -- the in-group prefix
+// is summed on the fly from p32 (at most 32 terms).
+__host__ __device__ constexpr int tab_g2(int K) { return ((K + 31) / 32 + 2) / 2 * 2; }
+__host__ __device__ constexpr size_t tab_bytes_compact(int K) {
+    return static_cast<size_t>(tab_g2(K)) * 8 + static_cast<size_t>(4) * ((K + 3) & ~3);
+}
 
-template <bool VEC>
+template <bool VEC, bool COMPACT>
 __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double *__restrict__ denom, int V, int K,
                                   double alpha, double beta, char *__restrict__ tab) {
     extern __shared__ double inv64[];
@@ -1084,12 +1093,12 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
     for (int k = threadIdx.x; k < K; k += blockDim.x) inv64[k] = 1.0 / denom[k];
     __syncthreads();
     const int K4 = (K + 3) & ~3;
-    const size_t wt = tab_bytes(K);
+    const size_t wt = COMPACT ? tab_bytes_compact(K) : tab_bytes(K);
     const int nwarp = gridDim.x * (blockDim.x >> 5);
     for (int w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < V; w += nwarp) {
         const int32_t *nwk_row = nwk + static_cast<size_t>(w) * K;
         double *Pc = reinterpret_cast<double *>(tab + wt * w);
-        float *p32 = reinterpret_cast<float *>(Pc + tab_nc2(K));
+        float *p32 = reinterpret_cast<float *>(Pc + (COMPACT ? tab_g2(K) : tab_nc2(K)));
         float *L32 = p32 + K4;
         double carry = 0.0;
         for (int k0 = 0, c = 0; k0 < K; k0 += 128, ++c) {
@@ -1125,24 +1134,35 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
             }
             double excl = __shfl_up_sync(kFull, incl, 1);
             if (lane == 0) excl = 0.0;
-            const float f0 = d2f_trunc(excl + l0), f1 = d2f_trunc(excl + l1);
-            const float f2 = d2f_trunc(excl + l2), f3 = d2f_trunc(excl + l3);
-            if (VEC) {
-                if (k < K) *reinterpret_cast<float4 *>(L32 + l32_idx(k)) = make_float4(f0, f1, f2, f3);
+            if (COMPACT) {
+                // lane 8g starts group g of this chunk: its base is the group's prefix
+                if ((lane & 7) == 0 && k < K) Pc[4 * c + (lane >> 3)] = carry + excl;
             } else {
-                const float ff[4] = {f0, f1, f2, f3};
+                const float f0 = d2f_trunc(excl + l0), f1 = d2f_trunc(excl + l1);
+                const float f2 = d2f_trunc(excl + l2), f3 = d2f_trunc(excl + l3);
+                if (VEC) {
+                    if (k < K) *reinterpret_cast<float4 *>(L32 + l32_idx(k)) = make_float4(f0, f1, f2, f3);
+                } else {
+                    const float ff[4] = {f0, f1, f2, f3};
 #pragma unroll
-                for (int e = 0; e < 4; ++e)
-                    if (k + e < K) L32[l32_idx(k + e)] = ff[e];
+                    for (int e = 0; e < 4; ++e)
+                        if (k + e < K) L32[l32_idx(k + e)] = ff[e];
+                }
+                if (lane == 0) Pc[c] = carry;
             }
-            if (lane == 0) Pc[c] = carry;
             carry += __shfl_sync(kFull, incl, 31);
         }
-        if (lane == 0) Pc[(K + 127) / 128] = carry;
         // zero the padding so that the table bytes are deterministic
-        if (lane == 1 && tab_nc2(K) > (K + 127) / 128 + 1) Pc[tab_nc2(K) - 1] = 0.0;
+        if (COMPACT) {
+            const int G = (K + 31) / 32;
+            if (lane == 0) Pc[G] = carry;
+            if (lane == 1 && tab_g2(K) > G + 1) Pc[tab_g2(K) - 1] = 0.0;
+        } else {
+            if (lane == 0) Pc[(K + 127) / 128] = carry;
+            if (lane == 1 && tab_nc2(K) > (K + 127) / 128 + 1) Pc[tab_nc2(K) - 1] = 0.0;
+            for (int k = K + lane; k < 128 * ((K + 127) / 128); k += 32) L32[l32_idx(k)] = 0.0f;
+        }
         for (int k = K + lane; k < K4; k += 32) p32[k] = 0.0f;
-        for (int k = K + lane; k < 128 * ((K + 127) / 128); k += 32) L32[l32_idx(k)] = 0.0f;
     }
 }
 
@@ -1291,6 +1311,7 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
 // comparisons; the draw is then certified by the margins of the two prefixes
 // that bracket x, each against a rigorous bound on its error (the other
 // prefixes are farther from x by monotonicity); uncertain -> flag.
+template <bool COMPACT = false>
 __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t c0, uint32_t nl, uint32_t row,
                                           uint32_t crank, uint64_t cb, double Q64, double gS, const float *lsm,
                                           const float *blk, const float *p32, const float *L32, const double *Pc,
@@ -1363,6 +1384,45 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
                 flag = flag || (se - r32 <= fmaf(6.2e-7f * g32, se, eR)) ||
                        (sp > 0.0f && r32 - sp <= fmaf(6.2e-7f * g32, sp, eR));   // (2u + 8u)·s
                 z = static_cast<int>(we >> kTS);
+            }
+        } else if (COMPACT) {
+            // dense bucket, compact table: the 32-topic group by its fp64 base
+            // Pg (Pc here, NC = G groups), then the in-group prefix summed in
+            // fp32 from p32 (p32 2u, α u, <= 32 FMA roundings: 35u)
+            const double y = U * Q64 - (1.0 - U) * S;
+            const double ey = (1.0 - U) * gS * S + eps;
+            int g = 0;
+            for (int n = NC; n > 1;) {  // last group g with Pg[g] <= y
+                const int h = n >> 1;
+                if (Pc[g + h] <= y) g += h;
+                n -= h;
+            }
+            const double r = y - Pc[g];
+            const float r32 = static_cast<float>(r);
+            const float eR = static_cast<float>((ey + u * fabs(r)) * 1.0001 + 1e-30);
+            const float a32 = static_cast<float>(a.alpha);
+            const int kb = 32 * g, kn = min(K, kb + 32) - kb;
+            float l = 0.0f, lp = 0.0f, le = 0.0f;
+            int k = -1;
+            for (int j = 0; j < kn; ++j) {
+                const float ln = fmaf(a32, p32[kb + j], l);
+                if (ln > r32) {
+                    k = j;
+                    lp = l;
+                    le = ln;
+                    break;
+                }
+                l = ln;
+            }
+            if (k < 0) {  // none in the group: the last topic (X6 when it is K-1)
+                k = kn - 1;
+                z = kb + k;
+                flag = z < K - 1 || (k > 0 && r32 - l <= fmaf(2.2e-6f * g32, l, eR));
+            } else {
+                z = kb + k;
+                flag = (z < K - 1 && le - r32 <= fmaf(2.2e-6f * g32, le, eR)) ||
+                       (k > 0 && r32 - lp <= fmaf(2.2e-6f * g32, lp, eR)) ||
+                       (k == 0 && g > 0 && r <= ey);
             }
         } else {
             // dense bucket: first k with P[k] > y = x - S = U·Q - (1-U)·S;
@@ -1593,9 +1653,11 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
 __host__ __device__ constexpr size_t tile_cta_warp_bytes(int lmax) {
     return static_cast<size_t>(lmax) * (16 + 4 + 4) + 32 * 4 + 16;
 }
-__host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps, bool gnk) {
-    return (gnk ? 0 : static_cast<size_t>(4) * ((K + 3) & ~3)) + 2 * tab_bytes(K) + nwarps * tile_cta_warp_bytes(lmax) +
-           64;
+// large K (gnk): compact tables and n_k by global reductions; nb table buffers (<= 4)
+__host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps, bool gnk, int nb) {
+    return (gnk ? 0 : static_cast<size_t>(4) * ((K + 3) & ~3)) +
+           static_cast<size_t>(nb) * (gnk ? tab_bytes_compact(K) : tab_bytes(K)) +
+           nwarps * tile_cta_warp_bytes(lmax) + 128;
 }
 
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
@@ -1611,20 +1673,21 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     const int K = a.K;
     const int K4 = (K + 3) & ~3;
-    const int NC = (K + 127) / 128;
+    const int NC = GNK ? (K + 31) / 32 : (K + 127) / 128;  // groups of the dense prefix's fp64 level
     const int LM = a.lmax;
+    const int NB = a.nbuf;  // table buffers (2..4): items in flight per CTA
     const size_t wt = a.wt_bytes;
     int *nkh = GNK ? a.nk_next : reinterpret_cast<int *>(smem_dd);
     char *tabs = reinterpret_cast<char *>(smem_dd) + (GNK ? 0 : 4 * K4);
-    char *wb = tabs + 2 * wt + static_cast<size_t>(warp) * tile_cta_warp_bytes(LM);
+    char *wb = tabs + NB * wt + static_cast<size_t>(warp) * tile_cta_warp_bytes(LM);
     float *blk = reinterpret_cast<float *>(wb);
     float *lsm = blk + 4 * LM;
     uint32_t *lrow = reinterpret_cast<uint32_t *>(lsm + LM);
-    char *ctrl = tabs + 2 * wt + static_cast<size_t>(nwarps) * tile_cta_warp_bytes(LM);
-    uint64_t *bar = reinterpret_cast<uint64_t *>(ctrl);         // [2]
-    TileItem *items = reinterpret_cast<TileItem *>(ctrl + 16);  // [2]
-    uint32_t *slot = reinterpret_cast<uint32_t *>(ctrl + 48);   // [2]
-    uint32_t *left = slot + 2;                                  // [2]
+    char *ctrl = tabs + NB * wt + static_cast<size_t>(nwarps) * tile_cta_warp_bytes(LM);
+    uint64_t *bar = reinterpret_cast<uint64_t *>(ctrl);         // [4]
+    TileItem *items = reinterpret_cast<TileItem *>(ctrl + 32);  // [4]
+    uint32_t *slot = reinterpret_cast<uint32_t *>(ctrl + 96);   // [4]
+    uint32_t *left = slot + 4;                                  // [4]
     const double gS = 9.5 * 5.9604644775390625e-08 * a.slack;
 
     // buffer b <- the CTA's next work item (its table by bulk copy); the end
@@ -1647,25 +1710,23 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     if (!GNK)
         for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
     if (threadIdx.x == 0) {
-        mbar_init(bar, 1);
-        mbar_init(bar + 1, 1);
+        for (int b = 0; b < NB; ++b) mbar_init(bar + b, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        load(0);
-        load(1);
+        for (int b = 0; b < NB; ++b) load(b);
     }
     __syncthreads();
 
     unsigned n_exact = 0;
-    uint32_t ph[2] = {0u, 0u};
+    uint32_t phases = 0u;  // bit b: the parity of buffer b's next completion
     Blk8 ring[R];
     bool hdr[R];
-    for (int b = 0;; b ^= 1) {
-        mbar_wait(bar + b, ph[b]);
-        ph[b] ^= 1u;
+    for (int b = 0;; b = b + 1 < NB ? b + 1 : 0) {
+        mbar_wait(bar + b, (phases >> b) & 1u);
+        phases ^= 1u << b;
         const TileItem it = items[b];
         if (it.n == 0) break;
         const double *Pc = reinterpret_cast<const double *>(tabs + b * wt);
-        const float *p32 = reinterpret_cast<const float *>(Pc + tab_nc2(K));
+        const float *p32 = reinterpret_cast<const float *>(Pc + (GNK ? tab_g2(K) : tab_nc2(K)));
         const float *L32 = p32 + K4;
         const double Q64 = Pc[NC];
         const uint64_t cb = __ldg(a.cbase + it.word);
@@ -1694,8 +1755,8 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
                 int z;
                 bool flag;
                 uint32_t x0;
-                tile_draw(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, lsm, blk, p32, L32, Pc, NC, z, flag,
-                          x0);
+                tile_draw<GNK>(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, lsm, blk, p32, L32, Pc, NC, z,
+                               flag, x0);
                 tile_finish(a, hd.take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q,
                             n_exact);
                 b0 += static_cast<uint32_t>(hd.nb);
@@ -2030,14 +2091,25 @@ int configure_kernels(DevState &s) {
         s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1;
         // large K: CTA-shared double-buffered tables (sweep_tile_cta_kernel)
         s.tile_cta_gnk = s.K > kTileMaxK;
-        // as many warps as the shared memory holds: <= 16 at large K (one CTA per
-        // SM), <= 8 otherwise (two CTAs per SM: more items in flight)
+        // large K: one CTA per SM with up to 4 compact table buffers, keeping
+        // >= 12 warps; else two 8-warp CTAs per SM with 2 buffers each
         const int cmax = s.tile_cta_gnk ? 16 : 8;
-        int cwarps = 0;
-        while (cwarps < cmax && tile_cta_bytes(s.K, s.tile_lmax, cwarps + 1, s.tile_cta_gnk) + 1024 <=
-                                  static_cast<size_t>(max_optin))
-            ++cwarps;
-        const size_t cta_bytes = tile_cta_bytes(s.K, s.tile_lmax, cwarps, s.tile_cta_gnk);
+        auto fit = [&](int nb) {
+            int w = 0;
+            while (w < cmax && tile_cta_bytes(s.K, s.tile_lmax, w + 1, s.tile_cta_gnk, nb) + 1024 <=
+                                   static_cast<size_t>(max_optin))
+                ++w;
+            return w;
+        };
+        s.tile_nbuf = 2;
+        if (s.tile_cta_gnk)
+            for (int nb = 4; nb > 2; --nb)
+                if (fit(nb) >= 12) {
+                    s.tile_nbuf = nb;
+                    break;
+                }
+        const int cwarps = fit(s.tile_nbuf);
+        const size_t cta_bytes = tile_cta_bytes(s.K, s.tile_lmax, cwarps, s.tile_cta_gnk, s.tile_nbuf);
         s.sweep_tile_cta = s.sampler == 3 && !s.exclude_self && LDA_FUSE && cwarps >= 2;
         if (s.sampler == 3 && !s.sweep_tile_cta) s.sampler = 0;
         if (s.sweep_tile_cta) {
@@ -2055,10 +2127,12 @@ int configure_kernels(DevState &s) {
             s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
             s.sweep_fused = true;
         }
-        s.wt_bytes = tab_bytes(s.K);
+        s.wt_bytes = s.sweep_tile_cta && s.tile_cta_gnk ? tab_bytes_compact(s.K) : tab_bytes(s.K);
         if (s.sweep_tile || s.sweep_tile_cta)
-            for (const void *f : {reinterpret_cast<const void *>(&word_table_kernel<true>),
-                                  reinterpret_cast<const void *>(&word_table_kernel<false>)})
+            for (const void *f : {reinterpret_cast<const void *>(&word_table_kernel<true, false>),
+                                  reinterpret_cast<const void *>(&word_table_kernel<false, false>),
+                                  reinterpret_cast<const void *>(&word_table_kernel<true, true>),
+                                  reinterpret_cast<const void *>(&word_table_kernel<false, true>)})
                 if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) !=
                     cudaSuccess)
                     return e;
@@ -2199,10 +2273,19 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
             cudaSuccess)
             return e;
         const int wtb = static_cast<int>(std::min<int64_t>((static_cast<int64_t>(s.V) + 7) / 8, 8 * s.num_sms));
-        if ((s.K & 3) == 0)
-            word_table_kernel<true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta, s.wtab);
+        const bool compact = s.sweep_tile_cta && s.tile_cta_gnk;
+        if ((s.K & 3) == 0 && compact)
+            word_table_kernel<true, true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
+                                                                     s.wtab);
+        else if (compact)
+            word_table_kernel<false, true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
+                                                                      s.wtab);
+        else if ((s.K & 3) == 0)
+            word_table_kernel<true, false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
+                                                                      s.wtab);
         else
-            word_table_kernel<false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta, s.wtab);
+            word_table_kernel<false, false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
+                                                                       s.wtab);
         ++*launches;
         if (table_done_event && (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
             return e;
@@ -2226,6 +2309,7 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.slack = s.certify_slack;
         ta.wtab = s.wtab;
         ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
+        ta.nbuf = s.tile_nbuf;
         ta.t = t;
         uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
         for (int r = 0; r < 10; ++r) {

@@ -194,7 +194,7 @@ def test_tile_sampler_decomposition_and_fallback_rate():
 
 
 @pytest.mark.parametrize("sampler", [2, 3])
-@pytest.mark.parametrize("K", [37, 1024])
+@pytest.mark.parametrize("K", [37, 1024, 8192])
 def test_tile_sampler_exact_redraw_path(K, sampler):
     """Inflating the tile sampler's certification bounds (certify_slack) sends
     most tokens through the warp-collective fp64 redraw; the chains must still
