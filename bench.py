@@ -254,8 +254,8 @@ def run_b200(args):
     ms = ev0.elapsed_time(ev1)
     st = m.stats()
     log = m.sweep_log()
-    t = torch.tensor([ms, st["ms_sample"], st["ms_allreduce"], st["ms_theta"], st["ms_recount"]],
-                     device=dev, dtype=torch.float64)
+    t = torch.tensor([ms, st["ms_sample"], st["ms_allreduce"], st["ms_theta"], st["ms_recount"],
+                      st["ms_allreduce_exposed"]], device=dev, dtype=torch.float64)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms_max = float(t[0])
@@ -317,7 +317,8 @@ def run_b200(args):
                                    "word_tables": float(st["ms_table"]) / args.steps,
                                    "recount": float(t[4]) / args.steps,
                                    "theta": float(t[3]) / args.steps,
-                                   "allreduce_raw": float(t[2]) / args.steps},
+                                   "allreduce_raw": float(t[2]) / args.steps,
+                                   "allreduce_exposed": float(t[5]) / args.steps},
             "nnz_per_token": mean_nnz,
             "exact_redraws_per_step": st["n_exact_redraws"] / args.steps,
             "per_sweep_ms": [round(x, 4) for x in log["ms_sweep"].tolist()],

@@ -78,8 +78,11 @@ typedef struct lda_stats {
     int64_t n_exact_redraws;/* samplers 1, 2: tokens of the last lda_iterate
                                call whose fp32 draw could not be certified and
                                that were redrawn by the exact fp64 walk */
-    double ms_table;        /* sampler 2: the per-word table kernel (a3), part of
+    double ms_table;        /* samplers 2, 3: the per-word table kernel (a3), part of
                                ms_sample; ms_sample - ms_table = sampling kernel */
+    double ms_allreduce_exposed; /* world > 1: time the compute stream waited for
+                               the allreduce after the θ rebuild (the part of
+                               ms_allreduce not hidden behind it) */
 } lda_stats;
 
 /* Create a context.  D = global number of documents, V = vocabulary size,

@@ -46,7 +46,7 @@ class lda_stats(ctypes.Structure):
                 ("ms_last_sample", ctypes.c_double), ("sum_nnz_tok", ctypes.c_int64),
                 ("sum_nnz_doc", ctypes.c_int64), ("n_launches", ctypes.c_int64),
                 ("n_sample_chunks", ctypes.c_int64), ("n_exact_redraws", ctypes.c_int64),
-                ("ms_table", ctypes.c_double)]
+                ("ms_table", ctypes.c_double), ("ms_allreduce_exposed", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

@@ -594,6 +594,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     st.last_n = n;
     st.sweeps_done = static_cast<int64_t>(ctx->sweeps);
     st.ms_total = st.ms_sample = st.ms_recount = st.ms_theta = st.ms_allreduce = st.ms_table = 0;
+    st.ms_allreduce_exposed = 0;
     st.ms_last_sweep = st.ms_last_sample = 0;
     ctx->log_ms.assign(n, 0);
     ctx->log_ms_sample.assign(n, 0);
@@ -612,7 +613,13 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventElapsedTime(&b, E[1], E[2]));
         CU(cudaEventElapsedTime(&c, E[2], E[3]));
         CU(cudaEventElapsedTime(&tot, E[0], E[5]));
-        if (ctx->world > 1) CU(cudaEventElapsedTime(&d, E[2], E[4]));
+        float x = 0;
+        if (ctx->world > 1) {
+            CU(cudaEventElapsedTime(&d, E[2], E[4]));
+            // exposed: the compute stream's wait for the allreduce after the θ rebuild
+            CU(cudaEventElapsedTime(&x, E[3], E[5]));
+        }
+        st.ms_allreduce_exposed += x;
         st.ms_sample += a;
         st.ms_recount += b;
         st.ms_theta += c;
