@@ -1496,7 +1496,6 @@ template <int R>
 __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
     extern __shared__ double smem_dd[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int q = lane >> 2, sub = lane & 3;
     const int K = a.K;
     const int K4 = (K + 3) & ~3;
     const int NC = (K + 127) / 128;
