@@ -34,6 +34,7 @@ struct lda_ctx {
     int sampler = -1;  // auto
     int64_t tail_per_tile = 64;
     int64_t certify_slack = 1;
+    int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int threads = 0;
     // distribution
     int32_t rank = 0, world = 1;
@@ -252,6 +253,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "tail_per_tile") {
         if (value < 0 || value > (int64_t(1) << 30)) return fail(ctx, LDA_EINVAL, "tail_per_tile out of range");
         ctx->tail_per_tile = value;
+    } else if (k == "fused_recount") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "fused_recount must be 0 or 1");
+        ctx->fused_recount = static_cast<int>(value);
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
@@ -379,6 +383,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.filter32 = ctx->filter32;
     S.sampler = ctx->sampler;
     S.certify_slack = static_cast<double>(ctx->certify_slack);
+    S.tile_fused = ctx->fused_recount != 0;
     KL(lda::configure_kernels(S));
 
     lda::HostLayout &H = ctx->H;

@@ -967,6 +967,7 @@ struct TileArgs {
     const char *wtab;          // word tables (word_table_kernel), wt_bytes per word
     uint32_t wt_bytes;
     int nbuf;                  // sweep_tile_cta_kernel: table buffers per CTA
+    int recount;               // 1: the ϕ update fused here; 0: recount_kernel after the sweep
     uint32_t t;
     uint32_t key0[10], key1[10];
 };
@@ -1481,6 +1482,8 @@ __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool f
     // ---- z and the fused recount
     if (take) {
         a.z[p] = static_cast<uint16_t>(z);
+    }
+    if (take && a.recount) {
         const unsigned act = __activemask();
         const unsigned peers = __match_any_sync(act, z);
         if (lane == __ffs(peers) - 1) {
@@ -1633,8 +1636,9 @@ __global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
         }
     }
     __syncthreads();
-    for (int k = threadIdx.x; k < K; k += blockDim.x)
-        if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
+    if (a.recount)
+        for (int k = threadIdx.x; k < K; k += blockDim.x)
+            if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
     if (a.n_exact && lane == 0 && n_exact) atomicAdd(a.n_exact, static_cast<unsigned long long>(n_exact));
 }
 
@@ -1774,8 +1778,9 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     }
     if (!GNK) {
         __syncthreads();
-        for (int k = threadIdx.x; k < K; k += blockDim.x)
-            if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
+        if (a.recount)
+            for (int k = threadIdx.x; k < K; k += blockDim.x)
+                if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
     }
     if (a.n_exact && lane == 0 && n_exact) atomicAdd(a.n_exact, static_cast<unsigned long long>(n_exact));
 }
@@ -1791,6 +1796,12 @@ __global__ void zero_rows_kernel(const int32_t *__restrict__ words, int64_t n, i
     }
 }
 
+// Segmented recount (the ϕ update as a separate pass, L1273-1285): per work
+// item (a word's virtual token range, <= recount_tokens) a CTA builds the
+// topic histogram in shared memory, the warps taking the word's runs in turn
+// (each run contiguous in the word-major stream: coalesced z reads, no
+// per-token search), then writes the word's row of n_wk (global atomics only
+// for words split over several items) and accumulates n_k.
 __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc,
                                const Seg *__restrict__ segs, int K, const uint16_t *__restrict__ z,
                                int32_t *__restrict__ nwk, int32_t *__restrict__ nk,
@@ -1798,6 +1809,7 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
     extern __shared__ int smem_i[];
     int *hist = smem_i, *nkp = smem_i + K;
     __shared__ int s_ci;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
     for (int k = threadIdx.x; k < 2 * K; k += blockDim.x) smem_i[k] = 0;
     __syncthreads();
     for (;;) {
@@ -1808,8 +1820,15 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
         const RecountChunk c = rc[ci];
         const uint32_t w = c.word & 0x7FFFFFFFu;
         const bool split = (c.word >> 31) != 0u;
-        for (uint32_t j = threadIdx.x; j < c.vcount; j += blockDim.x)
-            atomicAdd(&hist[z[run_position(segs, c.seg0, c.segN, c.vbegin + j)]], 1);
+        const uint32_t vb = c.vbegin, ve = c.vbegin + c.vcount;
+        // runs s = seg0 + warp, seg0 + warp + nwarps, ... while they start before ve
+        for (uint32_t si = c.seg0 + warp; si < c.segN; si += nwarps) {
+            const Seg sg = segs[si];
+            if (sg.vstart >= ve) break;
+            const uint32_t rv0 = max(sg.vstart, vb), rv1 = min(segs[si + 1].vstart, ve);
+            const uint32_t p0 = sg.pos + (rv0 - sg.vstart);
+            for (uint32_t v = rv0 + lane; v < rv1; v += 32) atomicAdd(&hist[z[p0 + (v - rv0)]], 1);
+        }
         __syncthreads();
         int32_t *row = nwk + static_cast<size_t>(w) * K;
         for (int k = threadIdx.x; k < K; k += blockDim.x) {
@@ -2124,7 +2143,7 @@ int configure_kernels(DevState &s) {
                 cudaSuccess)
                 return e;
             s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
-            s.sweep_fused = true;
+            s.sweep_fused = s.tile_fused;
         }
         s.wt_bytes = s.sweep_tile_cta && s.tile_cta_gnk ? tab_bytes_compact(s.K) : tab_bytes(s.K);
         if (s.sweep_tile || s.sweep_tile_cta)
@@ -2147,7 +2166,7 @@ int configure_kernels(DevState &s) {
                 cudaSuccess)
                 return e;
             s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
-            s.sweep_fused = true;
+            s.sweep_fused = s.tile_fused;
         }
     }
     // recount
@@ -2268,8 +2287,9 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
     }
     if (s.sweep_tile || s.sweep_tile_cta) {
         // every row of the next n_wk is accumulated (words span tiles)
-        if ((e = cudaMemsetAsync(s.nwk_alt, 0, sizeof(int32_t) * (static_cast<size_t>(s.V) * s.K + s.K), st)) !=
-            cudaSuccess)
+        if (s.tile_fused &&
+            (e = cudaMemsetAsync(s.nwk_alt, 0, sizeof(int32_t) * (static_cast<size_t>(s.V) * s.K + s.K), st)) !=
+                cudaSuccess)
             return e;
         const int wtb = static_cast<int>(std::min<int64_t>((static_cast<int64_t>(s.V) + 7) / 8, 8 * s.num_sms));
         const bool compact = s.sweep_tile_cta && s.tile_cta_gnk;
@@ -2309,6 +2329,7 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.wtab = s.wtab;
         ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
         ta.nbuf = s.tile_nbuf;
+        ta.recount = s.tile_fused ? 1 : 0;
         ta.t = t;
         uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
         for (int r = 0; r < 10; ++r) {

@@ -197,6 +197,7 @@ struct DevState {
     bool sweep_tile_cta = false;    // its large-K form with CTA-shared tables (sampler 3)
     bool tile_cta_gnk = false;      // ... with n_k by global reductions and compact tables (K > kTileMaxK)
     int tile_nbuf = 2;              // ... its table buffers per CTA
+    bool tile_fused = true;         // option fused_recount: the tile samplers update n_wk / n_k themselves
     size_t tile_smem = 0;
     int tile_grid = 0, tile_block = 0, tile_lmax = 160;
     char *wtab = nullptr;           // tile sampler: per-word tables (p32, dense prefix), rebuilt every sweep

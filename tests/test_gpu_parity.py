@@ -175,6 +175,8 @@ def test_tile_sampler_decomposition_and_fallback_rate():
                      chunk_tokens=77)
     gc = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=300_000,
                      sampler=3)     # CTA-shared tables: same arithmetic, other batches
+    gd = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, tile_tokens=100_000,
+                     fused_recount=0)   # n_wk / n_k by the segmented recount kernel instead
     g0 = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, sampler=0)
     n_exact = 0
     for _ in range(6):
@@ -182,10 +184,13 @@ def test_tile_sampler_decomposition_and_fallback_rate():
         n_exact += ga.stats()["n_exact_redraws"]
         gb.iterate(1)
         gc.iterate(1)
+        gd.iterate(1)
         g0.iterate(1)
         za = ga.z()
         assert np.array_equal(za, gb.z())
         assert np.array_equal(za, gc.z())
+        assert np.array_equal(za, gd.z())
+        assert np.array_equal(ga.nwk(), gd.nwk()) and np.array_equal(ga.nk(), gd.nk())
         diff = np.count_nonzero(za != g0.z())
         assert diff <= 1e-6 * cfg.T + 2
         if diff:                       # keep the chains in lock step
