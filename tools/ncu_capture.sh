@@ -13,7 +13,7 @@ ncu --metrics gpu__time_duration.sum --clock-control none -k "$KRE" --csv \
     --log-file $OUT/launches_${TAG}_${CFG}.csv \
     python bench.py --config $CFG --steps 2 --warmup 3 --no-cpu-baseline > $OUT/launches_${TAG}_${CFG}.bench.log 2>&1
 ncu --set full --clock-control none --import-source on \
-    -k 'regex:^(sweep_tile_kernel|word_table_kernel|theta_kernel|gather_z_kernel|zero_rows_kernel|prologue_kernel)' -s 12 -c 5 \
+    -k 'regex:^(sweep_tile_kernel|word_table_kernel|recount_kernel|theta_kernel|gather_z_kernel|prologue_kernel)' -s 12 -c 6 \
     -o $OUT/prof_${TAG}_${CFG} -f \
     python bench.py --config $CFG --steps 1 --warmup 3 --no-cpu-baseline > $OUT/prof_${TAG}_${CFG}.log 2>&1
 ls -la $OUT
