@@ -1694,7 +1694,12 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     const double gS = 9.5 * 5.9604644775390625e-08 * a.slack;
 
     // buffer b <- the CTA's next work item (its table by bulk copy); the end
-    // of the queue is an item with n = 0
+    // of the queue is an item with n = 0.  items[b] / slot[b] / left[b] are
+    // published to the other warps by the buffer's mbarrier: the arrive below
+    // has release semantics and their try_wait acquire semantics (CTA scope);
+    // compute-sanitizer's racecheck does not model mbarrier ordering and
+    // reports this handoff as a hazard (memcheck is clean).  The loader runs
+    // only after every warp has left the buffer (left[b] reached 0).
     auto load = [&](int b) {
         const uint32_t ci = atomicAdd(a.counter, 1u);
         TileItem it = {0u, 0u, 0u, 0u};
