@@ -269,10 +269,15 @@ class LDA:
     def loglik(self):
         return lda_loglik(self.ctx)
 
-    def z(self):
-        z = np.empty(self.T, np.uint16)
-        lda_get_counts(self.ctx, z=z)
-        return z
+    def z(self, out=None):
+        """z in document order; `out` (uint16[T], e.g. a pinned buffer) is
+        filled in place when given."""
+        if out is None:
+            out = np.empty(self.T, np.uint16)
+        elif out.dtype != np.uint16 or out.shape != (self.T,) or not out.flags.c_contiguous:
+            raise ValueError("out must be a contiguous uint16 array of T entries")
+        lda_get_counts(self.ctx, z=out)
+        return out
 
     def set_z(self, z):
         lda_set_z(self.ctx, z)

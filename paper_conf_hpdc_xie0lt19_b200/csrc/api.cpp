@@ -389,11 +389,35 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     lda::HostLayout &H = ctx->H;
     // the per-token tables go to the device tile by tile, copied by a helper
     // thread while the host prepares the next tile
-    DA(S.tok_row, Tg);
-    DA(S.doc_map, Tg);
     const bool tile_layout = S.sweep_tile || S.sweep_tile_cta;
-    if (!tile_layout) DA(S.tok_crank, Tg);  // the tile samplers take ranks from their items
     lda::tmark("histogram, streams, configure");
+    // the large device buffers that do not depend on the layout are
+    // allocated by a helper thread while the host builds it (cudaMalloc of
+    // several GB takes ~0.3-0.5 s, all of it otherwise on the load path)
+    std::vector<std::pair<void **, size_t>> pre;
+    pre.push_back({reinterpret_cast<void **>(&S.tok_z), sizeof(uint16_t) * Tg});
+    if (ctx->theta_mode == 1) pre.push_back({reinterpret_cast<void **>(&S.z_doc), sizeof(uint16_t) * (Tg + 4)});
+    const size_t nwk_bytes = sizeof(int32_t) * (static_cast<size_t>(V) * K + K);
+    pre.push_back({reinterpret_cast<void **>(&S.nwk), nwk_bytes});
+    if (S.sweep_fused) pre.push_back({reinterpret_cast<void **>(&S.nwk_alt), nwk_bytes});
+    if (tile_layout) pre.push_back({reinterpret_cast<void **>(&S.wtab), S.wt_bytes * static_cast<size_t>(V)});
+    std::vector<void *> pre_done;
+    cudaError_t pre_err = cudaSuccess;
+    size_t pre_fail_bytes = 0;
+    std::thread pre_alloc([&] {
+        pre_err = cudaSetDevice(ctx->device);
+        for (auto &pa : pre) {
+            if (pre_err != cudaSuccess) break;
+            void *q = nullptr;
+            pre_err = cudaMalloc(&q, std::max<size_t>(pa.second, 1));
+            if (pre_err != cudaSuccess) {
+                pre_fail_bytes = pa.second;
+                break;
+            }
+            *pa.first = q;
+            pre_done.push_back(q);
+        }
+    });
     struct Job {
         uint64_t p0, p1, t0, t1;
     };
@@ -402,10 +426,21 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     std::condition_variable cv;
     bool jobs_done = false;
     cudaError_t copy_err = cudaSuccess;
+    std::vector<void *> tok_done;  // the copier's own buffers (allocated before its first copy)
     std::thread copier([&] {
         cudaSetDevice(ctx->device);
         cudaStream_t cs = nullptr;
         cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+        // the per-token tables' device buffers (the tile samplers take ranks from their items)
+        for (uint32_t **b : {&S.tok_row, &S.doc_map, tile_layout ? nullptr : &S.tok_crank}) {
+            if (!b || copy_err != cudaSuccess) continue;
+            void *q = nullptr;
+            copy_err = cudaMalloc(&q, std::max<size_t>(sizeof(uint32_t) * Tg, 1));
+            if (copy_err == cudaSuccess) {
+                *b = static_cast<uint32_t *>(q);
+                tok_done.push_back(q);
+            }
+        }
         for (;;) {
             Job j;
             {
@@ -415,6 +450,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                 j = jobs.front();
                 jobs.erase(jobs.begin());
             }
+            if (copy_err != cudaSuccess) continue;  // drain the queue
             cudaError_t r = cudaSuccess;
             const size_t np = (j.p1 - j.p0) * sizeof(uint32_t), nt = (j.t1 - j.t0) * sizeof(uint32_t);
             if (np && r == cudaSuccess)
@@ -450,8 +486,20 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     }
     cv.notify_one();
     copier.join();
+    pre_alloc.join();
+    ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
+    ctx->allocs.insert(ctx->allocs.end(), tok_done.begin(), tok_done.end());
+    if (pre_err != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ctx, pre_err == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
+                    std::string("cudaMalloc(") + std::to_string(pre_fail_bytes) + " B): " + cudaGetErrorString(pre_err));
+    }
     if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
-    if (copy_err != cudaSuccess) return fail(ctx, LDA_ECUDA, std::string("token table copy: ") + cudaGetErrorString(copy_err));
+    if (copy_err != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ctx, copy_err == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
+                    std::string("token tables (allocation or copy): ") + cudaGetErrorString(copy_err));
+    }
     lda::tmark("layout done, token tables on the device");
 
     S.V = V;
@@ -463,8 +511,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.beta = ctx->beta;
     S.seed = seed;
 
-    DA(S.tok_z, Tg);
-    if (ctx->theta_mode == 1) DA(S.z_doc, Tg + 4);
     DA(S.doc_ptr32, Dg + 1);
     DA(S.row_off32, std::max<int64_t>(Dg, 1));
     DA(S.segs, H.segs.size());
@@ -483,11 +529,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     if (S.sweep_tile || S.sweep_tile_cta) {
         DA(S.titems, H.titems.size());
         DA(S.cbase, V);
-        DA(S.wtab, S.wt_bytes * static_cast<size_t>(V));
     }
     DA(S.rows, H.rows32 * 8);
-    DA(S.nwk, static_cast<size_t>(V) * K + K);
-    if (S.sweep_fused) DA(S.nwk_alt, static_cast<size_t>(V) * K + K);
     S.n_zero_words = static_cast<int64_t>(H.zero_words.size());
     DA(S.zero_words, H.zero_words.size());
     DA(S.denom, K);

@@ -267,29 +267,47 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         });
         // bases: word-major positions (head words: this tile's segment; tail
         // words: their tail run) and canonical ranks, part by part
+        // (in parallel over word ranges: the tile's tokens of each word, the
+        // head words' segment starts by a serial prefix over the words, then
+        // every word's run start per part)
         auto &tc = tile_cnt[b];
         tc.assign(V, 0);
-        for (int32_t w = 0; w < V; ++w) {
-            uint32_t run_p = tail[w] ? tail_next[w] : static_cast<uint32_t>(pos);
-            uint32_t run_c = crank_run[w];
-            tcrank[static_cast<size_t>(b) * V + w] = run_c;
-            if (!tail[w]) tseg[static_cast<size_t>(b) * V + w] = static_cast<uint32_t>(pos);
-            for (int t = 0; t < nth; ++t) {
-                const uint32_t h = cnt[t][w];
-                pnext[t][w] = run_p;
-                cnext[t][w] = run_c;
-                run_p += h;
-                run_c += h;
-            }
-            const uint32_t n = run_c - crank_run[w];
-            crank_run[w] = run_c;
-            if (tail[w]) {
-                tail_next[w] = run_p;
-            } else {
+        auto word_parts = [&](auto &&f) {
+            run_parts([&](int t) {
+                f(static_cast<int32_t>(static_cast<int64_t>(V) * t / nth),
+                  static_cast<int32_t>(static_cast<int64_t>(V) * (t + 1) / nth));
+            });
+        };
+        uint32_t *tseg_b = tseg.data() + static_cast<size_t>(b) * V;
+        word_parts([&](int32_t w0, int32_t w1) {
+            for (int32_t w = w0; w < w1; ++w) {
+                if (tail[w]) continue;
+                uint32_t n = 0;
+                for (int t = 0; t < nth; ++t) n += cnt[t][w];
                 tc[w] = n;
-                pos += n;
             }
-        }
+        });
+        for (int32_t w = 0; w < V; ++w)
+            if (!tail[w]) {
+                tseg_b[w] = static_cast<uint32_t>(pos);
+                pos += tc[w];
+            }
+        word_parts([&](int32_t w0, int32_t w1) {
+            for (int32_t w = w0; w < w1; ++w) {
+                uint32_t run_p = tail[w] ? tail_next[w] : tseg_b[w];
+                uint32_t run_c = crank_run[w];
+                tcrank[static_cast<size_t>(b) * V + w] = run_c;
+                for (int t = 0; t < nth; ++t) {
+                    const uint32_t h = cnt[t][w];
+                    pnext[t][w] = run_p;
+                    cnext[t][w] = run_c;
+                    run_p += h;
+                    run_c += h;
+                }
+                crank_run[w] = run_c;
+                if (tail[w]) tail_next[w] = run_p;
+            }
+        });
         // scatter: canonical ranks in document order, then positions with the
         // part's documents by decreasing length, so that the 32 tokens a warp
         // draws together (consecutive in a word's run) come from documents of

@@ -942,6 +942,12 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kerne
 #ifndef LDA_TILE_WPC
 #define LDA_TILE_WPC 8
 #endif
+#ifndef LDA_TILE_LMAX
+#define LDA_TILE_LMAX 160
+#endif
+#ifndef LDA_TILE_MINB
+#define LDA_TILE_MINB 2
+#endif
 #ifndef LDA_TILE_MAXK
 #define LDA_TILE_MAXK 4096
 #endif
@@ -1496,7 +1502,7 @@ __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool f
 }
 
 template <int R>
-__global__ void __launch_bounds__(256, 2) sweep_tile_kernel(TileArgs a) {
+__global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_kernel(TileArgs a) {
     extern __shared__ double smem_dd[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int K = a.K;
@@ -2103,7 +2109,7 @@ int configure_kernels(DevState &s) {
     // table and the batch scratch; <= 8 warps per CTA
     {
         const size_t K4 = static_cast<size_t>((s.K + 3) & ~3);
-        s.tile_lmax = std::max(160, ((s.K + 1 + 31) / 32 + 3) & ~3);
+        s.tile_lmax = std::max(LDA_TILE_LMAX, ((s.K + 1 + 31) / 32 + 3) & ~3);
         const size_t cta = 4 * K4, per_warp = tile_warp_bytes(s.K, s.tile_lmax);
         int wpc = 0;
         while (wpc < LDA_TILE_WPC && cta + per_warp * (wpc + 1) + 1024 <= static_cast<size_t>(max_optin)) ++wpc;

@@ -148,6 +148,17 @@ def test_layout_invariants(sampler, tile_tokens, chunk_tokens, tail):
     assert st["items"] > 0 and st["runs"] > 0
 
 
+@pytest.mark.parametrize("sampler", [0, 2])
+def test_layout_invariants_multithreaded_tiles(sampler):
+    """Tiles of >= 2^16 tokens are split over the host threads (per-part
+    counts, per-word bases computed in parallel over word ranges): the same
+    invariants as above."""
+    doc_ptr, words = _corpus(5000, 3000, 9, max_len=80)
+    st = L.lda_layout_selfcheck(doc_ptr, words, 3000, 24, sampler=sampler, tile_tokens=90_000,
+                                chunk_tokens=512, tail_per_tile=8)
+    assert st["tiles"] >= 3 and st["items"] > 0 and st["runs"] > 0
+
+
 def test_layout_selfcheck_rejects_bad_input():
     doc_ptr, words = _corpus(10, 20, 1)
     bad = words.copy()
