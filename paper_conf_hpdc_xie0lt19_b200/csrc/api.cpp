@@ -391,10 +391,13 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // thread while the host prepares the next tile
     const bool tile_layout = S.sweep_tile || S.sweep_tile_cta;
     lda::tmark("histogram, streams, configure");
-    // the large device buffers that do not depend on the layout are
-    // allocated by a helper thread while the host builds it (cudaMalloc of
-    // several GB takes ~0.3-0.5 s, all of it otherwise on the load path)
+    // The device buffers are allocated by the copier thread below while the
+    // host builds the layout (cudaMalloc of ~10 GB takes ~0.3-0.5 s, all of
+    // it otherwise on the load path): first the per-token tables it copies
+    // into, then the large buffers that do not depend on the layout.
     std::vector<std::pair<void **, size_t>> pre;
+    for (uint32_t **t : {&S.tok_row, &S.doc_map, tile_layout ? nullptr : &S.tok_crank})
+        if (t) pre.push_back({reinterpret_cast<void **>(t), sizeof(uint32_t) * Tg});
     pre.push_back({reinterpret_cast<void **>(&S.tok_z), sizeof(uint16_t) * Tg});
     if (ctx->theta_mode == 1) pre.push_back({reinterpret_cast<void **>(&S.z_doc), sizeof(uint16_t) * (Tg + 4)});
     const size_t nwk_bytes = sizeof(int32_t) * (static_cast<size_t>(V) * K + K);
@@ -402,22 +405,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     if (S.sweep_fused) pre.push_back({reinterpret_cast<void **>(&S.nwk_alt), nwk_bytes});
     if (tile_layout) pre.push_back({reinterpret_cast<void **>(&S.wtab), S.wt_bytes * static_cast<size_t>(V)});
     std::vector<void *> pre_done;
-    cudaError_t pre_err = cudaSuccess;
     size_t pre_fail_bytes = 0;
-    std::thread pre_alloc([&] {
-        pre_err = cudaSetDevice(ctx->device);
-        for (auto &pa : pre) {
-            if (pre_err != cudaSuccess) break;
-            void *q = nullptr;
-            pre_err = cudaMalloc(&q, std::max<size_t>(pa.second, 1));
-            if (pre_err != cudaSuccess) {
-                pre_fail_bytes = pa.second;
-                break;
-            }
-            *pa.first = q;
-            pre_done.push_back(q);
-        }
-    });
     struct Job {
         uint64_t p0, p1, t0, t1;
     };
@@ -426,20 +414,20 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     std::condition_variable cv;
     bool jobs_done = false;
     cudaError_t copy_err = cudaSuccess;
-    std::vector<void *> tok_done;  // the copier's own buffers (allocated before its first copy)
     std::thread copier([&] {
         cudaSetDevice(ctx->device);
         cudaStream_t cs = nullptr;
         cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
-        // the per-token tables' device buffers (the tile samplers take ranks from their items)
-        for (uint32_t **b : {&S.tok_row, &S.doc_map, tile_layout ? nullptr : &S.tok_crank}) {
-            if (!b || copy_err != cudaSuccess) continue;
+        for (auto &pa : pre) {
+            if (copy_err != cudaSuccess) break;
             void *q = nullptr;
-            copy_err = cudaMalloc(&q, std::max<size_t>(sizeof(uint32_t) * Tg, 1));
-            if (copy_err == cudaSuccess) {
-                *b = static_cast<uint32_t *>(q);
-                tok_done.push_back(q);
+            copy_err = cudaMalloc(&q, std::max<size_t>(pa.second, 1));
+            if (copy_err != cudaSuccess) {
+                pre_fail_bytes = pa.second;
+                break;
             }
+            *pa.first = q;
+            pre_done.push_back(q);
         }
         for (;;) {
             Job j;
@@ -479,27 +467,22 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
                                       tile_layout ? 2 : (S.sweep_quad ? 1 : 0),
                                       ctx->tail_per_tile * kscale, H,
-                                      on_final);
+                                      on_final, local.data());
     {
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
     }
     cv.notify_one();
     copier.join();
-    pre_alloc.join();
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
-    ctx->allocs.insert(ctx->allocs.end(), tok_done.begin(), tok_done.end());
-    if (pre_err != cudaSuccess) {
-        cudaGetLastError();
-        return fail(ctx, pre_err == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
-                    std::string("cudaMalloc(") + std::to_string(pre_fail_bytes) + " B): " + cudaGetErrorString(pre_err));
-    }
-    if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
     if (copy_err != cudaSuccess) {
         cudaGetLastError();
         return fail(ctx, copy_err == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
-                    std::string("token tables (allocation or copy): ") + cudaGetErrorString(copy_err));
+                    pre_fail_bytes ? std::string("cudaMalloc(") + std::to_string(pre_fail_bytes) +
+                                         " B): " + cudaGetErrorString(copy_err)
+                                   : std::string("token table copy: ") + cudaGetErrorString(copy_err));
     }
+    if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
     lda::tmark("layout done, token tables on the device");
 
     S.V = V;

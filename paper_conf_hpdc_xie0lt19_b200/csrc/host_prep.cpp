@@ -131,7 +131,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &L,
-                         const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final) {
+                         const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final,
+                         const int64_t *word_counts) {
     const bool build_pairs = sampler == 1;
     const int64_t T = doc_ptr[D];
     L.D = D;
@@ -179,7 +180,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 
     // Word counts of the shard (parallel histogram).
     std::vector<int64_t> wc(V, 0);
-    word_histogram(words, T, V, nthreads, wc.data());
+    if (word_counts) std::copy(word_counts, word_counts + V, wc.begin());
+    else word_histogram(words, T, V, nthreads, wc.data());
     L.word_count = wc;
 
     // Tail words (tile sampler only): words with too few tokens per document
@@ -206,13 +208,16 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         return "host allocation of the token tables failed";
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
     if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";
-    // first touch in parallel (every entry is written below)
+    // first touch in parallel, one store per 4 KB page (the kernel zeroes
+    // the pages; every entry is written below)
     parallel_for(nthreads, T, [&](int, int64_t b, int64_t e) {
-        std::fill(L.tok_row.data() + b, L.tok_row.data() + e, 0u);
-        std::fill(L.doc_map.data() + b, L.doc_map.data() + e, 0u);
-        if (!tile_layout) {
-            std::fill(L.tok_crank.data() + b, L.tok_crank.data() + e, 0u);
-            std::fill(ctmp.data() + b, ctmp.data() + e, 0u);
+        for (int64_t i = b; i < e; i += 1024) {
+            L.tok_row[i] = 0u;
+            L.doc_map[i] = 0u;
+            if (!tile_layout) {
+                L.tok_crank[i] = 0u;
+                ctmp[i] = 0u;
+            }
         }
     });
     tmark("layout: host tables");
@@ -238,6 +243,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     std::vector<uint32_t> tcrank(static_cast<size_t>(nt) * V, 0);  // rank of a (tile, word) run's first token
     std::vector<std::vector<uint32_t>> cnt(nthreads, std::vector<uint32_t>(V));
     std::vector<std::vector<uint32_t>> pnext(nthreads, std::vector<uint32_t>(V));
+    std::vector<std::vector<uint64_t>> roff(nthreads), rbuf(nthreads);  // tile layout: region buckets
     std::vector<std::vector<uint32_t>> cnext(nthreads, std::vector<uint32_t>(V));
 
     uint64_t pos = 0;  // start of the current tile's segment
@@ -317,13 +323,44 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         run_parts([&](int t) {
             auto &next = pnext[t];
             if (tile_layout) {
+                // Two passes instead of one scatter of 4-byte rows over the
+                // whole tile segment (a cache-line miss per token): (A) the
+                // positions in document order (doc_map, sequential) with
+                // (position, row) pairs appended to per-region buckets of
+                // 2^kRegion positions; (B) the buckets region by region
+                // (the rows of one region stay in cache).  Tail words'
+                // tokens are written directly.
+                constexpr int kRegion = 15;
+                const uint64_t nreg = ((pos - pos_tile) >> kRegion) + 1;
+                auto &off = roff[t];
+                off.assign(nreg + 1, 0);
+                for (int32_t w = 0; w < V; ++w) {  // bucket sizes from the runs
+                    const uint32_t c = cnt[t][w];
+                    if (c == 0 || tail[w]) continue;
+                    const uint64_t a = next[w] - pos_tile, e = a + c;
+                    for (uint64_t r = a >> kRegion; r <= (e - 1) >> kRegion; ++r)
+                        off[r + 1] += std::min(e, (r + 1) << kRegion) - std::max(a, r << kRegion);
+                }
+                for (uint64_t r = 0; r < nreg; ++r) off[r + 1] += off[r];
+                auto &buf = rbuf[t];
+                if (buf.size() < off[nreg]) buf.resize(off[nreg]);
                 for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
                     const uint32_t row = L.row_off32[d];
                     for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
-                        const uint32_t p = next[words[i]]++;
+                        const int32_t w = words[i];
+                        const uint32_t p = next[w]++;
                         L.doc_map[i] = p;
-                        L.tok_row[p] = row;
+                        if (tail[w]) {
+                            L.tok_row[p] = row;
+                        } else {
+                            const uint64_t r = (p - pos_tile) >> kRegion;
+                            buf[off[r]++] = (static_cast<uint64_t>(p) << 32) | row;
+                        }
                     }
+                }
+                for (uint64_t j = 0, n = off[nreg]; j < n; ++j) {  // buf: region by region
+                    const uint64_t x = buf[j];
+                    L.tok_row[x >> 32] = static_cast<uint32_t>(x);
                 }
                 return;
             }

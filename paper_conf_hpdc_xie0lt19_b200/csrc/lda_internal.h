@@ -134,7 +134,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &out,
-                         const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {});
+                         const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {},
+                         const int64_t *word_counts = nullptr);  // V local tokens per word, if known
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
