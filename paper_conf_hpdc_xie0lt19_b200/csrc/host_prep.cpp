@@ -2,6 +2,7 @@
 // validation, the word-first token order (L1189-1191), the document-word map
 // (L1297-1303), fixed-capacity θ rows (CSR with short column index,
 // L1235-1243) and the heavy-first work-item tables (L1203-1221).
+#include <atomic>
 #include <sys/mman.h>
 
 #include <algorithm>
@@ -243,7 +244,6 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     std::vector<uint32_t> tcrank(static_cast<size_t>(nt) * V, 0);  // rank of a (tile, word) run's first token
     std::vector<std::vector<uint32_t>> cnt(nthreads, std::vector<uint32_t>(V));
     std::vector<std::vector<uint32_t>> pnext(nthreads, std::vector<uint32_t>(V));
-    std::vector<std::vector<uint64_t>> roff(nthreads), rbuf(nthreads);  // tile layout: region buckets
     std::vector<std::vector<uint32_t>> cnext(nthreads, std::vector<uint32_t>(V));
 
     uint64_t pos = 0;  // start of the current tile's segment
@@ -323,44 +323,13 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         run_parts([&](int t) {
             auto &next = pnext[t];
             if (tile_layout) {
-                // Two passes instead of one scatter of 4-byte rows over the
-                // whole tile segment (a cache-line miss per token): (A) the
-                // positions in document order (doc_map, sequential) with
-                // (position, row) pairs appended to per-region buckets of
-                // 2^kRegion positions; (B) the buckets region by region
-                // (the rows of one region stay in cache).  Tail words'
-                // tokens are written directly.
-                constexpr int kRegion = 15;
-                const uint64_t nreg = ((pos - pos_tile) >> kRegion) + 1;
-                auto &off = roff[t];
-                off.assign(nreg + 1, 0);
-                for (int32_t w = 0; w < V; ++w) {  // bucket sizes from the runs
-                    const uint32_t c = cnt[t][w];
-                    if (c == 0 || tail[w]) continue;
-                    const uint64_t a = next[w] - pos_tile, e = a + c;
-                    for (uint64_t r = a >> kRegion; r <= (e - 1) >> kRegion; ++r)
-                        off[r + 1] += std::min(e, (r + 1) << kRegion) - std::max(a, r << kRegion);
-                }
-                for (uint64_t r = 0; r < nreg; ++r) off[r + 1] += off[r];
-                auto &buf = rbuf[t];
-                if (buf.size() < off[nreg]) buf.resize(off[nreg]);
                 for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
                     const uint32_t row = L.row_off32[d];
                     for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
-                        const int32_t w = words[i];
-                        const uint32_t p = next[w]++;
+                        const uint32_t p = next[words[i]]++;
                         L.doc_map[i] = p;
-                        if (tail[w]) {
-                            L.tok_row[p] = row;
-                        } else {
-                            const uint64_t r = (p - pos_tile) >> kRegion;
-                            buf[off[r]++] = (static_cast<uint64_t>(p) << 32) | row;
-                        }
+                        L.tok_row[p] = row;
                     }
-                }
-                for (uint64_t j = 0, n = off[nreg]; j < n; ++j) {  // buf: region by region
-                    const uint64_t x = buf[j];
-                    L.tok_row[x >> 32] = static_cast<uint32_t>(x);
                 }
                 return;
             }
@@ -393,24 +362,38 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // chunk_tokens, tile by tile, heavy-first inside each tile.
     L.titems.clear();
     if (sampler == 2) {
-        for (int b = 0; b < nt; ++b) {
-            const size_t first = L.titems.size();
-            for (int32_t w = 0; w < V; ++w) {
-                const int64_t n = tile_cnt[b][w];
-                if (n == 0) continue;
-                const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
-                const uint32_t pos = tseg[static_cast<size_t>(b) * V + w];
-                for (int64_t q = 0; q < pieces; ++q) {
-                    const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
-                    L.titems.push_back(TileItem{static_cast<uint32_t>(w), pos + static_cast<uint32_t>(vb),
-                                                static_cast<uint32_t>(ve - vb),
-                                                tcrank[static_cast<size_t>(b) * V + w] + static_cast<uint32_t>(vb)});
+        // tiles in parallel (threads take tiles in turn), then concatenated in tile order
+        std::vector<std::vector<TileItem>> per(nt);
+        std::atomic<int> next_tile{0};
+        auto make = [&] {
+            for (int b; (b = next_tile.fetch_add(1)) < nt;) {
+                auto &it = per[b];
+                for (int32_t w = 0; w < V; ++w) {
+                    const int64_t n = tile_cnt[b][w];
+                    if (n == 0) continue;
+                    const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
+                    const uint32_t pos = tseg[static_cast<size_t>(b) * V + w];
+                    for (int64_t q = 0; q < pieces; ++q) {
+                        const int64_t vb = n * q / pieces, ve = n * (q + 1) / pieces;
+                        it.push_back(TileItem{static_cast<uint32_t>(w), pos + static_cast<uint32_t>(vb),
+                                              static_cast<uint32_t>(ve - vb),
+                                              tcrank[static_cast<size_t>(b) * V + w] + static_cast<uint32_t>(vb)});
+                    }
                 }
+                std::stable_sort(it.begin(), it.end(), [](const TileItem &x, const TileItem &y) { return x.n > y.n; });
             }
-            std::stable_sort(L.titems.begin() + first, L.titems.end(),
-                             [](const TileItem &x, const TileItem &y) { return x.n > y.n; });
+        };
+        {
+            std::vector<std::thread> th;
+            for (int t = 1; t < std::min(nthreads, nt); ++t) th.emplace_back(make);
+            make();
+            for (auto &x : th) x.join();
         }
-        if (L.titems.size() >= (uint64_t(1) << 32) - 1) return "too many tile sampler items";
+        size_t total = 0;
+        for (auto &it : per) total += it.size();
+        if (total >= (uint64_t(1) << 32) - 1) return "too many tile sampler items";
+        L.titems.reserve(total);
+        for (auto &it : per) L.titems.insert(L.titems.end(), it.begin(), it.end());
     }
 
     tmark("layout: tile items");
