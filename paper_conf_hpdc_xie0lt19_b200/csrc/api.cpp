@@ -441,7 +441,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             if (copy_err != cudaSuccess) continue;  // drain the queue
             cudaError_t r = cudaSuccess;
             const size_t np = (j.p1 - j.p0) * sizeof(uint32_t), nt = (j.t1 - j.t0) * sizeof(uint32_t);
-            if (np && r == cudaSuccess)
+            if (np && r == cudaSuccess && H.tok_row.data())
                 r = cudaMemcpyAsync(S.tok_row + j.p0, H.tok_row.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
             if (np && r == cudaSuccess && S.tok_crank)
                 r = cudaMemcpyAsync(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
@@ -467,7 +467,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
                                       tile_layout ? 2 : (S.sweep_quad ? 1 : 0),
                                       ctx->tail_per_tile * kscale, H,
-                                      on_final, local.data());
+                                      on_final, local.data(), /*host_tok_row=*/!tile_layout);
     {
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
@@ -545,6 +545,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(cudaMemsetAsync(S.rows, 0, H.rows32 * 32, ctx->stream));
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
+    if (tile_layout) KL(lda::launch_tok_row(S, ctx->stream));
     // a1: random init (t = 0), then the count rebuild.
     CU(cudaStreamSynchronize(ctx->stream));
     lda::tmark("H2D copies");

@@ -133,7 +133,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &L,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final,
-                         const int64_t *word_counts) {
+                         const int64_t *word_counts, bool host_tok_row) {
     const bool build_pairs = sampler == 1;
     const int64_t T = doc_ptr[D];
     L.D = D;
@@ -205,7 +205,12 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // documents by decreasing length inside a part (similar θ row lengths in
     // a warp), ranks stored per token.
     const bool tile_layout = sampler == 2;
-    if (!L.tok_row.allocate(T) || !L.doc_map.allocate(T) || (!tile_layout && !L.tok_crank.allocate(T)))
+    // tile layout: the rows of the tokens (a random 4-byte scatter over the
+    // word-major stream, the costliest part of the host pass) are left to
+    // the device unless asked for (launch_tok_row from doc_map)
+    const bool want_row = !tile_layout || host_tok_row;
+    if ((want_row && !L.tok_row.allocate(T)) || !L.doc_map.allocate(T) ||
+        (!tile_layout && !L.tok_crank.allocate(T)))
         return "host allocation of the token tables failed";
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
     if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";
@@ -213,7 +218,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // the pages; every entry is written below)
     parallel_for(nthreads, T, [&](int, int64_t b, int64_t e) {
         for (int64_t i = b; i < e; i += 1024) {
-            L.tok_row[i] = 0u;
+            if (want_row) L.tok_row[i] = 0u;
             L.doc_map[i] = 0u;
             if (!tile_layout) {
                 L.tok_crank[i] = 0u;
@@ -322,6 +327,10 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         // carries its canonical rank.)
         run_parts([&](int t) {
             auto &next = pnext[t];
+            if (tile_layout && !want_row) {
+                for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) L.doc_map[i] = next[words[i]]++;
+                return;
+            }
             if (tile_layout) {
                 for (int64_t d = tdoc[t]; d < tdoc[t + 1]; ++d) {
                     const uint32_t row = L.row_off32[d];

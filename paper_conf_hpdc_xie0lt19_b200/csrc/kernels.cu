@@ -1799,6 +1799,18 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
 // ---------------------------------------------------------------------------
 // a4 epilogue (separate kernel): n_wk / n_k recount from z.
 // ---------------------------------------------------------------------------
+// a0 on the device: the θ row of every token's document at its word-major
+// position (warp per document: coalesced doc_map reads, scattered stores).
+__global__ void tok_row_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
+                               const uint32_t *__restrict__ doc_map, uint32_t *__restrict__ tok_row, int64_t D) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = static_cast<int64_t>(gridDim.x) * (blockDim.x >> 5);
+    for (int64_t d = static_cast<int64_t>(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); d < D; d += nw) {
+        const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1], row = row_off32[d];
+        for (uint32_t i = s + lane; i < e; i += 32) tok_row[doc_map[i]] = row;
+    }
+}
+
 __global__ void zero_rows_kernel(const int32_t *__restrict__ words, int64_t n, int32_t *__restrict__ nwk,
                                  int K) {
     for (int64_t i = blockIdx.x; i < n; i += gridDim.x) {
@@ -2235,6 +2247,13 @@ int launch_recount(const DevState &s, void *stream, int *launches) {
     recount_kernel<<<s.sweep_grid > 0 ? s.num_sms * 4 : 1, 256, 8 * s.K, st>>>(
         s.rchunks, s.n_rchunks, s.segs, s.K, s.tok_z, s.nwk, nk, s.counter + 1);
     ++*launches;
+    return cudaGetLastError();
+}
+
+int launch_tok_row(const DevState &s, void *stream) {
+    if (s.D > 0)
+        tok_row_kernel<<<s.num_sms * 8, 256, 0, static_cast<cudaStream_t>(stream)>>>(s.doc_ptr32, s.row_off32,
+                                                                                    s.doc_map, s.tok_row, s.D);
     return cudaGetLastError();
 }
 

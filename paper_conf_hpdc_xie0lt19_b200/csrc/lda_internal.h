@@ -135,7 +135,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &out,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {},
-                         const int64_t *word_counts = nullptr);  // V local tokens per word, if known
+                         const int64_t *word_counts = nullptr,  // V local tokens per word, if known
+                         bool host_tok_row = true);  // tile layout: false = tok_row left to the device (launch_tok_row)
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
@@ -221,6 +222,8 @@ struct DevState {
 
 int configure_kernels(DevState &s);
 int launch_init(const DevState &s, void *stream);
+// tok_row[doc_map[i]] = row_off32[d(i)] on the device (the tile layout's host pass leaves it out)
+int launch_tok_row(const DevState &s, void *stream);
 int launch_recount(const DevState &s, void *stream, int *launches);
 int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches);
 // z in document order <-> word-major, through doc_map (device buffers of T entries; zd 16-byte aligned)
