@@ -215,8 +215,10 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
     if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";
     // first touch in parallel, one store per 4 KB page (the kernel zeroes
-    // the pages; every entry is written below)
-    parallel_for(nthreads, T, [&](int, int64_t b, int64_t e) {
+    // the pages; every entry is written below).  Not needed when only
+    // doc_map is built: the tile pass writes it in order, part by part, in
+    // parallel.
+    if (want_row || !tile_layout) parallel_for(nthreads, T, [&](int, int64_t b, int64_t e) {
         for (int64_t i = b; i < e; i += 1024) {
             if (want_row) L.tok_row[i] = 0u;
             L.doc_map[i] = 0u;
