@@ -8,7 +8,7 @@ TAG=${1:-r01}
 CFG=${2:-pubmed}
 OUT=gpurun_out
 mkdir -p $OUT
-KRE='regex:^(sweep_kernel|sweep_quad_kernel|sweep_tile_kernel|word_table_kernel|recount_kernel|theta_kernel|gather_z_kernel|prologue_kernel|zero_rows_kernel|init_kernel|ll_word_kernel|ll_doc_kernel|ll_final_kernel)'
+KRE='regex:^(tok_row_kernel|init_tile_kernel|sweep_tile_cta_kernel|sweep_kernel|sweep_quad_kernel|sweep_tile_kernel|word_table_kernel|recount_kernel|theta_kernel|gather_z_kernel|prologue_kernel|zero_rows_kernel|init_kernel|ll_word_kernel|ll_doc_kernel|ll_final_kernel)'
 ncu --metrics gpu__time_duration.sum --clock-control none -k "$KRE" --csv \
     --log-file $OUT/launches_${TAG}_${CFG}.csv \
     python bench.py --config $CFG --steps 2 --warmup 3 --no-cpu-baseline > $OUT/launches_${TAG}_${CFG}.bench.log 2>&1
