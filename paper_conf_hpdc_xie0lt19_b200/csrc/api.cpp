@@ -343,8 +343,10 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     const int64_t Dg = doc_end - doc_begin;
     bool range_err = false;
     lda::tmark(nullptr);
-    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err);
-    lda::tmark("validate");
+    // one pass over the words: validation + the local word histogram
+    std::vector<int64_t> local(ctx->V, 0);
+    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, local.data());
+    lda::tmark("validate + word histogram");
     if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
     if (ctx->K > 16384)
         return fail(ctx, LDA_ERANGE, "K > 16384 is not supported by this build's shared-memory layout");
@@ -357,8 +359,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
 
     // Local word histogram -> canonical bases.  c for rank g's tokens of word
     // w starts at Σ_{w'<w} T(w') + Σ_{g'<g} T_{g'}(w)   (X18, §8(c) step 2).
-    std::vector<int64_t> local(V, 0);
-    lda::word_histogram(words, Tg, V, ctx->threads, local.data());
     std::vector<int64_t> all(static_cast<size_t>(V) * ctx->world, 0);
     if (ctx->world > 1) {
         int64_t *d_all = nullptr;
@@ -406,6 +406,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     if (tile_layout) pre.push_back({reinterpret_cast<void **>(&S.wtab), S.wt_bytes * static_cast<size_t>(V)});
     std::vector<void *> pre_done;
     size_t pre_fail_bytes = 0;
+    uint64_t pre_rows32 = 0;
     struct Job {
         uint64_t p0, p1, t0, t1;
     };
@@ -418,6 +419,13 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         cudaSetDevice(ctx->device);
         cudaStream_t cs = nullptr;
         cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+        // the θ rows: 128-byte aligned rows of min(L_d, K) + 1 words (the
+        // layout's row_off32; checked against H.rows32 after the layout)
+        uint64_t r32 = 4;
+        for (int64_t d = 0; d < Dg; ++d)
+            r32 += 4 * static_cast<uint64_t>((std::min<int64_t>(doc_ptr[d + 1] - doc_ptr[d], K) + 1 + 31) / 32);
+        pre_rows32 = r32;
+        pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
         for (auto &pa : pre) {
             if (copy_err != cudaSuccess) break;
             void *q = nullptr;
@@ -483,6 +491,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                    : std::string("token table copy: ") + cudaGetErrorString(copy_err));
     }
     if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
+    if (pre_rows32 != H.rows32) return fail(ctx, LDA_ECUDA, "internal: θ row storage size mismatch");
     lda::tmark("layout done, token tables on the device");
 
     S.V = V;
@@ -513,7 +522,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         DA(S.titems, H.titems.size());
         DA(S.cbase, V);
     }
-    DA(S.rows, H.rows32 * 8);
     S.n_zero_words = static_cast<int64_t>(H.zero_words.size());
     DA(S.zero_words, H.zero_words.size());
     DA(S.denom, K);

@@ -92,7 +92,7 @@ void word_histogram(const int32_t *words, int64_t T, int32_t V, int nthreads, in
 }
 
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
-                            bool *range_error) {
+                            bool *range_error, int64_t *word_counts) {
     *range_error = false;
     if (D < 0) return "negative document count";
     if (!doc_ptr) return "doc_ptr is NULL";
@@ -114,17 +114,30 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
     if (T > 0 && !words) return "words is NULL";
     int nth = host_threads(0);
     std::vector<int64_t> bad(nth, -1);
+    // with word_counts: the same pass counts the tokens of every word
+    const int nparts = T < (1 << 16) ? 1 : nth;
+    std::vector<std::vector<uint32_t>> h(word_counts ? nparts : 0, std::vector<uint32_t>(V, 0u));
     parallel_for(nth, T, [&](int t, int64_t b, int64_t e) {
-        for (int64_t i = b; i < e; ++i)
-            if (words[i] < 0 || words[i] >= V) {
+        uint32_t *hh = word_counts ? h[t].data() : nullptr;
+        for (int64_t i = b; i < e; ++i) {
+            const int32_t w = words[i];
+            if (w < 0 || w >= V) {
                 bad[t] = i;
                 return;
             }
+            if (hh) hh[w]++;
+        }
     });
     for (int64_t i : bad)
         if (i >= 0)
             return "word id " + std::to_string(words[i]) + " at token " + std::to_string(i) +
                    " outside [0, V)";
+    if (word_counts)
+        for (int32_t w = 0; w < V; ++w) {
+            int64_t c = 0;
+            for (const auto &hh : h) c += hh[w];
+            word_counts[w] = c;
+        }
     return "";
 }
 

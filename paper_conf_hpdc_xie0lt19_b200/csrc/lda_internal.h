@@ -141,7 +141,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
-                            bool *range_error);
+                            bool *range_error, int64_t *word_counts = nullptr);  // V counts, if wanted
 
 int host_threads(int requested);
 
