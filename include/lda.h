@@ -68,14 +68,14 @@ typedef struct lda_stats {
     double ms_sample;       /* prologue + sampling kernel (Alg. 2, K1) */
     double ms_recount;      /* n_wk / n_k rebuild (K2) */
     double ms_theta;        /* θ rebuild (K3+K4) */
-    double ms_allreduce;    /* raw NCCL allreduce time on the comm stream (0 if world==1) */
+    double ms_allreduce;    /* raw allreduce time on the comm stream (0 if world==1) */
     double ms_last_sweep;   /* compute-stream time of the last sweep only */
     double ms_last_sample;  /* sampling kernel time of the last sweep only */
     int64_t sum_nnz_tok;    /* Σ_t nnz_{d(t)} read by the last sweep's sampler */
     int64_t sum_nnz_doc;    /* Σ_d nnz_d of θ after the last sweep */
     int64_t n_launches;     /* library kernels launched by the last call */
     int64_t n_sample_chunks;/* sampler work items (word chunks) */
-    int64_t n_exact_redraws;/* samplers 1, 2: tokens of the last lda_iterate
+    int64_t n_exact_redraws;/* samplers 2, 3: tokens of the last lda_iterate
                                call whose fp32 draw could not be certified and
                                that were redrawn by the exact fp64 walk */
     double ms_table;        /* samplers 2, 3: the per-word table kernel (a3), part of
@@ -83,44 +83,55 @@ typedef struct lda_stats {
     double ms_allreduce_exposed; /* world > 1: time the compute stream waited for
                                the allreduce after the θ rebuild (the part of
                                ms_allreduce not hidden behind it) */
+    int64_t tile_tokens;    /* document tile size the layout used (0: one tile) */
+    int32_t n_tiles;        /* tiles, including the tail tile */
+    int32_t sampler;        /* the sampler that runs: 0, 2 or 3 (see "sampler") */
+    double bytes_alg;       /* SURVEY §8(d) algorithmic bytes of the last sweep on
+                               this rank: 20·T_g + 4·Σ_t nnz_d(t) + 8·V·K
+                               + 4·Σ_d nnz'_d + 8·D_g */
+    double bytes_sample;    /* the sampling kernel's share of it:
+                               14·T_g + 4·Σ_t nnz_d(t) + 4·V·K */
 } lda_stats;
 
 /* Create a context.  D = global number of documents, V = vocabulary size,
  * K = number of topics, α, β = Dirichlet hyper-parameters (Eq. 1; the paper
  * uses α = 50/K, β = 0.01 at L1339, X1).  No device work is done.
  * Errors: LDA_EINVAL unless D >= 1, V >= 1, 1 <= K <= 65536 (topic ids are
- * uint16, L1239-1243), α and β finite and > 0.  *out is set to NULL on error. */
+ * uint16, L1239-1243), α and β finite and > 0; LDA_ERANGE for
+ * 16384 < K <= 65536 (this build packs a θ entry as topic << 18 | count and
+ * keeps K-length histograms in shared memory).  *out is set to NULL on error. */
 int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_ctx **out);
 
 /* Set an integer option before lda_load_corpus (LDA_ESTATE after).  Keys:
  *   "device"        CUDA device ordinal (default 0)
  *   "exclude_self"  0 (default; Eq. 1 as printed, X2) or 1 (remove the
- *                   token's own old topic from the counts it draws against)
+ *                   token's own old topic from the counts it draws against;
+ *                   runs on sampler 0)
+ *   "tile_tokens"   -1 (default, auto): split the documents into tiles whose
+ *                   θ rows fill about half the L2 (one tile if all rows fit)
+ *                   and sample tile by tile, so that every tile's rows are
+ *                   read from HBM about once per sweep; 0: one tile; n > 0:
+ *                   tiles of about n tokens
  *   "chunk_tokens"  max tokens per sampling work item (default 4096)
  *   "recount_tokens" max tokens per n_wk recount work item (default 65536)
- *   "tile_tokens"   split the documents into tiles of about this many tokens
- *                   and sample tile by tile (0 = one tile, the default)
  *   "threads"       host threads for corpus preparation (default: all)
  *   "sampler"       -1 (default): 2 if K <= 4096, else 3.
- *                   2: tile sampler -- work items are the tokens
- *                   of one word inside one document tile, queued tile by
- *                   tile so the tiles' θ rows stay in L2; one warp per item,
- *                   the word's p* and dense-prefix table (built once per sweep)
+ *                   2: tile sampler -- work items are the tokens of one word
+ *                   inside one document tile, queued tile by tile so the
+ *                   tiles' θ rows stay in L2; one warp per item, the word's
+ *                   p* and dense-prefix table (built once per sweep)
  *                   bulk-copied to shared memory, four lanes walk a θ row
  *                   line by line, draws in fp32 certified against rigorous
  *                   error bounds (uncertain tokens redrawn in fp64).
- *                   Needs exclude_self = 0 and K within its shared-memory
- *                   layout (else sampler 0); at K = 8192 its per-warp
- *                   tables leave too few warps per SM (measured slower
- *                   than sampler 0, hence the default).
- *                   3: the tile sampler with the word table shared by the
- *                   8 warps of a CTA (double-buffered) -- large K (at
- *                   K = 8192: 1.7x the lane-per-token sampler); same draws
- *                   as 2.  Falls back to 0 when its tables do not fit.
- *                   1: quad sampler over (word, document) pairs.
- *                   0: lane-per-token fp64 sampler (32-byte row blocks).
- *                   The samplers differ only in rounding at a CDF boundary
- *                   (draws differ only within fp64 rounding of it).
+ *                   3: the tile sampler with the word tables shared by the
+ *                   warps of a CTA (several buffers in flight) -- large K;
+ *                   same draws as 2.
+ *                   0: lane-per-token fp64 sampler (32-byte row blocks); the
+ *                   path of exclude_self = 1.
+ *                   2 and 3 fall back to 0 with exclude_self = 1 or when
+ *                   their shared-memory layout does not fit.  The samplers
+ *                   differ only in rounding at a CDF boundary (draws differ
+ *                   only within fp64 rounding of it).
  *   "tail_per_tile" samplers 2, 3: words with fewer than this many tokens
  *                   per document tile on average are sampled as one
  *                   corpus-wide item each (default 64; 0 = off).  Sampler 3
@@ -133,15 +144,12 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   2.7 % faster per sweep at PubMed shape); 1 = accumulated
  *                   by the sampler itself (warp-aggregated reductions).  Same
  *                   counts.
- *   "certify_slack" sampler 2, tests only: multiply every certification
+ *   "certify_slack" samplers 2, 3, tests only: multiply every certification
  *                   bound by this factor (default 1) -- more tokens take the
  *                   exact fp64 redraw; the draws must not change
- *   "filter32"      sampler 0 only.  1: draw each token in fp32 first and
- *                   redo it in fp64 when its uniform lies within the fp32
- *                   error bound of a CDF boundary — results identical to 0
- *                   (always fp64, default)
- *   "theta_mode"    θ rebuild: 0 = fused gather+histogram (default),
- *                   1 = two-phase (z gathered into document order first)
+ *   "loglik_every"  n > 0: lda_iterate evaluates the LL/token (as lda_loglik)
+ *                   after every sweep t with t % n == 0, outside the sweep's
+ *                   timed phases; read with lda_get_loglik_log (default 0)
  * Results do not depend on chunk_tokens, recount_tokens, tile_tokens or
  * threads (the draw of every token is a function of the frozen counts and
  * its canonical index only).
@@ -157,6 +165,25 @@ int lda_init_dist(lda_ctx *ctx, int32_t rank, int32_t world, const void *nccl_un
 
 /* Write a fresh 128-byte ncclUniqueId to out128 (host-only helper). */
 int lda_nccl_unique_id(void *out128);
+
+/* In-process multi-GPU: a group of `world` ranks (1..16) in ONE process,
+ * each rank a context driven by its own host thread, on its own GPU (P2P
+ * over NVLink) or several on one GPU.  The n_wk/n_k exchange of Eq. 4
+ * (L935-937) reads the peers' device buffers directly: a reduce-scatter
+ * kernel (rank r sums slice r over all ranks in place), then an all-gather
+ * kernel, ordered by host barriers.  Collective calls (lda_load_corpus,
+ * lda_iterate, lda_loglik, lda_set_z) must be made by every rank's thread
+ * concurrently; a rank that fails or does not arrive within 600 s breaks
+ * the group (every later collective fails with LDA_ECUDA).
+ * lda_peer_group_create: *out receives the group handle (LDA_EINVAL for a
+ * bad world).  lda_init_peer: join as `rank` before lda_load_corpus
+ * (LDA_EINVAL: bad or duplicate rank; LDA_ESTATE: after load or after
+ * lda_init_dist).  The group's state is shared by its contexts:
+ * lda_peer_group_destroy may be called once every rank has joined. */
+typedef struct lda_peer_group lda_peer_group;
+int lda_peer_group_create(int32_t world, lda_peer_group **out);
+int lda_init_peer(lda_ctx *ctx, lda_peer_group *group, int32_t rank);
+void lda_peer_group_destroy(lda_peer_group *group);
 
 /* Token-balanced contiguous document partition (§4 "evenly
  * partitioned by number of tokens", X21): rank g owns documents
@@ -179,7 +206,7 @@ int lda_canonical_bases(int32_t V, int32_t world, int32_t rank, const int64_t *w
 
 /* Host-only diagnostic (no device needed): build the token layout that
  * lda_load_corpus would build for a one-rank corpus (doc_ptr: D+1 offsets,
- * words: T ids < V) with the given sampler (0-3), tile_tokens,
+ * words: T ids < V) with the given sampler (0, 2 or 3), tile_tokens,
  * chunk_tokens and tail_per_tile, and check its invariants against brute
  * force: doc_map is a permutation of [0, T); tok_row[doc_map[i]] is the θ
  * row of token i's document; every (tile, word) run holds only that word;
@@ -240,6 +267,12 @@ int lda_get_stats(lda_ctx *ctx, lda_stats *out);
 int lda_get_sweep_log(lda_ctx *ctx, int32_t cap, double *ms_sweep, double *ms_sample, double *ms_recount,
                       double *ms_theta, double *ms_allreduce, int64_t *sum_nnz_tok, int64_t *sum_nnz_doc,
                       int32_t *n_out);
+
+/* LL/token log of the last lda_iterate call (option "loglik_every"): up to
+ * `cap` entries of each non-NULL array -- the sweep counter t after which
+ * it was taken and the LL/token (lda_loglik's definition).  *n_out = number
+ * of entries in that call. */
+int lda_get_loglik_log(lda_ctx *ctx, int32_t cap, int64_t *sweep, double *ll_per_token, int32_t *n_out);
 
 /* The CUDA stream (cudaStream_t) the sweep kernels run on; valid after
  * lda_load_corpus until lda_destroy. */

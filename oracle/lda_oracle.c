@@ -34,6 +34,9 @@
  * No function is "parity unpinned".
  */
 #include <math.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -335,6 +338,40 @@ void orc_sweep(int64_t D, int32_t V, int32_t K, double alpha, double beta,
     memcpy(z, z_new, sizeof(uint16_t) * (size_t)T);
     free(z_new);
     orc_counts(D, V, K, doc_ptr, words, z, n_wk, n_k, n_dk);
+}
+
+/* oracle-omp (optional): the same SWEEP with the documents'
+ * draws spread over the host cores (OpenMP; without -fopenmp the pragma is
+ * ignored and this is orc_sweep).  Every draw reads only the counts frozen at
+ * the start of the sweep and its own counter-based uniform (X3, X9), so the
+ * order of the documents cannot change any result: z and the counts are
+ * bit-identical to orc_sweep's (pinned in tests/test_oracle_pins.py).  Used
+ * only to make the 100-sweep LL parity run on a 1M-token corpus tractable. */
+void orc_sweep_omp(int64_t D, int32_t V, int32_t K, double alpha, double beta,
+                   const int64_t *doc_ptr, const int32_t *words, const int64_t *canon,
+                   uint64_t seed, uint32_t t, int exclude_self, uint16_t *z,
+                   int32_t *n_wk, int32_t *n_k, int32_t *n_dk, double *margin)
+{
+    int64_t T = doc_ptr[D];
+    uint16_t *z_new = (uint16_t *)malloc(sizeof(uint16_t) * (size_t)(T > 0 ? T : 1));
+    int64_t d;
+#pragma omp parallel for schedule(dynamic, 64)
+    for (d = 0; d < D; d++)
+        orc_draw_docs(d, d + 1, V, K, alpha, beta, doc_ptr, words, canon, seed, t, exclude_self, z,
+                      n_wk, n_k, n_dk, z_new, margin);
+    memcpy(z, z_new, sizeof(uint16_t) * (size_t)T);
+    free(z_new);
+    orc_counts(D, V, K, doc_ptr, words, z, n_wk, n_k, n_dk);
+}
+
+/* number of threads orc_sweep_omp uses (1 without OpenMP) */
+int orc_omp_threads(void)
+{
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
 }
 
 /* SEQUENTIAL mode: textbook collapsed Gibbs sampling (CGS, L389-409 "CGS

@@ -28,7 +28,7 @@ def build_oracle(force: bool = False) -> str:
     """Compile the C oracle (plain gcc, IEEE fp64, no FMA contraction)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         cmd = ["gcc", "-std=c11", "-O2", "-fPIC", "-shared", "-ffp-contract=off",
-               "-fno-fast-math", _SRC, "-o", _LIB + ".tmp", "-lm"]
+               "-fno-fast-math", "-fopenmp", _SRC, "-o", _LIB + ".tmp", "-lm"]
         subprocess.check_call(cmd)
         os.replace(_LIB + ".tmp", _LIB)
     return _LIB
@@ -77,6 +77,10 @@ def lib():
                                     c.c_double, _i64p, _i32p, _i64p, c.c_uint64, c.c_uint32,
                                     c.c_int, _u16p, _i32p, _i32p, _i32p, _u16p, c.c_void_p]
         L.orc_draw_docs.restype = None
+        L.orc_sweep_omp.argtypes = L.orc_sweep.argtypes
+        L.orc_sweep_omp.restype = None
+        L.orc_omp_threads.argtypes = []
+        L.orc_omp_threads.restype = c.c_int
         L.orc_sweep_sequential.argtypes = [c.c_int64, c.c_int32, c.c_int32, c.c_double,
                                            c.c_double, _i64p, _i32p, _i64p, c.c_uint64,
                                            c.c_uint32, _u16p, _i32p, _i32p, _i32p]
@@ -159,17 +163,24 @@ def draw(K, V, alpha, beta, nwk_row, n_k, ndk_row, x0, exclude_self=0, z_old=-1)
 
 
 def draw_docs(d_begin, d_end, doc_ptr, words, canon, V, K, alpha, beta, seed, t, z, n_wk, n_k,
-              n_dk, exclude_self=0):
+              n_dk, exclude_self=0, margins=False):
     """New topics of the tokens of documents [d_begin, d_end) against the given
-    global counts (input order; other entries of the result are 0)."""
+    global counts (input order; other entries of the result are 0).  canon[i]
+    is token i's global canonical index, n_dk the dense rows of these
+    documents.  With margins=True also returns each token's margin."""
     z = np.ascontiguousarray(z, np.uint16)
     out = np.zeros_like(z)
+    m = np.full(len(z), np.inf) if margins else None
     lib().orc_draw_docs(d_begin, d_end, V, K, alpha, beta, np.ascontiguousarray(doc_ptr, np.int64),
                         np.ascontiguousarray(words, np.int32), np.ascontiguousarray(canon, np.int64),
                         seed, t, exclude_self, z, np.ascontiguousarray(n_wk, np.int32).reshape(-1),
                         np.ascontiguousarray(n_k, np.int32), np.ascontiguousarray(n_dk, np.int32).reshape(-1),
-                        out, None)
-    return out
+                        out, _vp(m))
+    return (out, m) if margins else out
+
+
+def omp_threads() -> int:
+    return int(lib().orc_omp_threads())
 
 
 def loglik(doc_ptr, V, K, alpha, beta, n_wk, n_k, n_dk):
@@ -227,12 +238,15 @@ class OracleLDA:
         self.z[:] = np.asarray(z, np.uint16)
         self._recount()
 
-    def iterate(self, n=1, mode="sweep", exclude_self=0, margins=False):
+    def iterate(self, n=1, mode="sweep", exclude_self=0, margins=False, parallel=False):
+        """mode "sweep" (the GPU semantics) or "sequential"; parallel=True runs
+        the sweep's draws on all host cores (oracle-omp, bit-identical)."""
         m = np.empty(self.T, np.float64) if margins else None
+        sweep = lib().orc_sweep_omp if parallel else lib().orc_sweep
         for _ in range(n):
             self.t += 1
             if mode == "sweep":
-                lib().orc_sweep(self.D, self.V, self.K, self.alpha, self.beta,
+                sweep(self.D, self.V, self.K, self.alpha, self.beta,
                                 self.doc_ptr, self.words, self.canon, self.seed,
                                 self.t, exclude_self, self.z, self.n_wk, self.n_k,
                                 self.n_dk, _vp(m))

@@ -23,11 +23,12 @@ STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4:
           -5: "LDA_ENCCL", -6: "LDA_ESTATE"}
 
 # every symbol include/lda.h declares
-ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_partition_docs",
+ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_peer_group_create",
+               "lda_init_peer", "lda_peer_group_destroy", "lda_partition_docs",
                "lda_canonical_bases", "lda_layout_selfcheck",
                "lda_load_corpus", "lda_iterate", "lda_loglik", "lda_get_counts", "lda_get_stats",
-               "lda_get_sweep_log", "lda_get_stream", "lda_set_z", "lda_destroy", "lda_last_error",
-               "lda_version")
+               "lda_get_sweep_log", "lda_get_loglik_log", "lda_get_stream", "lda_set_z", "lda_destroy",
+               "lda_last_error", "lda_version")
 
 
 class LDAError(RuntimeError):
@@ -46,7 +47,9 @@ class lda_stats(ctypes.Structure):
                 ("ms_last_sample", ctypes.c_double), ("sum_nnz_tok", ctypes.c_int64),
                 ("sum_nnz_doc", ctypes.c_int64), ("n_launches", ctypes.c_int64),
                 ("n_sample_chunks", ctypes.c_int64), ("n_exact_redraws", ctypes.c_int64),
-                ("ms_table", ctypes.c_double), ("ms_allreduce_exposed", ctypes.c_double)]
+                ("ms_table", ctypes.c_double), ("ms_allreduce_exposed", ctypes.c_double),
+                ("tile_tokens", ctypes.c_int64), ("n_tiles", ctypes.c_int32), ("sampler", ctypes.c_int32),
+                ("bytes_alg", ctypes.c_double), ("bytes_sample", ctypes.c_double)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -69,6 +72,10 @@ def lib():
             "lda_set_option": ([_vp, ctypes.c_char_p, _i64], ctypes.c_int),
             "lda_init_dist": ([_vp, _i32, _i32, _vp], ctypes.c_int),
             "lda_nccl_unique_id": ([_vp], ctypes.c_int),
+            "lda_peer_group_create": ([_i32, ctypes.POINTER(_vp)], ctypes.c_int),
+            "lda_init_peer": ([_vp, _vp, _i32], ctypes.c_int),
+            "lda_peer_group_destroy": ([_vp], None),
+            "lda_get_loglik_log": ([_vp, _i32, _vp, _vp, ctypes.POINTER(_i32)], ctypes.c_int),
             "lda_partition_docs": ([_i64, _vp, _i32, _vp], ctypes.c_int),
             "lda_canonical_bases": ([_i32, _i32, _i32, _vp, _vp, ctypes.POINTER(_i64)], ctypes.c_int),
             "lda_layout_selfcheck": ([_i64, _i32, _i32, _vp, _vp, _i32, _i64, _i64, _i64, _vp, ctypes.c_char_p,
@@ -149,7 +156,7 @@ def lda_layout_selfcheck(doc_ptr, words, V, K, sampler=2, tile_tokens=0, chunk_t
     r = lib().lda_layout_selfcheck(len(doc_ptr) - 1, int(V), int(K), _p(doc_ptr), _p(words), int(sampler),
                                    int(tile_tokens), int(chunk_tokens), int(tail_per_tile), _p(st), buf, 256)
     if r != 0:
-        raise LDAError(f"lda_layout_selfcheck: {buf.value.decode()} (status {r})")
+        raise LDAError(r, f"lda_layout_selfcheck: {buf.value.decode()}")
     return dict(zip(("tiles", "items", "tail_words", "runs"), st.tolist()))
 
 
@@ -166,6 +173,11 @@ def lda_canonical_bases(word_counts, rank):
 def lda_load_corpus(ctx, doc_begin, doc_end, doc_ptr, words, seed):
     doc_ptr = np.ascontiguousarray(doc_ptr, np.int64)
     words = np.ascontiguousarray(words, np.int32)
+    # the C side reads doc_ptr[0 .. doc_end-doc_begin] and words[0 .. doc_ptr[-1])
+    if doc_ptr.ndim != 1 or len(doc_ptr) != int(doc_end) - int(doc_begin) + 1:
+        raise LDAError(LDA_EINVAL, "len(doc_ptr) must be doc_end - doc_begin + 1")
+    if len(doc_ptr) and (doc_ptr[-1] < 0 or len(words) < int(doc_ptr[-1])):
+        raise LDAError(LDA_EINVAL, "len(words) must be >= doc_ptr[-1]")
     _check(lib().lda_load_corpus(ctx, int(doc_begin), int(doc_end), _p(doc_ptr), _p(words),
                                  int(seed) & 0xFFFFFFFFFFFFFFFF), ctx)
 
@@ -180,9 +192,25 @@ def lda_loglik(ctx) -> float:
     return v.value
 
 
+def _out(a, dtype, n, name):
+    if a is None:
+        return
+    if a.dtype != dtype or not a.flags.c_contiguous or a.size < n:
+        raise LDAError(LDA_EINVAL, f"{name} must be a C-contiguous {np.dtype(dtype).name} array of >= {n} entries")
+
+
 def lda_get_counts(ctx, n_wk=None, n_k=None, ndk_ptr=None, ndk_topic=None, ndk_count=None, z=None,
-                   want_nnz=False):
-    """Fills the given (preallocated, C-contiguous) numpy arrays; returns nnz."""
+                   want_nnz=False, shape=None):
+    """Fills the given (preallocated, C-contiguous) numpy arrays; returns nnz.
+    shape = (V, K, D_g, T_g) enables the size checks (LDA does this)."""
+    if shape is not None:
+        V, K, Dg, Tg = shape
+        _out(n_wk, np.int32, V * K, "n_wk")
+        _out(n_k, np.int32, K, "n_k")
+        _out(ndk_ptr, np.int64, Dg + 1, "ndk_ptr")
+        _out(z, np.uint16, Tg, "z")
+    _out(ndk_topic, np.uint16, 0, "ndk_topic")
+    _out(ndk_count, np.int32, 0, "ndk_count")
     nnz = _i64()
     cap = 0 if ndk_topic is None else len(ndk_topic)
     if ndk_count is not None:
@@ -215,14 +243,61 @@ def lda_get_sweep_log(ctx) -> dict:
     return arr
 
 
+def lda_get_loglik_log(ctx) -> dict:
+    n = _i32()
+    _check(lib().lda_get_loglik_log(ctx, 0, None, None, ctypes.byref(n)), ctx)
+    sw = np.zeros(n.value, np.int64)
+    ll = np.zeros(n.value, np.float64)
+    _check(lib().lda_get_loglik_log(ctx, n.value, _p(sw), _p(ll), ctypes.byref(n)), ctx)
+    return {"sweep": sw, "ll_per_token": ll}
+
+
+def lda_peer_group_create(world):
+    h = _vp()
+    _check(lib().lda_peer_group_create(int(world), ctypes.byref(h)))
+    return h
+
+
+def lda_init_peer(ctx, group, rank):
+    _check(lib().lda_init_peer(ctx, group, int(rank)), ctx)
+
+
+def lda_peer_group_destroy(group):
+    if group:
+        lib().lda_peer_group_destroy(group)
+
+
+class PeerGroup:
+    """In-process group of `world` ranks (include/lda.h lda_peer_group_*):
+    each rank's LDA is driven by its own thread; the n_wk/n_k exchange reads
+    the peers' device buffers directly."""
+
+    def __init__(self, world):
+        self.world = int(world)
+        self.h = lda_peer_group_create(self.world)
+
+    def close(self):
+        if self.h:
+            lda_peer_group_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
 def lda_get_stream(ctx) -> int:
     s = _vp()
     _check(lib().lda_get_stream(ctx, ctypes.byref(s)), ctx)
     return int(s.value or 0)
 
 
-def lda_set_z(ctx, z):
+def lda_set_z(ctx, z, T=None):
     z = np.ascontiguousarray(z, np.uint16)
+    if T is not None and z.shape != (int(T),):
+        raise LDAError(LDA_EINVAL, f"z must hold exactly T = {T} topics")
     _check(lib().lda_set_z(ctx, _p(z)), ctx)
 
 
@@ -255,6 +330,9 @@ class LDA:
     def init_dist(self, rank, world, unique_id):
         lda_init_dist(self.ctx, rank, world, unique_id)
 
+    def init_peer(self, group, rank):
+        lda_init_peer(self.ctx, group.h if isinstance(group, PeerGroup) else group, rank)
+
     def load(self, doc_ptr, words, seed, doc_begin=0, doc_end=None):
         self.doc_begin = int(doc_begin)
         self.doc_end = self.D if doc_end is None else int(doc_end)
@@ -276,20 +354,23 @@ class LDA:
             out = np.empty(self.T, np.uint16)
         elif out.dtype != np.uint16 or out.shape != (self.T,) or not out.flags.c_contiguous:
             raise ValueError("out must be a contiguous uint16 array of T entries")
-        lda_get_counts(self.ctx, z=out)
+        lda_get_counts(self.ctx, z=out, shape=self._shape())
         return out
 
+    def _shape(self):
+        return (self.V, self.K, self.doc_end - self.doc_begin, self.T)
+
     def set_z(self, z):
-        lda_set_z(self.ctx, z)
+        lda_set_z(self.ctx, z, T=self.T)
 
     def nwk(self):
         a = np.empty(self.V * self.K, np.int32)
-        lda_get_counts(self.ctx, n_wk=a)
+        lda_get_counts(self.ctx, n_wk=a, shape=self._shape())
         return a.reshape(self.V, self.K)
 
     def nk(self):
         a = np.empty(self.K, np.int32)
-        lda_get_counts(self.ctx, n_k=a)
+        lda_get_counts(self.ctx, n_k=a, shape=self._shape())
         return a
 
     def theta_csr(self):
@@ -298,7 +379,7 @@ class LDA:
         ptr = np.empty(Dg + 1, np.int64)
         top = np.empty(nnz, np.uint16)
         cnt = np.empty(nnz, np.int32)
-        lda_get_counts(self.ctx, ndk_ptr=ptr, ndk_topic=top, ndk_count=cnt)
+        lda_get_counts(self.ctx, ndk_ptr=ptr, ndk_topic=top, ndk_count=cnt, shape=self._shape())
         return ptr, top, cnt
 
     def ndk_dense(self):
@@ -314,6 +395,9 @@ class LDA:
 
     def sweep_log(self):
         return lda_get_sweep_log(self.ctx)
+
+    def loglik_log(self):
+        return lda_get_loglik_log(self.ctx)
 
     def stream(self):
         return lda_get_stream(self.ctx)

@@ -1,13 +1,6 @@
-"""Launch configuration shared by bench.py and the full-size parity test, so
-the parity test checks exactly the configuration the bench times."""
-
-# Options passed to lda_set_option for the timed runs.
-BENCH_OPTIONS = {
-    "chunk_tokens": 4096,
-    "recount_tokens": 65536,
-    "tile_tokens": 16_000_000,
-    "theta_mode": 1,
-}
+"""Byte models shared by bench.py, the tools and the tests.  The bench runs
+the library's defaults (no lda_set_option calls): the timed configuration is
+the one lda_create -> lda_load_corpus -> lda_iterate gives every user."""
 
 # Algorithmic bytes per sweep, per GPU:
 #   B_alg = T_g·20 + 4·Σ_t nnz_{d(t)} + 8·V·K + 4·Σ_d nnz'_d + 8·D_g

@@ -28,27 +28,26 @@ struct lda_ctx {
     int exclude_self = 0;
     int64_t chunk_tokens = 4096;
     int64_t recount_tokens = 65536;
-    int64_t tile_tokens = 0;
-    int theta_mode = 0;
-    int filter32 = 0;
+    int64_t tile_tokens = -1;  // auto: tiles whose θ rows fill about half the L2
     int sampler = -1;  // auto
     int64_t tail_per_tile = 64;
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int threads = 0;
-    // distribution
+    // distribution: the exchange of Eq. 4 (NCCL or the in-process peer group)
     int32_t rank = 0, world = 1;
-    ncclComm_t comm = nullptr;
+    std::unique_ptr<lda::Comm> comm;
     // state
     bool loaded = false;
     int failed = 0;
     std::string err;
     uint64_t sweeps = 0;
     int64_t T_global = 0;
+    int64_t tile_tokens_used = 0;
     lda::HostLayout H;
     lda::DevState S;
     cudaStream_t stream = nullptr, comm_stream = nullptr;
-    std::vector<cudaEvent_t> ev;  // 6 per sweep
+    std::vector<cudaEvent_t> ev;  // 7 per sweep
     lda_stats stats{};
     std::vector<void *> allocs;
     // θ statistics: Σ_d L_d·nnz_d (= Σ_t nnz_{d(t)}) and Σ_d nnz_d of the
@@ -58,61 +57,21 @@ struct lda_ctx {
     size_t stat_log_cap = 0;
     std::vector<double> log_ms, log_ms_sample, log_ms_recount, log_ms_theta, log_ms_comm;
     std::vector<int64_t> log_nnz_tok, log_nnz_doc;
+    // option loglik_every: LL/token after every n-th sweep of lda_iterate
+    int64_t loglik_every = 0;
+    double *d_ll_log = nullptr;
+    std::vector<int64_t> ll_sweep;
+    std::vector<double> ll_value;
+};
+
+// Handle of an in-process peer group (shared by its ranks' contexts).
+struct lda_peer_group {
+    std::shared_ptr<lda::PeerGroup> g;
 };
 
 namespace {
 
-// NCCL is opened at run time (only multi-GPU contexts need it), so that
-// loading liblda.so never pins an NCCL build into the process before torch
-// loads its own.  dlopen("libnccl.so.2") returns the copy already loaded by
-// torch when there is one; LDA_NCCL_LIBRARY overrides the path.
-struct NcclApi {
-    ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
-    ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
-    ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
-                              cudaStream_t) = nullptr;
-    ncclResult_t (*AllGather)(const void *, void *, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
-    ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
-    const char *(*GetErrorString)(ncclResult_t) = nullptr;
-    std::string err;
-    bool ok = false;
-};
-
-NcclApi load_nccl() {
-    NcclApi a;
-    const char *env = std::getenv("LDA_NCCL_LIBRARY");
-    const char *cands[] = {env, "libnccl.so.2", "libnccl.so"};
-    void *h = nullptr;
-    for (const char *c : cands) {
-        if (!c) continue;
-        h = dlopen(c, RTLD_NOW | RTLD_GLOBAL);
-        if (h) break;
-    }
-    if (!h) {
-        a.err = std::string("cannot dlopen NCCL: ") + dlerror();
-        return a;
-    }
-#define LDA_SYM(field, name)                                              \
-    a.field = reinterpret_cast<decltype(a.field)>(dlsym(h, name));        \
-    if (!a.field) {                                                       \
-        a.err = std::string("NCCL symbol missing: ") + name;              \
-        return a;                                                         \
-    }
-    LDA_SYM(GetUniqueId, "ncclGetUniqueId")
-    LDA_SYM(CommInitRank, "ncclCommInitRank")
-    LDA_SYM(AllReduce, "ncclAllReduce")
-    LDA_SYM(AllGather, "ncclAllGather")
-    LDA_SYM(CommDestroy, "ncclCommDestroy")
-    LDA_SYM(GetErrorString, "ncclGetErrorString")
-#undef LDA_SYM
-    a.ok = true;
-    return a;
-}
-
-const NcclApi &nccl() {
-    static NcclApi api = load_nccl();
-    return api;
-}
+constexpr int32_t kMaxK = 16384;
 
 int fail(lda_ctx *c, int code, const std::string &msg) {
     if (c) {
@@ -137,12 +96,16 @@ int fail(lda_ctx *c, int code, const std::string &msg) {
                         std::string(#call) + ": " + cudaGetErrorString(static_cast<cudaError_t>(e_))); \
     } while (0)
 
-#define NC(call)                                                                                  \
-    do {                                                                                          \
-        if (!nccl().ok) return fail(ctx, LDA_ENCCL, nccl().err);                                  \
-        ncclResult_t r_ = nccl().call;                                                            \
-        if (r_ != ncclSuccess)                                                                    \
-            return fail(ctx, LDA_ENCCL, std::string(#call) + ": " + nccl().GetErrorString(r_));   \
+// a collective of the context's communicator; failures are sticky
+#define COMM(call)                                                  \
+    do {                                                            \
+        std::string e_;                                             \
+        int r_ = ctx->comm->call;                                   \
+        if (r_ != LDA_OK) {                                         \
+            ctx->err = std::string(ctx->comm->name()) + ": " + e_;  \
+            ctx->failed = r_ == LDA_ENCCL ? LDA_ENCCL : LDA_ECUDA;  \
+            return ctx->failed;                                     \
+        }                                                           \
     } while (0)
 
 #define PRECHECK(ctx)                                   \
@@ -185,8 +148,7 @@ int rebuild_counts(lda_ctx *ctx, int *launches) {
     lda::DevState &S = ctx->S;
     KL(lda::launch_recount(S, ctx->stream, launches));
     if (ctx->world > 1) {
-        NC(AllReduce(S.nwk, S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ncclInt32, ncclSum, ctx->comm,
-                         ctx->stream));
+        COMM(allreduce_i32(S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ctx->stream, e_));
     }
     KL(lda::launch_theta(S, S.stat, ctx->stream, launches));
     unsigned long long hs[2] = {0, 0};
@@ -213,6 +175,9 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
     *out = nullptr;
     if (D < 1 || V < 1 || K < 1 || K > 65536) return LDA_EINVAL;
     if (!std::isfinite(alpha) || !std::isfinite(beta) || !(alpha > 0) || !(beta > 0)) return LDA_EINVAL;
+    // u16 topic ids allow K <= 65536 (L1239-1243); this build's θ entry
+    // (topic << 18 | count) and shared-memory histograms stop at 16384
+    if (K > kMaxK) return LDA_ERANGE;
     lda_ctx *c = new (std::nothrow) lda_ctx();
     if (!c) return LDA_ENOMEM;
     c->D = D;
@@ -242,13 +207,11 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
         if (value < 256 || value > (int64_t(1) << 31)) return fail(ctx, LDA_EINVAL, "recount_tokens out of range");
         ctx->recount_tokens = value;
     } else if (k == "tile_tokens") {
-        if (value < 0) return fail(ctx, LDA_EINVAL, "tile_tokens must be >= 0");
+        if (value < -1) return fail(ctx, LDA_EINVAL, "tile_tokens must be -1 (auto) or >= 0");
         ctx->tile_tokens = value;
-    } else if (k == "filter32") {
-        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "filter32 must be 0 or 1");
-        ctx->filter32 = static_cast<int>(value);
     } else if (k == "sampler") {
-        if (value < -1 || value > 3) return fail(ctx, LDA_EINVAL, "sampler must be -1 (auto), 0, 1, 2 or 3");
+        if (value != -1 && value != 0 && value != 2 && value != 3)
+            return fail(ctx, LDA_EINVAL, "sampler must be -1 (auto), 0, 2 or 3");
         ctx->sampler = static_cast<int>(value);
     } else if (k == "tail_per_tile") {
         if (value < 0 || value > (int64_t(1) << 30)) return fail(ctx, LDA_EINVAL, "tail_per_tile out of range");
@@ -259,9 +222,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
-    } else if (k == "theta_mode") {
-        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_mode must be 0 or 1");
-        ctx->theta_mode = static_cast<int>(value);
+    } else if (k == "loglik_every") {
+        if (value < 0 || value > (int64_t(1) << 31)) return fail(ctx, LDA_EINVAL, "loglik_every must be >= 0");
+        ctx->loglik_every = value;
     } else if (k == "threads") {
         if (value < 0 || value > 1024) return fail(ctx, LDA_EINVAL, "threads out of range");
         ctx->threads = static_cast<int>(value);
@@ -273,24 +236,50 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
 
 int lda_nccl_unique_id(void *out128) {
     if (!out128) return LDA_EINVAL;
-    ncclUniqueId id;
-    if (!nccl().ok || nccl().GetUniqueId(&id) != ncclSuccess) return LDA_ENCCL;
-    std::memcpy(out128, &id, sizeof(id));
-    return LDA_OK;
+    std::string err;
+    return lda::nccl_unique_id(out128, err);
 }
 
 int lda_init_dist(lda_ctx *ctx, int32_t rank, int32_t world, const void *uid) {
     PRECHECK(ctx);
     if (ctx->loaded || ctx->comm) return fail(ctx, LDA_ESTATE, "lda_init_dist must precede lda_load_corpus");
     if (world < 1 || rank < 0 || rank >= world) return fail(ctx, LDA_EINVAL, "bad rank/world");
+    if (world == 1) {
+        ctx->rank = 0;
+        ctx->world = 1;
+        return LDA_OK;
+    }
+    if (!uid) return fail(ctx, LDA_EINVAL, "null nccl unique id");
+    std::string err;
+    int r = lda::make_nccl_comm(rank, world, uid, ctx->device, ctx->comm, err);
+    if (r != LDA_OK) return fail(ctx, r, err);
     ctx->rank = rank;
     ctx->world = world;
-    if (world == 1) return LDA_OK;
-    if (!uid) return fail(ctx, LDA_EINVAL, "null nccl unique id");
-    CU(cudaSetDevice(ctx->device));
-    ncclUniqueId id;
-    std::memcpy(&id, uid, sizeof(id));
-    NC(CommInitRank(&ctx->comm, world, id, rank));
+    return LDA_OK;
+}
+
+int lda_peer_group_create(int32_t world, lda_peer_group **out) {
+    if (!out) return LDA_EINVAL;
+    *out = nullptr;
+    if (world < 1 || world > lda::kMaxPeers) return LDA_EINVAL;
+    lda_peer_group *h = new (std::nothrow) lda_peer_group();
+    if (!h) return LDA_ENOMEM;
+    h->g = std::make_shared<lda::PeerGroup>(world);
+    *out = h;
+    return LDA_OK;
+}
+
+void lda_peer_group_destroy(lda_peer_group *g) { delete g; }
+
+int lda_init_peer(lda_ctx *ctx, lda_peer_group *g, int32_t rank) {
+    PRECHECK(ctx);
+    if (ctx->loaded || ctx->comm) return fail(ctx, LDA_ESTATE, "lda_init_peer must precede lda_load_corpus");
+    if (!g || !g->g) return fail(ctx, LDA_EINVAL, "null peer group");
+    std::string err;
+    int r = lda::make_peer_comm(g->g, rank, ctx->device, ctx->comm, err);
+    if (r != LDA_OK) return fail(ctx, r, err);
+    ctx->rank = rank;
+    ctx->world = g->g->world();
     return LDA_OK;
 }
 
@@ -345,12 +334,17 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     lda::tmark(nullptr);
     // one pass over the words: validation + the local word histogram
     std::vector<int64_t> local(ctx->V, 0);
-    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, local.data());
+    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, local.data(), ctx->threads);
     lda::tmark("validate + word histogram");
     if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
-    if (ctx->K > 16384)
-        return fail(ctx, LDA_ERANGE, "K > 16384 is not supported by this build's shared-memory layout");
     const int64_t Tg = doc_ptr[Dg];
+    // θ row storage: 128-byte aligned rows of min(L_d, K) + 1 words, in
+    // 32-byte units (the layout's row_off32; checked against H.rows32 after
+    // the layout).  Its range is checked here, before any allocation.
+    uint64_t r32 = 4;
+    for (int64_t d = 0; d < Dg; ++d)
+        r32 += 4 * static_cast<uint64_t>((std::min<int64_t>(doc_ptr[d + 1] - doc_ptr[d], ctx->K) + 1 + 31) / 32);
+    if (r32 >= (uint64_t(1) << 32) - 60) return fail(ctx, LDA_ERANGE, "θ row storage exceeds 2^32 x 32 bytes");
     const int32_t V = ctx->V, K = ctx->K;
 
     CU(cudaSetDevice(ctx->device));
@@ -365,8 +359,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         DA(d_all, all.size());
         CU(cudaMemcpyAsync(d_all + static_cast<size_t>(ctx->rank) * V, local.data(), sizeof(int64_t) * V,
                            cudaMemcpyHostToDevice, ctx->stream));
-        NC(AllGather(d_all + static_cast<size_t>(ctx->rank) * V, d_all, V, ncclInt64, ctx->comm,
-                         ctx->stream));
+        COMM(allgather_i64(d_all + static_cast<size_t>(ctx->rank) * V, d_all, V, ctx->stream, e_));
         CU(cudaMemcpyAsync(all.data(), d_all, sizeof(int64_t) * all.size(), cudaMemcpyDeviceToHost, ctx->stream));
         CU(cudaStreamSynchronize(ctx->stream));
     } else {
@@ -380,7 +373,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     lda::DevState &S = ctx->S;
     S.K = K;
     S.exclude_self = ctx->exclude_self;
-    S.filter32 = ctx->filter32;
     S.sampler = ctx->sampler;
     S.certify_slack = static_cast<double>(ctx->certify_slack);
     S.tile_fused = ctx->fused_recount != 0;
@@ -390,6 +382,24 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // the per-token tables go to the device tile by tile, copied by a helper
     // thread while the host prepares the next tile
     const bool tile_layout = S.sweep_tile || S.sweep_tile_cta;
+    // the tile samplers' line tables flag a row's first line in bit 31
+    if (tile_layout && r32 >= (uint64_t(1) << 31) - 60)
+        return fail(ctx, LDA_ERANGE,
+                    "θ row storage exceeds 2^31 x 32 bytes (64 GB) on one rank: use more ranks or sampler 0");
+    // tiles (Alg. 1 WorkSchedule1's resident shard, sampled tile by tile):
+    // auto = tiles whose θ rows fill about half the L2, so that a tile's rows
+    // are read from HBM about once per sweep
+    int64_t tile_tokens = ctx->tile_tokens;
+    if (tile_tokens < 0) {
+        int l2 = 0;
+        CU(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, ctx->device));
+        const double target = 0.5 * static_cast<double>(l2 > 0 ? l2 : (126 << 20));
+        const double row_bytes = 32.0 * static_cast<double>(r32);
+        tile_tokens = row_bytes <= target ? 0
+                                          : std::max<int64_t>(int64_t(1) << 20,
+                                                              static_cast<int64_t>(Tg * (target / row_bytes)));
+    }
+    ctx->tile_tokens_used = tile_tokens;
     lda::tmark("histogram, streams, configure");
     // The device buffers are allocated by the copier thread below while the
     // host builds the layout (cudaMalloc of ~10 GB takes ~0.3-0.5 s, all of
@@ -399,14 +409,14 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     for (uint32_t **t : {&S.tok_row, &S.doc_map, tile_layout ? nullptr : &S.tok_crank})
         if (t) pre.push_back({reinterpret_cast<void **>(t), sizeof(uint32_t) * Tg});
     pre.push_back({reinterpret_cast<void **>(&S.tok_z), sizeof(uint16_t) * Tg});
-    if (ctx->theta_mode == 1) pre.push_back({reinterpret_cast<void **>(&S.z_doc), sizeof(uint16_t) * (Tg + 4)});
+    pre.push_back({reinterpret_cast<void **>(&S.z_doc), sizeof(uint16_t) * (Tg + 8)});
     const size_t nwk_bytes = sizeof(int32_t) * (static_cast<size_t>(V) * K + K);
     pre.push_back({reinterpret_cast<void **>(&S.nwk), nwk_bytes});
     if (S.sweep_fused) pre.push_back({reinterpret_cast<void **>(&S.nwk_alt), nwk_bytes});
     if (tile_layout) pre.push_back({reinterpret_cast<void **>(&S.wtab), S.wt_bytes * static_cast<size_t>(V)});
     std::vector<void *> pre_done;
     size_t pre_fail_bytes = 0;
-    uint64_t pre_rows32 = 0;
+    const uint64_t pre_rows32 = r32;
     struct Job {
         uint64_t p0, p1, t0, t1;
     };
@@ -419,12 +429,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         cudaSetDevice(ctx->device);
         cudaStream_t cs = nullptr;
         cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
-        // the θ rows: 128-byte aligned rows of min(L_d, K) + 1 words (the
-        // layout's row_off32; checked against H.rows32 after the layout)
-        uint64_t r32 = 4;
-        for (int64_t d = 0; d < Dg; ++d)
-            r32 += 4 * static_cast<uint64_t>((std::min<int64_t>(doc_ptr[d + 1] - doc_ptr[d], K) + 1 + 31) / 32);
-        pre_rows32 = r32;
         pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
         for (auto &pa : pre) {
             if (copy_err != cudaSuccess) break;
@@ -471,9 +475,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // grow with K (tiles and the tail threshold scaled by K/1024; measured at
     // K = 8192 on the NYTimes shape: 1.94 -> 2.4 G tokens/s)
     const int64_t kscale = S.sweep_tile_cta ? std::max<int64_t>(1, K / 1024) : 1;
-    std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), ctx->tile_tokens * kscale,
+    std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), tile_tokens * kscale,
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
-                                      tile_layout ? 2 : (S.sweep_quad ? 1 : 0),
+                                      tile_layout ? 2 : 0,
                                       ctx->tail_per_tile * kscale, H,
                                       on_final, local.data(), /*host_tok_row=*/!tile_layout);
     {
@@ -483,6 +487,11 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     cv.notify_one();
     copier.join();
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
+    // a range error of the layout takes precedence over an allocation error
+    if (!e.empty()) {
+        cudaGetLastError();
+        return fail(ctx, LDA_ERANGE, e);
+    }
     if (copy_err != cudaSuccess) {
         cudaGetLastError();
         return fail(ctx, copy_err == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
@@ -490,7 +499,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                          " B): " + cudaGetErrorString(copy_err)
                                    : std::string("token table copy: ") + cudaGetErrorString(copy_err));
     }
-    if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
     if (pre_rows32 != H.rows32) return fail(ctx, LDA_ECUDA, "internal: θ row storage size mismatch");
     lda::tmark("layout done, token tables on the device");
 
@@ -512,11 +520,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     DA(S.rchunks, H.rchunks.size());
     S.n_split = static_cast<int64_t>(H.split_words.size());
     DA(S.split_words, H.split_words.size());
-    S.n_pchunks = static_cast<int64_t>(H.pchunks.size());
-    if (S.sweep_quad) {
-        DA(S.pchunks, H.pchunks.size());
-        DA(S.pairs, H.pairs.size());
-    }
     S.n_titems = static_cast<int64_t>(H.titems.size());
     if (S.sweep_tile || S.sweep_tile_cta) {
         DA(S.titems, H.titems.size());
@@ -542,10 +545,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(h2d(S.rchunks, H.rchunks.data(), sizeof(lda::RecountChunk) * H.rchunks.size()));
     CU(h2d(S.split_words, H.split_words.data(), sizeof(int32_t) * H.split_words.size()));
     CU(h2d(S.zero_words, H.zero_words.data(), sizeof(int32_t) * H.zero_words.size()));
-    if (S.sweep_quad) {
-        CU(h2d(S.pchunks, H.pchunks.data(), sizeof(lda::PairChunk) * H.pchunks.size()));
-        CU(h2d(S.pairs, H.pairs.data(), sizeof(lda::PairRec) * H.pairs.size()));
-    }
     if (S.sweep_tile || S.sweep_tile_cta) {
         CU(h2d(S.titems, H.titems.data(), sizeof(lda::TileItem) * H.titems.size()));
         CU(h2d(S.cbase, cbase.data(), sizeof(uint64_t) * V));
@@ -566,7 +565,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // host copies no longer needed on the device side (doc_map kept for get_counts)
     H.tok_row.release();
     H.tok_crank.release();
-    std::vector<lda::PairRec>().swap(H.pairs);
     std::vector<lda::TileItem>().swap(H.titems);
     lda::tmark("free host copies");
     ctx->loaded = true;
@@ -576,6 +574,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     ctx->stats.global_tokens = ctx->T_global;
     ctx->stats.world = ctx->world;
     ctx->stats.n_sample_chunks = (S.sweep_tile || S.sweep_tile_cta) ? S.n_titems : S.n_chunks;
+    ctx->stats.tile_tokens = ctx->tile_tokens_used;
+    ctx->stats.n_tiles = S.ntiles;
+    ctx->stats.sampler = S.sweep_tile ? 2 : (S.sweep_tile_cta ? 3 : 0);
     ctx->stats.sum_nnz_doc = ctx->cur_nnz;
     return LDA_OK;
 }
@@ -597,8 +598,15 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
             ctx->d_stat_log = nullptr;
         }
         DA(ctx->d_stat_log, 2 * static_cast<size_t>(n));
+        if (ctx->d_ll_log) {
+            CU(cudaFree(ctx->d_ll_log));
+            ctx->allocs.erase(std::find(ctx->allocs.begin(), ctx->allocs.end(), static_cast<void *>(ctx->d_ll_log)));
+            ctx->d_ll_log = nullptr;
+        }
+        DA(ctx->d_ll_log, 2 * static_cast<size_t>(n));
         ctx->stat_log_cap = n;
     }
+    std::vector<int64_t> ll_at;  // sweeps after which the LL is logged
     int launches = 0;
     CU(cudaMemsetAsync(S.stat + 2, 0, sizeof(unsigned long long), ctx->stream));
     for (int32_t s = 0; s < n; ++s) {
@@ -610,19 +618,37 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         if (S.sweep_fused) std::swap(S.nwk, S.nwk_alt);  // the sampler wrote the next counts
         else KL(lda::launch_recount(S, ctx->stream, &launches));
         CU(cudaEventRecord(E[2], ctx->stream));
-        if (ctx->world > 1) {
-            // ϕ sync overlapped with the θ update (§6.2)
-            CU(cudaStreamWaitEvent(ctx->comm_stream, E[2], 0));
-            NC(AllReduce(S.nwk, S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ncclInt32, ncclSum,
-                             ctx->comm, ctx->comm_stream));
-            CU(cudaEventRecord(E[4], ctx->comm_stream));
-        }
+        // θ update (depends only on z) on the compute stream while ϕ is
+        // summed over the ranks on the comm stream (§6.2)
         KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches));
         CU(cudaEventRecord(E[3], ctx->stream));
-        if (ctx->world > 1) CU(cudaStreamWaitEvent(ctx->stream, E[4], 0));
+        if (ctx->world > 1) {
+            CU(cudaStreamWaitEvent(ctx->comm_stream, E[2], 0));
+            COMM(allreduce_i32(S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ctx->comm_stream, e_));
+            CU(cudaEventRecord(E[4], ctx->comm_stream));
+            CU(cudaStreamWaitEvent(ctx->stream, E[4], 0));
+        }
         CU(cudaEventRecord(E[5], ctx->stream));
+        if (ctx->loglik_every > 0 && t % static_cast<uint64_t>(ctx->loglik_every) == 0) {
+            // after the sweep's events: not part of its time (X23)
+            int ll_launches = 0;
+            KL(lda::launch_loglik(S, ctx->rank == 0, ctx->stream, &ll_launches));
+            if (ctx->world > 1) COMM(allreduce_f64(S.ll_out, 2, ctx->stream, e_));
+            CU(cudaMemcpyAsync(ctx->d_ll_log + 2 * ll_at.size(), S.ll_out, 2 * sizeof(double),
+                               cudaMemcpyDeviceToDevice, ctx->stream));
+            ll_at.push_back(static_cast<int64_t>(t));
+        }
     }
     CU(cudaStreamSynchronize(ctx->stream));
+    {
+        std::vector<double> hl(2 * ll_at.size());
+        if (!hl.empty())
+            CU(cudaMemcpy(hl.data(), ctx->d_ll_log, hl.size() * sizeof(double), cudaMemcpyDeviceToHost));
+        ctx->ll_sweep = ll_at;
+        ctx->ll_value.assign(ll_at.size(), 0.0);
+        for (size_t i = 0; i < ll_at.size(); ++i)
+            ctx->ll_value[i] = (hl[2 * i] + hl[2 * i + 1]) / static_cast<double>(ctx->T_global > 0 ? ctx->T_global : 1);
+    }
     unsigned long long n_exact = 0;
     CU(cudaMemcpy(&n_exact, S.stat + 2, sizeof(n_exact), cudaMemcpyDeviceToHost));
     ctx->stats.n_exact_redraws = static_cast<int64_t>(n_exact);
@@ -683,6 +709,27 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     }
     st.sum_nnz_doc = ctx->cur_nnz;
     st.n_launches = launches;
+    // SURVEY §8(d) byte model of the last sweep (this rank): B_alg and the
+    // sampling kernel's share B_sample
+    if (n > 0) {
+        const double Tg = static_cast<double>(S.T), VK = static_cast<double>(S.V) * S.K;
+        const double ntok = static_cast<double>(st.sum_nnz_tok);
+        st.bytes_alg = 20.0 * Tg + 4.0 * ntok + 8.0 * VK + 4.0 * static_cast<double>(st.sum_nnz_doc) +
+                       8.0 * static_cast<double>(S.D);
+        st.bytes_sample = 14.0 * Tg + 4.0 * ntok + 4.0 * VK;
+    }
+    return LDA_OK;
+}
+
+int lda_get_loglik_log(lda_ctx *ctx, int32_t cap, int64_t *sweep, double *ll_per_token, int32_t *n_out) {
+    PRECHECK(ctx);
+    const int32_t n = static_cast<int32_t>(ctx->ll_sweep.size());
+    if (n_out) *n_out = n;
+    const int32_t m = std::min(n, std::max(cap, 0));
+    for (int32_t i = 0; i < m; ++i) {
+        if (sweep) sweep[i] = ctx->ll_sweep[i];
+        if (ll_per_token) ll_per_token[i] = ctx->ll_value[i];
+    }
     return LDA_OK;
 }
 
@@ -712,8 +759,7 @@ int lda_loglik(lda_ctx *ctx, double *ll) {
     CU(cudaSetDevice(ctx->device));
     int launches = 0;
     KL(lda::launch_loglik(ctx->S, ctx->rank == 0, ctx->stream, &launches));
-    if (ctx->world > 1)
-        NC(AllReduce(ctx->S.ll_out, ctx->S.ll_out, 2, ncclFloat64, ncclSum, ctx->comm, ctx->stream));
+    if (ctx->world > 1) COMM(allreduce_f64(ctx->S.ll_out, 2, ctx->stream, e_));
     double h[2];
     CU(cudaMemcpyAsync(h, ctx->S.ll_out, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
     CU(cudaStreamSynchronize(ctx->stream));
@@ -816,7 +862,7 @@ void lda_destroy(lda_ctx *ctx) {
         if (ctx->stream) cudaStreamDestroy(ctx->stream);
         if (ctx->comm_stream) cudaStreamDestroy(ctx->comm_stream);
     }
-    if (ctx->comm && nccl().ok) nccl().CommDestroy(ctx->comm);
+    ctx->comm.reset();
     delete ctx;
 }
 
@@ -832,10 +878,10 @@ int lda_layout_selfcheck(int64_t D, int32_t V, int32_t K, const int64_t *doc_ptr
         }
         return static_cast<int>(LDA_EINVAL);
     };
-    if (D < 0 || V < 1 || K < 1 || !doc_ptr || sampler < 0 || sampler > 3 || chunk_tokens < 1)
+    if (D < 0 || V < 1 || K < 1 || !doc_ptr || sampler < 0 || sampler > 3 || sampler == 1 || chunk_tokens < 1)
         return bad("invalid arguments");
     bool range_err = false;
-    std::string v = lda::validate_corpus(doc_ptr, words, D, V, &range_err);
+    std::string v = lda::validate_corpus(doc_ptr, words, D, V, &range_err, nullptr, 0);
     if (!v.empty()) return bad(v);
     const int64_t T = doc_ptr[D];
     std::vector<int64_t> cbase(V, 0), wc(V, 0);

@@ -92,7 +92,7 @@ void word_histogram(const int32_t *words, int64_t T, int32_t V, int nthreads, in
 }
 
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
-                            bool *range_error, int64_t *word_counts) {
+                            bool *range_error, int64_t *word_counts, int nthreads) {
     *range_error = false;
     if (D < 0) return "negative document count";
     if (!doc_ptr) return "doc_ptr is NULL";
@@ -112,7 +112,7 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
         return "more than 2^32-1 tokens on one rank";
     }
     if (T > 0 && !words) return "words is NULL";
-    int nth = host_threads(0);
+    int nth = host_threads(nthreads);
     std::vector<int64_t> bad(nth, -1);
     // with word_counts: the same pass counts the tokens of every word
     const int nparts = T < (1 << 16) ? 1 : nth;
@@ -147,7 +147,6 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int sampler, int64_t tail_per_tile, HostLayout &L,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final,
                          const int64_t *word_counts, bool host_tok_row) {
-    const bool build_pairs = sampler == 1;
     const int64_t T = doc_ptr[D];
     L.D = D;
     L.T = T;
@@ -156,7 +155,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     nthreads = host_threads(nthreads);
 
     // θ rows: 1 header word (nnz) + capacity min(L_d, K) entries, rounded up
-    // to whole 128-byte lines (the quad sampler reads a row line by line);
+    // to whole 128-byte lines (the tile samplers read a row line by line);
     // words past nnz are kept zero (zero-mass padding the sampler reads
     // without a bounds check).  Offsets are in 32-byte units.
     L.doc_ptr32.resize(D + 1);
@@ -214,7 +213,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 
     // Tile samplers: documents keep their order inside each tile part, so a
     // word's run holds its tokens in canonical order and a token's rank is
-    // its item's base + offset (no per-token rank table).  Samplers 0 / 1:
+    // its item's base + offset (no per-token rank table).  Sampler 0:
     // documents by decreasing length inside a part (similar θ row lengths in
     // a warp), ranks stored per token.
     const bool tile_layout = sampler == 2;
@@ -449,7 +448,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // canonical index continues word w's run on this rank (cbase[w] + v).
     L.chunks.clear();
     L.zero_words.clear();
-    if (sampler != 2) {  // samplers 0 / 1 only (the tile samplers use their own items)
+    if (sampler != 2) {  // sampler 0 only (the tile samplers use their own items)
         for (int32_t w = 0; w < V; ++w) {
             const int64_t n = L.word_count[w];
             const int64_t pieces = (n + chunk_tokens - 1) / chunk_tokens;
@@ -473,73 +472,6 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     }
 
     tmark("layout: runs + sampler chunks");
-    // Quad-sampler items: the same word chunks, their tokens (virtual order:
-    // tile by tile, documents by decreasing length) grouped into runs of
-    // equal θ row = (word, doc) pairs of at most 255 tokens.
-    L.pchunks.clear();
-    L.pairs.clear();
-    if (build_pairs) {
-        std::vector<uint16_t> row_cl(L.rows32, 0);  // θ row offset -> capacity in 128-byte lines
-        for (int64_t d = 0; d < D; ++d) {
-            const uint64_t end = d + 1 < D ? L.row_off32[d + 1] : off32;
-            row_cl[L.row_off32[d]] = static_cast<uint16_t>((end - L.row_off32[d]) / 4);
-        }
-        const int64_t nc = static_cast<int64_t>(L.chunks.size());
-        // visit the positions of chunk c in virtual order: f(position)
-        auto walk = [&](const SampleChunk &c, auto &&f) {
-            uint32_t s = c.seg0;
-            for (uint32_t v = c.vbegin; v < c.vbegin + c.count; ++v) {
-                while (L.segs[s + 1].vstart <= v) ++s;
-                f(L.segs[s].pos + (v - L.segs[s].vstart));
-            }
-        };
-        std::vector<uint32_t> np(nc + 1, 0);
-        parallel_for(nthreads, nc, [&](int, int64_t b, int64_t e) {
-            for (int64_t ci = b; ci < e; ++ci) {
-                uint32_t n = 0, prev_row = 0xFFFFFFFFu, m = 0;
-                walk(L.chunks[ci], [&](uint32_t p) {
-                    if (L.tok_row[p] != prev_row || m == 255) {
-                        ++n;
-                        prev_row = L.tok_row[p];
-                        m = 0;
-                    }
-                    ++m;
-                });
-                np[ci + 1] = n;
-            }
-        });
-        for (int64_t ci = 0; ci < nc; ++ci) np[ci + 1] += np[ci];
-        if (np[nc] >= (uint64_t(1) << 32) - 1) return "too many (word, doc) pairs";
-        L.pairs.resize(np[nc]);
-        L.pchunks.resize(nc);
-        parallel_for(nthreads, nc, [&](int, int64_t b, int64_t e) {
-            for (int64_t ci = b; ci < e; ++ci) {
-                const SampleChunk &c = L.chunks[ci];
-                PairRec *out = L.pairs.data() + np[ci];
-                int64_t n = -1;
-                walk(c, [&](uint32_t p) {
-                    const uint32_t row = L.tok_row[p];
-                    if (n < 0 || out[n].row != row || (out[n].mcl & 0xFFu) == 255u) {
-                        ++n;
-                        out[n].row = row;
-                        out[n].crank = L.tok_crank[p];
-                        out[n].pos = p;
-                        out[n].mcl = static_cast<uint32_t>(row_cl[row]) << 8;
-                    }
-                    out[n].mcl += 1;
-                });
-                PairChunk &q = L.pchunks[ci];
-                q.word = c.word;
-                q.pbegin = np[ci];
-                q.npairs = np[ci + 1] - np[ci];
-                q.ntok = c.count;
-                q.split = c.pad & 1u;
-                q.pad = 0;
-                q.c_base = c.c_base;
-            }
-        });
-    }
-
     // Recount work items: per word, pieces of at most recount_tokens.
     L.rchunks.clear();
     L.split_words.clear();
@@ -561,7 +493,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     }
     std::stable_sort(L.rchunks.begin(), L.rchunks.end(),
                      [](const RecountChunk &a, const RecountChunk &b) { return a.vcount > b.vcount; });
-    tmark("layout: pairs + recount chunks");
+    tmark("layout: recount chunks");
     return "";
 }
 

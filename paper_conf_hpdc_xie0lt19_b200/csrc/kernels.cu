@@ -20,6 +20,7 @@
 
 #include <algorithm>
 #include <cstdint>
+#include <cstring>
 
 #include "lda_internal.h"
 
@@ -34,9 +35,6 @@ constexpr int kSweepThreads = 256;
 constexpr int kMaxBlk = 16;  // block-end prefixes kept per token for the sparse rescan
 #ifndef LDA_RING
 #define LDA_RING 3
-#endif
-#ifndef LDA_MATCH
-#define LDA_MATCH 0
 #endif
 #ifndef LDA_FUSE
 #define LDA_FUSE 1
@@ -219,80 +217,10 @@ struct Mass {
     }
 };
 
-// The exact (fp64) draw of one token, as the fp64 walk in sweep_kernel
-// computes it, by linear scans: fallback of the fp32 filter for tokens whose
-// uniform lies within the filter's error bound of a CDF boundary.
-__device__ __noinline__ int draw_exact(const uint32_t *rw, uint32_t len, const double *pstar, const double *P,
-                                       double Q, int K, uint32_t x0) {
-    const uint32_t nblk = (len + 8u) >> 3;
-    double S = 0.0;
-    for (uint32_t b = 0; b < nblk; ++b) {
-        const Blk8 u = ld_nc_v8(rw + 8 * b);
-        for (int e = (b == 0 ? 1 : 0); e < 8; ++e)
-            S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], S);
-    }
-    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
-    if (x < S) {
-        double C = 0.0;
-        for (uint32_t b = 0; b < nblk; ++b) {
-            const Blk8 u = ld_nc_v8(rw + 8 * b);
-            for (int e = (b == 0 ? 1 : 0); e < 8; ++e) {
-                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], C);
-                if (C > x) return static_cast<int>(u.w[e] >> kTS);
-            }
-        }
-        return K - 1;
-    }
-    int lo = 0, hi = K - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (S + P[mid] > x) hi = mid;
-        else lo = mid + 1;
-    }
-    return lo;
-}
-
-// The same exact walk, inlined (ptxas 12.9 crashes on a call to the
-// __noinline__ version from sweep_quad_kernel).
-__device__ __forceinline__ int draw_exact_inl(const uint32_t *rw, uint32_t len, const double *pstar,
-                                              const double *P, double Q, int K, uint32_t x0) {
-    const uint32_t nblk = (len + 8u) >> 3;
-    double S = 0.0;
-    for (uint32_t b = 0; b < nblk; ++b) {
-        Blk8 u = ld_nc_v8(rw + 8 * b);
-        if (b == 0u) u.w[0] = 0u;  // header word: zero mass
-#pragma unroll
-        for (int e = 0; e < 8; ++e) S = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], S);
-    }
-    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
-    if (x < S) {
-        double C = 0.0;
-        int z = -1;
-        for (uint32_t b = 0; z < 0 && b < nblk; ++b) {
-            Blk8 u = ld_nc_v8(rw + 8 * b);
-            if (b == 0u) u.w[0] = 0u;
-#pragma unroll
-            for (int e = 0; e < 8; ++e) {
-                C = fma(static_cast<double>(u.w[e] & 0xFFFFu), pstar[u.w[e] >> kTS], C);
-                if (z < 0 && C > x) z = static_cast<int>(u.w[e] >> kTS);
-            }
-        }
-        return z < 0 ? K - 1 : z;
-    }
-    int lo = 0, hi = K - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi) >> 1;
-        if (S + P[mid] > x) hi = mid;
-        else lo = mid + 1;
-    }
-    return lo;
-}
-
 // SMEMP: p*/P in shared memory (LDS addressing); else in a global scratch
 // slice per CTA (large K).
-template <bool EXCL, bool SMEMP, bool F32>
+template <bool EXCL, bool SMEMP>
 __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(SweepArgs a) {
-    static_assert(!F32 || (SMEMP && !EXCL), "the fp32 filter needs p* in smem and exclude_self = 0");
     extern __shared__ double smem_d[];
     __shared__ int s_ci;
     __shared__ double s_wtot[kSweepThreads / 32];
@@ -303,9 +231,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
     double *blkC = smem_d;
     double *pstar = SMEMP ? smem_d + kMaxBlk * kSweepThreads : a.gscratch + static_cast<size_t>(blockIdx.x) * 2 * K;
     double *P = pstar + K;
-    float *p32 = reinterpret_cast<float *>(smem_d + kMaxBlk * kSweepThreads + 2 * K);  // fp32 copy of p*
-    float *blk32 = reinterpret_cast<float *>(blkC);
-    int *hist = reinterpret_cast<int *>(p32 + K);
+    int *hist = reinterpret_cast<int *>(smem_d + kMaxBlk * kSweepThreads + 2 * K);
     int *nkp = hist + K;
     if (SMEMP) {
         for (int k = tid; k < 2 * K; k += kSweepThreads) hist[k] = 0;
@@ -330,7 +256,6 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                 if (k < K) {
                     const double ps = (static_cast<double>(__ldg(nwk_row + k)) + a.beta) / __ldg(a.denom + k);
                     pstar[k] = ps;
-                    if (SMEMP) p32[k] = static_cast<float>(ps);
                     run = run + a.alpha * ps;
                     P[k] = run;
                 }
@@ -356,7 +281,6 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
             cur_word = static_cast<int>(ch.word);
         }
         const double Q = P[K - 1];
-        const float Q32 = static_cast<float>(Q);
 
         // One sampler per lane; each thread draws tokens j, j+256, ...  The
         // row is streamed in 32-byte blocks (one 256-bit load per block per
@@ -392,74 +316,6 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
             for (int i = 1; i < kRing; ++i)
                 if (static_cast<uint32_t>(i) < nblk) q[i] = ld_nc_v8(rw + 8 * i);
             int z;
-            if constexpr (F32) {
-                // fp32 filter (see draw_exact): the same walk in single
-                // precision plus a bound on its distance to the fp64 walk
-                float S = 0.0f;
-#pragma unroll
-                for (int e = 1; e < 8; ++e) S = fmaf(static_cast<float>(q[0].w[e] & 0xFFFFu), p32[q[0].w[e] >> kTS], S);
-                blk32[tid] = S;
-                if (static_cast<uint32_t>(kRing) < nblk) q[0] = ld_nc_v8(rw + 8 * kRing);
-                for (uint32_t base = 0; base < nblk; base += kRing) {
-#pragma unroll
-                    for (int i = 0; i < kRing; ++i) {
-                        const uint32_t b = base + i;
-                        if (b == 0) continue;
-                        if (b >= nblk) break;
-                        const Blk8 u = q[i];
-                        const uint32_t nx = b + kRing;
-                        if (nx < nblk) q[i] = ld_nc_v8(rw + 8 * nx);
-#pragma unroll
-                        for (int e = 0; e < 8; ++e)
-                            S = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> kTS], S);
-                        if (b < kMaxBlk) blk32[b * kSweepThreads + tid] = S;
-                    }
-                }
-                const float tot = S + Q32;
-                const float xf = __uint2float_rn(x0) * 2.3283064365386962890625e-10f * tot;
-                // |(C32 - x32) - (C64 - x64)| <= (2·nnz + 6)·2^-24·total (first order)
-                const float B = (2.0f * static_cast<float>(len) + 8.0f) * 6.0e-8f * tot;
-                bool ok = fabsf(xf - S) > B;
-                z = -1;
-                if (ok) {
-                    if (xf < S) {
-                        const uint32_t nb = nblk < kMaxBlk ? nblk : kMaxBlk;
-                        uint32_t b = 0;
-                        for (; b < nb; ++b) {
-                            const float d = blk32[b * kSweepThreads + tid] - xf;
-                            if (fabsf(d) <= B) { ok = false; break; }
-                            if (d > 0.0f) break;
-                        }
-                        float C = b == 0 ? 0.0f : blk32[(b - 1) * kSweepThreads + tid];
-                        for (; ok && z < 0 && b < nblk; ++b) {  // one block, or a linear tail past kMaxBlk
-                            const Blk8 u = ld_nc_v8(rw + 8 * b);
-#pragma unroll
-                            for (int e = 0; e < 8; ++e) {
-                                if (b == 0 && e == 0) continue;
-                                C = fmaf(static_cast<float>(u.w[e] & 0xFFFFu), p32[u.w[e] >> kTS], C);
-                                const float d = C - xf;
-                                if (z < 0 && ok) {
-                                    if (fabsf(d) <= B) ok = false;
-                                    else if (d > 0.0f) z = static_cast<int>(u.w[e] >> kTS);
-                                }
-                            }
-                        }
-                        if (z < 0) ok = false;
-                    } else {
-                        const double Sd = S, xd = xf, Bd = B;
-                        int lo = 0, hi = K - 1;
-                        while (lo < hi) {
-                            const int mid = (lo + hi) >> 1;
-                            const double d = (Sd + P[mid]) - xd;
-                            if (fabs(d) <= Bd) { ok = false; break; }
-                            if (d > 0.0) hi = mid;
-                            else lo = mid + 1;
-                        }
-                        z = lo;
-                    }
-                }
-                if (!ok) z = draw_exact(rw, len, pstar, P, Q, K, x0);
-            } else {
             // pass 1: S over the row, block-end prefixes to smem
             double S = 0.0;
 #pragma unroll
@@ -516,17 +372,8 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                 }
                 z = lo;  // K-1 also when x >= S + Q by rounding (X6 fallback)
             }
-            }
             a.z[p] = static_cast<uint16_t>(z);
-            if (SMEMP) {
-#if LDA_MATCH
-                // one shared atomic per distinct topic among the active lanes
-                const unsigned peers = __match_any_sync(__activemask(), z);
-                if (lane == __ffs(peers) - 1) atomicAdd(&hist[z], __popc(peers));
-#else
-                atomicAdd(&hist[z], 1);
-#endif
-            }
+            if (SMEMP) atomicAdd(&hist[z], 1);
         }
         __syncthreads();
         if (SMEMP) {
@@ -554,111 +401,6 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
     }
 }
 
-// ---------------------------------------------------------------------------
-// a3 + a4, quad sampler (the default path).
-//
-// Same chunk queue, p*/P prefix and fused recount as sweep_kernel; the
-// tokens of a chunk come as (word, doc) pairs (PairRec): consecutive tokens
-// of the word in one document share the document's θ row, hence S and the
-// sparse prefix of Eq. 6-7 -- one row walk per pair, one draw per token.
-// A warp takes 32 pairs at a time:
-//   H  (lane per pair)  the row header (nnz) of each pair -> its line count.
-//   A  (quad per pair)  four lanes read one 128-byte line of a θ row per
-//      step (lane `sub` holds entries 8·sub .. 8·sub+7 of the line: one
-//      256-bit load each, one L1 wavefront per line instead of one per
-//      32-byte block), each sums its 8 masses n_dk·p*(k) in fp32 from a
-//      4-byte p* table (half the shared-memory bank conflicts of the fp64
-//      table), a quad scan gives the prefix at every 8-entry block end
-//      (kept for kQBlk blocks) and the pair's S.  A register ring of R lines
-//      per lane runs ahead across the quad's four pairs.
-//   B  (lane per pair)  Philox uniform of each of the pair's m tokens,
-//      x = U·(S+Q) in fp64; sparse: binary search of the block-end prefixes
-//      and the sequential rescan of that block (first C > x, X5/X6); dense:
-//      binary search of S + P[k] (P exact fp64).  Every comparison is made
-//      only if it clears the fp32 error bound 2ε; a token with any closer
-//      comparison is redrawn by the exact fp64 walk in the oracle's order
-//      (draw_exact), so the filter never changes a draw except within
-//      fp64 rounding of a boundary (excused within 1e-6).
-//   z store + shared histogram (ϕ recount, fused as in sweep_kernel).
-// ---------------------------------------------------------------------------
-constexpr int kQBlk = 16;            // block-end prefixes kept per pair (blocks of 8 entries)
-constexpr int kQStride = kQBlk + 1;  // odd stride (words): lane-per-pair reads hit distinct banks
-constexpr int kQWarpWords = 32 * 4 + 32 + 32 + 32 * kQStride;  // per warp: recs, S, nnz, blk
-#ifndef LDA_QRING
-#define LDA_QRING 3
-#endif
-#ifndef LDA_QUAD_MINB
-#define LDA_QUAD_MINB 3
-#endif
-#ifndef LDA_QDEBUG
-#define LDA_QDEBUG 0
-#endif
-#if LDA_QDEBUG
-__device__ unsigned long long g_qdbg[8];
-#define QDBG(i) atomicAdd(&g_qdbg[i], 1ull)
-#else
-#define QDBG(i)
-#endif
-
-struct QuadArgs {
-    const PairChunk *chunks;
-    int64_t n_chunks;
-    const uint4 *pairs;
-    uint16_t *z;
-    const uint32_t *rows;
-    const int32_t *nwk;
-    const double *denom;
-    uint32_t *counter;
-    int32_t *nwk_next;
-    int32_t *nk_next;
-    unsigned long long *n_exact;  // tokens redrawn by the exact fp64 walk (statistics)
-    int K;
-    double alpha, beta;
-    uint32_t t;
-    uint32_t key0[10], key1[10];
-};
-
-// p*(k) = (n_wk + β)/(n_k + Vβ) (fp64, and its fp32 rounding p32) and the
-// inclusive prefix P of α·p*(k) in smem (Eq. 8); all threads of the CTA call
-// it; ends with a barrier.
-__device__ __forceinline__ void build_word_prefix(const int32_t *__restrict__ nwk_row,
-                                                  const double *__restrict__ denom, int K, double alpha,
-                                                  double beta, double *pstar, double *P, float *p32,
-                                                  double *s_wtot) {
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int E = (K + kSweepThreads - 1) / kSweepThreads;
-    const int kb = tid * E;
-    double run = 0.0;
-    for (int e = 0; e < E; ++e) {
-        const int k = kb + e;
-        if (k < K) {
-            const double ps = (static_cast<double>(__ldg(nwk_row + k)) + beta) / __ldg(denom + k);
-            pstar[k] = ps;
-            p32[k] = static_cast<float>(ps);
-            run = run + alpha * ps;
-            P[k] = run;
-        }
-    }
-    double incl = run;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const double y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
-    }
-    double lex = __shfl_up_sync(kFull, incl, 1);
-    if (lane == 0) lex = 0.0;
-    if (lane == 31) s_wtot[warp] = incl;
-    __syncthreads();
-    double off = 0.0;
-    for (int i = 0; i < warp; ++i) off += s_wtot[i];
-    off = off + lex;
-    for (int e = 0; e < E; ++e) {
-        const int k = kb + e;
-        if (k < K) P[k] = off + P[k];
-    }
-    __syncthreads();
-}
-
 // count (low 16 bits of a θ entry) as float, exactly: bits 0x4B00:count = 2^23 + c
 __device__ __forceinline__ float count_f32(uint32_t e) {
     return __uint_as_float(__byte_perm(e, 0x4B00u, 0x5410)) - 8388608.0f;
@@ -669,241 +411,6 @@ __device__ __forceinline__ float tab32(const float *__restrict__ p32, uint32_t e
 }
 __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc) {
     return fmaf(count_f32(e), tab32(p32, e), acc);
-}
-
-template <int R>
-__global__ void __launch_bounds__(kSweepThreads, LDA_QUAD_MINB) sweep_quad_kernel(QuadArgs a) {
-    extern __shared__ double smem_d[];
-    __shared__ int s_ci;
-    __shared__ double s_wtot[kSweepThreads / 32];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int q = lane >> 2, sub = lane & 3;
-    const int K = a.K;
-    // smem: [p*: K f64][P: K f64][p32: K f32][hist: K i32][nk partial: K i32] (16-byte aligned end)
-    //       [per warp: recs uint4[32], S f32[32], nnz u32[32], blk f32[32][kQStride]]
-    double *pstar = smem_d;
-    double *P = pstar + K;
-    float *p32 = reinterpret_cast<float *>(P + K);
-    int *hist = reinterpret_cast<int *>(p32 + K);
-    int *nkp = hist + K;
-    uint32_t *wbase = reinterpret_cast<uint32_t *>(smem_d) + ((28 * K + 15) / 16) * 4 + warp * kQWarpWords;
-    uint4 *wR = reinterpret_cast<uint4 *>(wbase);
-    float *wS = reinterpret_cast<float *>(wbase + 128);
-    uint32_t *wN = wbase + 160;
-    float *wB = reinterpret_cast<float *>(wbase + 192);
-    for (int k = tid; k < 2 * K; k += kSweepThreads) hist[k] = 0;
-    int cur_word = -1;
-    unsigned n_exact = 0;
-
-    for (;;) {
-        if (tid == 0) s_ci = static_cast<int>(atomicAdd(a.counter, 1u));
-        __syncthreads();
-        const int ci = s_ci;
-        if (ci >= a.n_chunks) break;
-        const PairChunk ch = a.chunks[ci];
-        if (static_cast<int>(ch.word) != cur_word) {
-            build_word_prefix(a.nwk + static_cast<size_t>(ch.word) * K, a.denom, K, a.alpha, a.beta, pstar, P,
-                              p32, s_wtot);
-            cur_word = static_cast<int>(ch.word);
-        }
-        const double Q = P[K - 1];
-        const uint32_t nb = (ch.npairs + 31u) >> 5;
-
-        for (uint32_t b = static_cast<uint32_t>(warp); b < nb; b += kSweepThreads / 32) {
-            // ---- H: the batch's 32 pair records and their rows' nnz
-            const uint32_t pi = 32u * b + static_cast<uint32_t>(lane);
-            uint4 rec = make_uint4(0u, 0u, 0u, 0u);
-            uint32_t nnz = 0, nl = 0;
-            if (pi < ch.npairs) {
-                rec = ld_nc_v4(a.pairs + ch.pbegin + pi);
-                nnz = __ldg(a.rows + static_cast<size_t>(rec.x) * 8);
-                nl = (nnz + 32u) >> 5;  // 128-byte lines holding words 0..nnz
-            }
-            wR[lane] = rec;
-            wN[lane] = nnz;
-            const uint32_t lines = nl + __shfl_down_sync(kFull, nl, 8) + __shfl_down_sync(kFull, nl, 16) +
-                                   __shfl_down_sync(kFull, nl, 24);
-            const int nsteps = static_cast<int>(__reduce_max_sync(kFull, lane < 8 ? lines : 0u));
-            __syncwarp();
-
-            // ---- A: stream the quad's lines (pair r, line i) through a ring;
-            // pairs j = 8r + q; invalid pairs (nnz of an absent pair = 0 lines)
-            // only at the end.  A lane loads its 32-byte block only if the
-            // block holds a word <= nnz (words past nnz are zero).
-            int ir = 0;
-            uint32_t ii = 0, rwI = wR[q].x, nzI = wN[q], nlI = (pi - lane + q < ch.npairs) ? (nzI + 32u) >> 5 : 0u;
-            if (nlI == 0u) ir = 4;
-            Blk8 ring[R];
-#define LDA_QISSUE(slot)                                                                                  \
-    if (ir < 4) {                                                                                         \
-        if (32u * ii + 8u * sub <= nzI)                                                                   \
-            ring[slot] = ld_nc_v8(a.rows + (static_cast<size_t>(rwI) + 4u * ii + sub) * 8);              \
-        if (++ii >= nlI) {                                                                                \
-            ii = 0;                                                                                       \
-            if (++ir < 4) {                                                                               \
-                const uint32_t jn = 8u * ir + q;                                                          \
-                rwI = wR[jn].x;                                                                           \
-                nzI = wN[jn];                                                                             \
-                nlI = (pi - lane + jn < ch.npairs) ? (nzI + 32u) >> 5 : 0u;                              \
-                if (nlI == 0u) ir = 4;                                                                    \
-            }                                                                                             \
-        }                                                                                                 \
-    }
-#pragma unroll
-            for (int s2 = 0; s2 < R; ++s2) LDA_QISSUE(s2)
-            int cr = 0;
-            uint32_t ci2 = 0, nzC = wN[q], nlC = (pi - lane + q < ch.npairs) ? (nzC + 32u) >> 5 : 0u;
-            if (nlC == 0u) cr = 4;
-            float run = 0.0f;
-            for (int base = 0; base < nsteps; base += R) {
-#pragma unroll
-                for (int s2 = 0; s2 < R; ++s2) {
-                    if (base + s2 >= nsteps) break;
-                    Blk8 u = ring[s2];
-                    LDA_QISSUE(s2)
-                    const bool live = cr < 4;
-                    float sp = 0.0f;
-                    if (live && 32u * ci2 + 8u * sub <= nzC) {
-                        if (ci2 == 0u && sub == 0) u.w[0] = 0u;  // word 0 = nnz header, not an entry
-#pragma unroll
-                        for (int e = 0; e < 8; ++e) sp = entry_mass32(u.w[e], p32, sp);
-                    }
-                    float v = sp;
-                    float y = __shfl_up_sync(kFull, v, 1, 4);
-                    if (sub >= 1) v += y;
-                    y = __shfl_up_sync(kFull, v, 2, 4);
-                    if (sub >= 2) v += y;
-                    const float qt = __shfl_sync(kFull, v, 3, 4);
-                    if (live) {
-                        const int j = 8 * cr + q;
-                        const uint32_t bidx = 4u * ci2 + sub;
-                        if (bidx < static_cast<uint32_t>(kQBlk)) wB[j * kQStride + bidx] = run + v;
-                        run += qt;
-                        if (++ci2 >= nlC) {
-                            if (sub == 0) wS[j] = run;
-                            run = 0.0f;
-                            ci2 = 0;
-                            if (++cr < 4) {
-                                const uint32_t jn = 8u * cr + q;
-                                nzC = wN[jn];
-                                nlC = (pi - lane + jn < ch.npairs) ? (nzC + 32u) >> 5 : 0u;
-                                if (nlC == 0u) cr = 4;
-                            }
-                        }
-                    }
-                }
-            }
-#undef LDA_QISSUE
-            __syncwarp();
-
-            // ---- B: lane `lane` draws the m tokens of pair `lane`
-            const uint32_t m = rec.w & 0xFFu;
-            if (m) {
-                const double S = static_cast<double>(wS[lane]);  // fp32 S', exact in fp64
-                const double tot = S + Q;
-                // fp32 error bounds (first order, u = 2^-24), with nl lines:
-                //   prefix C' at a block end, after the rescan of a block:
-                //     |C' - C| <= (20 + nl)·u·C  (p32 rounding, 8 FFMA of a
-                //     lane block, 2 quad-scan and <= nl running additions,
-                //     8 rescan FFMA);  |S' - S| <= (12 + nl)·u·S
-                //   x = U·(S' + Q):  |x' - x| <= U·|S' - S|
-                //   y = x - S' (dense offset): |y' - y| <= (1 - U)·|S' - S|
-                // A decision is taken only with a margin above its bound
-                // (+ 2^-50·tot for the fp64 roundings); otherwise the token
-                // is redrawn by the exact fp64 walk.
-                const uint32_t nl = (nnz + 32u) >> 5;
-                const double es = static_cast<double>(12u + nl) * 5.9604644775390625e-08 * S;
-                const double ec = static_cast<double>(34u + 2u * nl) * 5.9604644775390625e-08;
-                const double er = 8.8817841970012523e-16 * tot;
-                const uint32_t nblk = (nnz + 8u) >> 3;  // 8-word blocks holding words 0..nnz
-                const int nbl = nblk < static_cast<uint32_t>(kQBlk) ? static_cast<int>(nblk) : kQBlk;
-                const uint32_t *rw = a.rows + static_cast<size_t>(rec.x) * 8;
-                const float *Bp = wB + lane * kQStride;
-                for (uint32_t k = 0; k < m; ++k) {
-                    const uint32_t x0 = philox_x0_sched(ch.c_base + rec.y + k, a.t, a.key0, a.key1);
-                    const double U = static_cast<double>(x0) * 2.3283064365386962890625e-10;
-                    const double x = U * tot;
-                    const double y = x - S;
-                    const double ed = (1.0 - U) * es + er;
-                    bool ok = fabs(y) > ed;
-                    QDBG(0);
-                    if (!ok) QDBG(1);
-                    int z = K - 1;
-                    if (ok && y < 0.0) {
-                        // sparse bucket: first stored block end > x, then the
-                        // sequential rescan of that block (past kQBlk: linear)
-                        const double ex = ec * x + er;
-                        int lo = 0, hi = nbl;
-                        while (lo < hi) {
-                            const int mid = (lo + hi) >> 1;
-                            const double c = static_cast<double>(Bp[mid]);
-                            const double d = c - x;
-                            if (fabs(d) <= ex + ec * c) { ok = false; QDBG(2); }
-                            if (d > 0.0) hi = mid;
-                            else lo = mid + 1;
-                        }
-                        float c32 = lo == 0 ? 0.0f : Bp[lo - 1];
-                        z = -1;
-                        for (uint32_t blk = static_cast<uint32_t>(lo); ok && z < 0 && blk < nblk; ++blk) {
-                            Blk8 u = ld_nc_v8(rw + 8 * blk);
-                            if (blk == 0u) u.w[0] = 0u;
-#pragma unroll
-                            for (int e = 0; e < 8; ++e) {
-                                c32 = entry_mass32(u.w[e], p32, c32);
-                                const double c = static_cast<double>(c32);
-                                const double d = c - x;
-                                if (z < 0 && (u.w[e] & 0xFFFFu)) {
-                                    if (fabs(d) <= ex + ec * c) { ok = false; QDBG(3); }
-                                    else if (d > 0.0) z = static_cast<int>(u.w[e] >> kTS);
-                                }
-                            }
-                        }
-                        if (z < 0 && ok) { ok = false; QDBG(4); }
-                    } else if (ok) {
-                        // dense bucket: first k with P[k] > y, i.e. S + P[k] > x
-                        // (K-1 if none, X6)
-                        int lo = 0, hi = K - 1;
-                        while (lo < hi) {
-                            const int mid = (lo + hi) >> 1;
-                            const double d = P[mid] - y;
-                            if (fabs(d) <= ed) { ok = false; QDBG(5); }
-                            if (d > 0.0) hi = mid;
-                            else lo = mid + 1;
-                        }
-                        z = lo;
-                    }
-                    if (!ok) {
-                        z = draw_exact_inl(rw, nnz, pstar, P, Q, K, x0);
-                        ++n_exact;
-                    }
-                    a.z[rec.z + k] = static_cast<uint16_t>(z);
-                    atomicAdd(&hist[z], 1);
-                }
-            }
-            __syncwarp();
-        }
-        __syncthreads();
-        // fused n_wk recount (ϕ update, L1273-1285), as in sweep_kernel
-        int32_t *row = a.nwk_next + static_cast<size_t>(ch.word) * K;
-        const bool split = (ch.split & 1u) != 0u;
-        for (int k = tid; k < K; k += kSweepThreads) {
-            const int h = hist[k];
-            if (split) {
-                if (h) atomicAdd(row + k, h);
-            } else {
-                row[k] = h;
-            }
-            nkp[k] += h;
-            hist[k] = 0;
-        }
-        __syncthreads();
-    }
-    for (int k = tid; k < K; k += kSweepThreads)
-        if (nkp[k]) atomicAdd(a.nk_next + k, nkp[k]);
-    if (a.n_exact) {
-        const unsigned tot = __reduce_add_sync(kFull, n_exact);
-        if (lane == 0 && tot) atomicAdd(a.n_exact, static_cast<unsigned long long>(tot));
-    }
 }
 
 // ---------------------------------------------------------------------------
@@ -1906,11 +1413,9 @@ __global__ void scatter_z_kernel(const uint32_t *__restrict__ doc_map, const uin
         zw[doc_map[i]] = zd[i];
 }
 
-// GATHERED = false: z through the doc-word map (fused); true: zd is z in
-// document order (phase B of the two-phase variant).
-template <bool GATHERED>
+// Phase B: zd is z in document order (gather_z_kernel).
 __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
-                             const uint32_t *__restrict__ doc_map, const uint16_t *__restrict__ z,
+                             const uint16_t *__restrict__ zd,
                              uint32_t *__restrict__ rows, int64_t D, int K,
                              unsigned long long *__restrict__ stat) {
     extern __shared__ uint32_t smem_u[];
@@ -1945,7 +1450,7 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
 #pragma unroll
             for (int r = 0; r < 4; ++r) {
                 const uint32_t i = i0 + 32u * r + lane;
-                kk[r] = i < e ? (GATHERED ? z[i] : z[doc_map[i]]) : 0xFFFFFFFFu;
+                kk[r] = i < e ? zd[i] : 0xFFFFFFFFu;
             }
 #pragma unroll
             for (int r = 0; r < 4; ++r) {
@@ -2061,6 +1566,96 @@ __global__ void ll_final_kernel(const double *__restrict__ part_w, int nw, const
 }
 
 // ---------------------------------------------------------------------------
+// Peer-memory collectives (the in-process PeerComm backend of Eq. 4's
+// exchange, comm.cpp): every rank's buffer is a device pointer readable by
+// the others (the same GPU, or P2P over NVLink).  16-byte vectors, L2-only
+// loads (another GPU's memory is never cached in this SM's L1).
+// ---------------------------------------------------------------------------
+struct PeerPtrs {
+    const char *p[kMaxPeers];
+};
+
+__host__ __device__ inline size_t peer_slice_lo(size_t n, int world, int q, size_t vw) {
+    return q >= world ? n : (n * static_cast<size_t>(q) / static_cast<size_t>(world)) / vw * vw;
+}
+
+template <class T>
+__global__ void peer_rs_kernel(PeerPtrs src, int world, T *__restrict__ own, size_t lo, size_t hi) {
+    constexpr int VW = 16 / sizeof(T);
+    const size_t nv = (hi - lo) / VW;
+    const size_t stride = static_cast<size_t>(gridDim.x) * blockDim.x;
+    for (size_t i = static_cast<size_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < nv; i += stride) {
+        const size_t off = (lo + i * VW) * sizeof(T);
+        T acc[VW];
+#pragma unroll
+        for (int j = 0; j < VW; ++j) acc[j] = T(0);
+        for (int q = 0; q < world; ++q) {
+            const uint4 v = __ldcg(reinterpret_cast<const uint4 *>(src.p[q] + off));
+            T t[VW];
+            memcpy(t, &v, 16);
+#pragma unroll
+            for (int j = 0; j < VW; ++j) acc[j] += t[j];
+        }
+        uint4 o;
+        memcpy(&o, acc, 16);
+        *reinterpret_cast<uint4 *>(reinterpret_cast<char *>(own) + off) = o;
+    }
+    // ragged tail of the last slice
+    for (size_t e = lo + nv * VW + static_cast<size_t>(blockIdx.x) * blockDim.x + threadIdx.x; e < hi; e += stride) {
+        T acc = T(0);
+        for (int q = 0; q < world; ++q) acc += reinterpret_cast<const T *>(src.p[q])[e];
+        own[e] = acc;
+    }
+}
+
+__global__ void peer_copy_kernel(const char *__restrict__ src, char *__restrict__ dst, size_t b0, size_t b1) {
+    // [b0, b1) bytes, b0 16-byte aligned
+    const size_t nv = (b1 - b0) / 16;
+    const size_t stride = static_cast<size_t>(gridDim.x) * blockDim.x;
+    for (size_t i = static_cast<size_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < nv; i += stride)
+        *reinterpret_cast<uint4 *>(dst + b0 + 16 * i) = __ldcg(reinterpret_cast<const uint4 *>(src + b0 + 16 * i));
+    for (size_t b = b0 + 16 * nv + static_cast<size_t>(blockIdx.x) * blockDim.x + threadIdx.x; b < b1; b += stride)
+        dst[b] = src[b];
+}
+
+static unsigned peer_grid(size_t work) {
+    const size_t g = (work + 255) / 256;
+    return static_cast<unsigned>(std::max<size_t>(1, std::min<size_t>(g, 148 * 8)));
+}
+
+int launch_peer_reduce_scatter(void *const *ptrs, int world, int rank, void *own, size_t n, size_t esz, int is_f64,
+                               void *stream) {
+    if (world < 1 || world > kMaxPeers) return cudaErrorInvalidValue;
+    PeerPtrs pp{};
+    for (int q = 0; q < world; ++q) pp.p[q] = static_cast<const char *>(ptrs[q]);
+    const size_t vw = 16 / esz;
+    const size_t lo = peer_slice_lo(n, world, rank, vw), hi = peer_slice_lo(n, world, rank + 1, vw);
+    if (hi <= lo) return cudaSuccess;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (is_f64)
+        peer_rs_kernel<double><<<peer_grid((hi - lo) / vw + 1), 256, 0, st>>>(pp, world, static_cast<double *>(own),
+                                                                            lo, hi);
+    else
+        peer_rs_kernel<int32_t><<<peer_grid((hi - lo) / vw + 1), 256, 0, st>>>(pp, world,
+                                                                             static_cast<int32_t *>(own), lo, hi);
+    return cudaGetLastError();
+}
+
+int launch_peer_all_gather(void *const *ptrs, int world, int rank, void *own, size_t n, size_t esz, void *stream) {
+    if (world < 1 || world > kMaxPeers) return cudaErrorInvalidValue;
+    const size_t vw = 16 / esz;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    for (int q = 0; q < world; ++q) {
+        if (q == rank) continue;
+        const size_t lo = peer_slice_lo(n, world, q, vw), hi = peer_slice_lo(n, world, q + 1, vw);
+        if (hi <= lo) continue;
+        peer_copy_kernel<<<peer_grid((hi - lo) / vw + 1), 256, 0, st>>>(static_cast<const char *>(ptrs[q]),
+                                                                       static_cast<char *>(own), lo * esz, hi * esz);
+    }
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
 // Launchers
 // ---------------------------------------------------------------------------
 int configure_kernels(DevState &s) {
@@ -2078,16 +1673,13 @@ int configure_kernels(DevState &s) {
         const bool smemp = LDA_FUSE && want + 2048 <= static_cast<size_t>(max_optin);
         s.sweep_smem = smemp ? want : blk;
         s.sweep_fused = smemp;
-        s.sweep_f32 = smemp && !s.exclude_self && s.filter32;
         const void *fn = nullptr;
         if (s.exclude_self)
-            fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<true, true, false>)
-                       : reinterpret_cast<const void *>(&sweep_kernel<true, false, false>);
-        else if (s.sweep_f32)
-            fn = reinterpret_cast<const void *>(&sweep_kernel<false, true, true>);
+            fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<true, true>)
+                       : reinterpret_cast<const void *>(&sweep_kernel<true, false>);
         else
-            fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<false, true, false>)
-                       : reinterpret_cast<const void *>(&sweep_kernel<false, false, false>);
+            fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<false, true>)
+                       : reinterpret_cast<const void *>(&sweep_kernel<false, false>);
         if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       static_cast<int>(s.sweep_smem))) != cudaSuccess)
             return e;
@@ -2095,27 +1687,6 @@ int configure_kernels(DevState &s) {
         if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, kSweepThreads, s.sweep_smem)) != cudaSuccess)
             return e;
         s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
-    }
-    // quad sampler (default): p*/P, histograms and per-warp pair prefixes in smem
-    {
-        const size_t want = static_cast<size_t>((28 * s.K + 15) / 16) * 16 +
-                            sizeof(uint32_t) * (kSweepThreads / 32) * kQWarpWords;
-        s.sweep_quad = s.sampler == 1 && !s.exclude_self && LDA_FUSE &&
-                       want + 2048 <= static_cast<size_t>(max_optin);
-        if (s.sweep_quad) {
-            const void *fn = reinterpret_cast<const void *>(&sweep_quad_kernel<LDA_QRING>);
-            s.quad_smem = want;
-            if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                          static_cast<int>(want))) != cudaSuccess)
-                return e;
-            int bps = 1;
-            if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, kSweepThreads, want)) != cudaSuccess)
-                return e;
-            s.quad_grid = s.num_sms * (bps > 0 ? bps : 1);
-            if (!s.sweep_fused) {  // the quad sampler always fuses the recount
-                s.sweep_fused = true;
-            }
-        }
     }
     // tile sampler (default): per CTA the n_k histogram, per warp the word
     // table and the batch scratch; <= 8 warps per CTA
@@ -2202,16 +1773,12 @@ int configure_kernels(DevState &s) {
     if (wpb < 1) return cudaErrorInvalidValue;
     s.theta_block = 32 * wpb;
     s.theta_smem = per_warp * wpb;
-    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel<true>),
-                                  cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  static_cast<int>(s.theta_smem))) != cudaSuccess)
-        return e;
-    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel<false>),
+    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel),
                                   cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   static_cast<int>(s.theta_smem))) != cudaSuccess)
         return e;
     int tb = 1;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, reinterpret_cast<const void *>(&theta_kernel<false>),
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, reinterpret_cast<const void *>(&theta_kernel),
                                                            s.theta_block, s.theta_smem)) != cudaSuccess)
         return e;
     s.theta_grid = s.num_sms * (tb > 0 ? tb : 1);
@@ -2275,16 +1842,13 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     if ((e = cudaMemsetAsync(stat_out, 0, 2 * sizeof(unsigned long long), st)) != cudaSuccess) return e;
-    if (s.z_doc) {
-        const int64_t thr = (s.T + 7) / 8;
+    const int64_t thr = (s.T + 7) / 8;
+    if (thr > 0) {
         gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, st>>>(s.doc_map, s.tok_z, s.z_doc, s.T);
         ++*launches;
-        theta_kernel<true><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.doc_map,
-                                                                           s.z_doc, s.rows, s.D, s.K, stat_out);
-    } else {
-        theta_kernel<false><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.doc_map,
-                                                                            s.tok_z, s.rows, s.D, s.K, stat_out);
     }
+    theta_kernel<<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.z_doc, s.rows, s.D,
+                                                                   s.K, stat_out);
     ++*launches;
     return cudaGetLastError();
 }
@@ -2377,34 +1941,6 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ++*launches;
         return cudaGetLastError();
     }
-    if (s.sweep_quad) {
-        QuadArgs qa;
-        qa.chunks = s.pchunks;
-        qa.n_chunks = s.n_pchunks;
-        qa.pairs = reinterpret_cast<const uint4 *>(s.pairs);
-        qa.z = s.tok_z;
-        qa.rows = s.rows;
-        qa.nwk = s.nwk;
-        qa.denom = s.denom;
-        qa.counter = s.counter;
-        qa.nwk_next = a.nwk_next;
-        qa.nk_next = a.nk_next;
-        qa.n_exact = s.stat + 2;
-        qa.K = s.K;
-        qa.alpha = s.alpha;
-        qa.beta = s.beta;
-        qa.t = t;
-        uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
-        for (int r = 0; r < 10; ++r) {
-            qa.key0[r] = k0;
-            qa.key1[r] = k1;
-            k0 += 0x9E3779B9u;
-            k1 += 0xBB67AE85u;
-        }
-        sweep_quad_kernel<LDA_QRING><<<s.quad_grid, kSweepThreads, s.quad_smem, st>>>(qa);
-        ++*launches;
-        return cudaGetLastError();
-    }
     a.chunks = s.chunks;
     a.n_chunks = s.n_chunks;
     a.segs = s.segs;
@@ -2430,23 +1966,15 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         k1 += 0xBB67AE85u;
     }
     if (s.exclude_self) {
-        if (s.sweep_fused) sweep_kernel<true, true, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
-        else sweep_kernel<true, false, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
-    } else if (s.sweep_f32) {
-        sweep_kernel<false, true, true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        if (s.sweep_fused) sweep_kernel<true, true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        else sweep_kernel<true, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
     } else {
-        if (s.sweep_fused) sweep_kernel<false, true, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
-        else sweep_kernel<false, false, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        if (s.sweep_fused) sweep_kernel<false, true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        else sweep_kernel<false, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
     }
     ++*launches;
     return cudaGetLastError();
 }
-
-#if LDA_QDEBUG
-extern "C" int lda_debug_counters(unsigned long long *out) {
-    return cudaMemcpyFromSymbol(out, g_qdbg, sizeof(g_qdbg));
-}
-#endif
 
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);

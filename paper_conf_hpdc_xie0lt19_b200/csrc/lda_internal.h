@@ -2,8 +2,11 @@
 // and the kernels (kernels.cu).  Not part of the ABI.
 #pragma once
 
+#include <condition_variable>
 #include <cstdint>
 #include <functional>
+#include <memory>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -70,26 +73,6 @@ struct RecountChunk {
     uint32_t pad[3];
 };
 
-// Quad sampler (sweep_quad_kernel): a word chunk's tokens grouped into
-// (word, doc) pairs -- consecutive tokens of the word in the same document,
-// which share the document's θ row and therefore S and the sparse prefix
-// (Eq. 6-7): one row walk per pair, one Philox draw per token.
-struct PairRec {
-    uint32_t row;    // θ row of the document, in 32-byte units (128-byte aligned)
-    uint32_t crank;  // canonical rank (within its word) of the pair's first token
-    uint32_t pos;    // word-major position of the first token (z[pos .. pos+m))
-    uint32_t mcl;    // m (tokens, 1..255) | row capacity in 128-byte lines << 8
-};
-struct PairChunk {
-    uint32_t word;
-    uint32_t pbegin;  // pairs [pbegin, pbegin + npairs)
-    uint32_t npairs;
-    uint32_t ntok;
-    uint32_t split;   // bit 0: the word is split over several chunks
-    uint32_t pad;
-    uint64_t c_base;  // canonical index of the rank's first token of the word
-};
-
 // Tile sampler (sweep_tile_kernel) work item: the tokens of one word inside
 // one document tile -- contiguous word-major positions [pos, pos + n) --
 // or a piece of them (at most chunk_tokens).  Items are queued tile by tile.
@@ -118,8 +101,6 @@ struct HostLayout {
     std::vector<int32_t> split_words;  // words whose row is accumulated atomically (recount)
     std::vector<int32_t> zero_words;   // words split over sampler chunks or without tokens
     std::vector<int64_t> word_count;   // V local tokens per word
-    std::vector<PairChunk> pchunks;    // quad sampler items (same split as `chunks`), heavy-first
-    std::vector<PairRec> pairs;        // their (word, doc) pairs, chunk by chunk
     std::vector<TileItem> titems;      // tile sampler items: tile-major, heavy-first inside a tile
 };
 
@@ -141,7 +122,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
-                            bool *range_error, int64_t *word_counts = nullptr);  // V counts, if wanted
+                            bool *range_error, int64_t *word_counts = nullptr,  // V counts, if wanted
+                            int nthreads = 0);                                    // 0: all host threads
 
 int host_threads(int requested);
 
@@ -167,7 +149,7 @@ struct DevState {
     uint16_t *tok_z = nullptr;      // T (word-major)
     uint32_t *doc_map = nullptr;    // T
     uint32_t *tok_crank = nullptr;  // T (word-major); null for the tile samplers (ranks from the items)
-    uint16_t *z_doc = nullptr;      // T, z in document order (two-phase θ rebuild only)
+    uint16_t *z_doc = nullptr;      // T, z in document order (θ rebuild, phase A)
     uint32_t *doc_ptr32 = nullptr;  // D+1
     uint32_t *row_off32 = nullptr;  // D
     Seg *segs = nullptr;
@@ -177,9 +159,6 @@ struct DevState {
     int64_t n_rchunks = 0;
     int32_t *split_words = nullptr;
     int64_t n_split = 0;
-    PairRec *pairs = nullptr;       // quad sampler: (word, doc) pairs
-    PairChunk *pchunks = nullptr;
-    int64_t n_pchunks = 0;
     TileItem *titems = nullptr;     // tile sampler items
     int64_t n_titems = 0;
     uint64_t *cbase = nullptr;      // V: canonical index of the rank's first token of each word
@@ -190,11 +169,7 @@ struct DevState {
     int32_t *zero_words = nullptr;  // words whose next-n_wk row is zeroed before the sweep
     int64_t n_zero_words = 0;
     bool sweep_fused = false;
-    bool sweep_f32 = false;
-    int sampler = -1;               // option: -1 auto, 2 = tile sampler, 1 = quad-per-pair, 0 = lane-per-token
-    bool sweep_quad = false;        // the quad sampler is used (sampler 1, fits in smem, no exclude_self)
-    size_t quad_smem = 0;
-    int quad_grid = 0;
+    int sampler = -1;               // option: -1 auto, 2 = tile sampler, 3 = its CTA form, 0 = lane-per-token
     bool sweep_tile = false;        // the tile sampler is used (sampler 2, fits in smem, no exclude_self)
     bool sweep_tile_cta = false;    // its large-K form with CTA-shared tables (sampler 3)
     bool tile_cta_gnk = false;      // ... with n_k by global reductions and compact tables (K > kTileMaxK)
@@ -205,7 +180,6 @@ struct DevState {
     char *wtab = nullptr;           // tile sampler: per-word tables (p32, dense prefix), rebuilt every sweep
     size_t wt_bytes = 0;
     double certify_slack = 1.0;     // test option: scales the tile sampler's certification bounds
-    int filter32 = 0;               // option: fp32 filter with exact fp64 fallback
     double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch
     uint32_t *counter = nullptr;    // work counters [4]
@@ -231,5 +205,67 @@ int launch_gather_z(const DevState &s, uint16_t *zd, void *stream);
 int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream);
 int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event);
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches);
+
+// ---------------------------------------------------------------------------
+// The exchange of Eq. 4 (L935-937), comm.cpp.  All calls return an lda_status
+// and fill `err` on failure.  Buffers are device pointers on the rank's GPU;
+// `stream` is the stream after which the buffer is final (NCCL enqueues on
+// it; the peer backend synchronises it and returns with the result written).
+// ---------------------------------------------------------------------------
+constexpr int kMaxPeers = 16;
+
+class Comm {
+  public:
+    virtual ~Comm() = default;
+    virtual const char *name() const = 0;
+    virtual int allreduce_i32(int32_t *buf, size_t n, void *stream, std::string &err) = 0;  // in place, sum
+    virtual int allreduce_f64(double *buf, size_t n, void *stream, std::string &err) = 0;   // in place, sum
+    // recv[q*n .. (q+1)*n) = rank q's send[0 .. n)
+    virtual int allgather_i64(const int64_t *send, int64_t *recv, size_t n, void *stream, std::string &err) = 0;
+    int rank() const { return rank_; }
+    int world() const { return world_; }
+
+  protected:
+    int rank_ = 0, world_ = 1;
+};
+
+// In-process group of `world` ranks, each driven by its own host thread.
+class PeerGroup {
+  public:
+    explicit PeerGroup(int world);
+    int world() const { return world_; }
+    int join(int rank, int device, std::string &err);
+    int barrier(std::string &err);
+    void set_ptr(int rank, void *p);
+    void ptrs(void **out);
+    int device(int rank);
+    void mark_broken();
+
+  private:
+    int world_;
+    std::mutex mu_;
+    std::condition_variable cv_;
+    int arrived_ = 0;
+    uint64_t gen_ = 0;
+    bool broken_ = false;
+    int timeout_s_ = 600;
+    std::vector<void *> ptr_;
+    std::vector<int> dev_;
+    std::vector<int> joined_;
+};
+
+int nccl_unique_id(void *out128, std::string &err);
+int make_nccl_comm(int rank, int world, const void *uid, int device, std::unique_ptr<Comm> &out, std::string &err);
+int make_peer_comm(const std::shared_ptr<PeerGroup> &g, int rank, int device, std::unique_ptr<Comm> &out,
+                   std::string &err);
+
+// Peer-memory collective kernels (kernels.cu).  ptrs[q] = rank q's buffer of
+// n elements of esz bytes (4: int32, 8: fp64 when is_f64).  Slice q is
+// [lo(q), lo(q+1)) with lo(q) = 16-byte-aligned q·n/world.
+// reduce-scatter: own[slice rank] = Σ_q ptrs[q][slice rank] (rank order);
+// all-gather: own[slice q] = ptrs[q][slice q] for every q != rank.
+int launch_peer_reduce_scatter(void *const *ptrs, int world, int rank, void *own, size_t n, size_t esz, int is_f64,
+                               void *stream);
+int launch_peer_all_gather(void *const *ptrs, int world, int rank, void *own, size_t n, size_t esz, void *stream);
 
 }  // namespace lda

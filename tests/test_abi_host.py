@@ -37,7 +37,12 @@ def test_create_validation():
         with pytest.raises(L.LDAError) as e:
             L.lda_create(*args)
         assert e.value.code == L.LDA_EINVAL
-    L.lda_destroy(L.lda_create(1, 1, 65536, 1.0, 1.0))
+    L.lda_destroy(L.lda_create(1, 1, 16384, 1.0, 1.0))
+    # u16 topic ids go to 65536 (L1239-1243); this build's θ entry stops at 16384
+    for K in (16385, 65536):
+        with pytest.raises(L.LDAError) as e:
+            L.lda_create(1, 1, K, 1.0, 1.0)
+        assert e.value.code == L.LDA_ERANGE
 
 
 def test_options_validation():
@@ -46,7 +51,11 @@ def test_options_validation():
         L.lda_set_option(ctx, "exclude_self", 1)
         L.lda_set_option(ctx, "chunk_tokens", 64)
         L.lda_set_option(ctx, "tile_tokens", 0)
-        for key, val in [("exclude_self", 2), ("chunk_tokens", 1), ("nonsense", 1), ("device", -1)]:
+        L.lda_set_option(ctx, "tile_tokens", -1)
+        L.lda_set_option(ctx, "loglik_every", 5)
+        for key, val in [("exclude_self", 2), ("chunk_tokens", 1), ("nonsense", 1), ("device", -1),
+                         ("sampler", 1), ("tile_tokens", -2), ("loglik_every", -1), ("theta_mode", 1),
+                         ("filter32", 1)]:
             with pytest.raises(L.LDAError) as e:
                 L.lda_set_option(ctx, key, val)
             assert e.value.code == L.LDA_EINVAL
@@ -133,7 +142,7 @@ def _corpus(D, V, seed, max_len=40, empty=True):
     return doc_ptr, words
 
 
-@pytest.mark.parametrize("sampler", [0, 1, 2, 3])
+@pytest.mark.parametrize("sampler", [0, 2, 3])
 @pytest.mark.parametrize("tile_tokens,chunk_tokens,tail", [(0, 4096, 64), (900, 4096, 64), (700, 33, 8),
                                                             (500, 7, 1000), (300, 64, 0)])
 def test_layout_invariants(sampler, tile_tokens, chunk_tokens, tail):
@@ -165,3 +174,53 @@ def test_layout_selfcheck_rejects_bad_input():
     bad[0] = 20                                               # word id >= V
     with pytest.raises(L.LDAError):
         L.lda_layout_selfcheck(doc_ptr, bad, 20, 4)
+
+
+def test_peer_group_host_validation():
+    """In-process peer group (include/lda.h): handle life cycle and join
+    validation, no device needed."""
+    with pytest.raises(L.LDAError) as e:
+        L.lda_peer_group_create(0)
+    assert e.value.code == L.LDA_EINVAL
+    with pytest.raises(L.LDAError):
+        L.lda_peer_group_create(17)
+    g = L.PeerGroup(2)
+    a = L.lda_create(10, 5, 16, 0.1, 0.01)
+    b = L.lda_create(10, 5, 16, 0.1, 0.01)
+    c = L.lda_create(10, 5, 16, 0.1, 0.01)
+    try:
+        L.lda_init_peer(a, g.h, 0)
+        for ctx, rank in [(b, 0), (b, 2), (b, -1)]:          # duplicate / out of range
+            with pytest.raises(L.LDAError) as e:
+                L.lda_init_peer(ctx, g.h, rank)
+            assert e.value.code == L.LDA_EINVAL
+        L.lda_init_peer(b, g.h, 1)
+        with pytest.raises(L.LDAError) as e:                  # a context joins once
+            L.lda_init_peer(a, g.h, 1)
+        assert e.value.code == L.LDA_ESTATE
+        g.close()                                             # contexts keep the group alive
+        L.lda_set_option(c, "threads", 2)
+    finally:
+        for ctx in (a, b, c):
+            L.lda_destroy(ctx)
+
+
+def test_python_binding_checks_buffer_lengths():
+    """The ctypes binding refuses short buffers before the C side could read
+    or write past them (argument marshalling only)."""
+    ctx = L.lda_create(2, 5, 8, 0.1, 0.01)
+    try:
+        with pytest.raises(L.LDAError) as e:                  # doc_ptr too short for [0, 2)
+            L.lda_load_corpus(ctx, 0, 2, np.array([0, 3], np.int64), np.arange(3, dtype=np.int32), 1)
+        assert e.value.code == L.LDA_EINVAL
+        with pytest.raises(L.LDAError) as e:                  # fewer words than doc_ptr[-1]
+            L.lda_load_corpus(ctx, 0, 2, np.array([0, 3, 5], np.int64), np.arange(4, dtype=np.int32), 1)
+        assert e.value.code == L.LDA_EINVAL
+        with pytest.raises(L.LDAError) as e:
+            L.lda_set_z(ctx, np.zeros(3, np.uint16), T=5)
+        assert e.value.code == L.LDA_EINVAL
+        with pytest.raises(L.LDAError) as e:
+            L.lda_get_counts(ctx, n_wk=np.zeros(39, np.int32), shape=(5, 8, 2, 5))
+        assert e.value.code == L.LDA_EINVAL
+    finally:
+        L.lda_destroy(ctx)

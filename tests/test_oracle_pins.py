@@ -289,3 +289,24 @@ def test_loglik_rises_on_tiny(tiny_corpus, tiny_cfg):
     assert np.all(np.diff(ll) > 0)
     assert ll[-1] - ll[0] >= 0.5
     assert -15.0 <= ll[-1] <= 0.0      # Fig. 8 axis range (L1509-1519)
+
+
+def test_oracle_omp_sweep_bit_identical():
+    """oracle-omp: the SWEEP with documents drawn on all host
+    cores must give exactly the single-threaded oracle's z, counts and
+    margins -- each draw reads only frozen counts and its own counter-based
+    uniform (X3, X9), so the order of the documents cannot matter."""
+    from paper_conf_hpdc_xie0lt19_b200 import synth
+    cfg = synth.scaled(synth.CONFIGS["nytimes"], 0.0005)          # ~50k tokens
+    doc_ptr, words = synth.to_numpy(*synth.generate_config(cfg, "cpu"))[:2]
+    K = 64
+    a = O.OracleLDA(cfg.D, cfg.V, K, 50.0 / K, 0.01).load(doc_ptr, words, 3)
+    b = O.OracleLDA(cfg.D, cfg.V, K, 50.0 / K, 0.01).load(doc_ptr, words, 3)
+    for _ in range(3):
+        ma = a.iterate(1, margins=True)
+        mb = b.iterate(1, margins=True, parallel=True)
+        assert np.array_equal(a.z, b.z)
+        assert np.array_equal(ma, mb)
+        assert np.array_equal(a.n_wk, b.n_wk) and np.array_equal(a.n_k, b.n_k)
+        assert np.array_equal(a.n_dk, b.n_dk)
+    assert O.omp_threads() >= 1

@@ -48,7 +48,7 @@ def run(config="tiny", sweeps=20, every=5, device_index=None, write=False, opts=
     bounds = L.lda_partition_docs(doc_ptr_full, world)
     d0, d1 = int(bounds[rank]), int(bounds[rank + 1])
     t0, t1 = int(doc_ptr_full[d0]), int(doc_ptr_full[d1])
-    o = dict(C.BENCH_OPTIONS if cfg.T > 10_000_000 else {})
+    o = {}
     o.update(opts or {})
     m = L.LDA(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, device=local, **o)
     if world > 1:

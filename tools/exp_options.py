@@ -2,7 +2,7 @@
 sampler under several lda_set_option sets in one process.
 
     python tools/exp_options.py --config pubmed --sweeps 5 --warmup 3 \
-        --set "filter32=0" --set "filter32=1"
+        --set "fused_recount=0" --set "fused_recount=1"
 
 Prints one line per option set: G tokens/s, ms per phase, nnz per token.
 Not a bench number (no clocks check, no e2e); bench.py is the contract.
@@ -41,7 +41,7 @@ def main():
     print(f"# {cfg.name}: generated in {time.time() - t0:.1f}s, lib {L.LIB_PATH}", flush=True)
     sets = args.set or [""]
     for s in sets:
-        opts = dict(C.BENCH_OPTIONS)
+        opts = {}
         for kv in filter(None, s.split(",")):
             k, v = kv.split("=")
             opts[k] = int(v)
