@@ -300,14 +300,18 @@ def run_b200(args):
     b_sweep = sum(C.bytes_sweep(T_g, D_g, cfg.V, cfg.K, int(a), int(b)) for a, b in
                   zip(log["sum_nnz_tok"], log["sum_nnz_doc"]))
     sweep_gbs = b_sweep / (float(np.sum(log["ms_sweep"])) / 1e3) / 1e9
-    traffic = None
+    # DRAM bytes per launch of the sampling kernel from the committed ncu
+    # capture of this config (profiles/traffic.json, tools/write_traffic.py)
+    traffic, traffic_src = None, None
     try:
-        with open(os.path.join(ROOT, "profiles", "latest_traffic.json")) as f:
-            tr = json.load(f)
-            if tr.get("config") == cfg.name:
-                traffic = tr.get("sweep_kernel_dram_bytes_per_launch")
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            tr = json.load(f).get(cfg.name)
+        if tr:
+            traffic = float(tr["sweep_kernel_dram_bytes_per_launch"])
+            traffic_src = f"{tr['report']} ({tr['round']})"
     except Exception:
         pass
+    t_sample_launch = t_sample / args.steps
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -329,12 +333,22 @@ def run_b200(args):
                        "alpha": cfg.alpha, "beta": cfg.beta, "seed": cfg.seed,
                        "timed_sweeps": [int(st["sweeps_done"]) - args.steps + 1, int(st["sweeps_done"])],
                        "l2": "inputs (GBs) larger than the 126 MB L2; no flush",
-                       "parallelism": f"doc-partitioned dp{world}", "options": opts},
+                       "parallelism": f"doc-partitioned dp{world}", "options": opts,
+                       "sampler": int(st["sampler"]), "tile_tokens": int(st["tile_tokens"]),
+                       "tiles": int(st["n_tiles"])},
             "roofline": {"bound": "hbm", "kernel": kernel, "achieved": achieved, "peak": peak,
                          "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                         "achieved_basis": "algorithmic bytes (SURVEY §8(d) B_sample, measured nnz) / "
+                                           "kernel event time",
                          "peak_source": peak_src,
                          "frac_of_8TBs_spec": achieved / 8000.0,
+                         "algorithmic_bytes_per_launch": b_sample / args.steps,
+                         "dram_achieved": (traffic / t_sample_launch / 1e9) if traffic else None,
+                         "dram_frac": (traffic / t_sample_launch / 1e9 / peak) if traffic else None,
+                         "traffic_over_algorithmic": (traffic / (b_sample / args.steps)) if traffic else None,
+                         "traffic_source": traffic_src,
                          "sweep_achieved": sweep_gbs, "sweep_frac": sweep_gbs / peak,
+                         "sweep_frac_of_8TBs_spec": sweep_gbs / 8000.0,
                          "bytes_per_token_model": b_sample / (T_g * args.steps)},
             "phases_ms_per_step": {"sample": float(t[1]) / args.steps,
                                    "sampler_kernel": 1e3 * t_sample / args.steps,

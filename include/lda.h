@@ -144,6 +144,11 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   2.7 % faster per sweep at PubMed shape); 1 = accumulated
  *                   by the sampler itself (warp-aggregated reductions).  Same
  *                   counts.
+ *   "comm_pipeline" world > 1 with the recount kernel (fused_recount = 0):
+ *                   recount n_wk in this many word ranges (default 4) and
+ *                   start the exchange (Eq. 4) of each range's rows as soon
+ *                   as it is recounted, overlapping the rest of the recount
+ *                   and the θ rebuild (§6.2).  Same counts.
  *   "certify_slack" samplers 2, 3, tests only: multiply every certification
  *                   bound by this factor (default 1) -- more tokens take the
  *                   exact fp64 redraw; the draws must not change

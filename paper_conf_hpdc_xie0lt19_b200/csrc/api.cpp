@@ -33,6 +33,7 @@ struct lda_ctx {
     int64_t tail_per_tile = 64;
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
+    int64_t comm_pipeline = 4;  // world > 1: word ranges whose rows are exchanged as soon as recounted (f1)
     int threads = 0;
     // distribution: the exchange of Eq. 4 (NCCL or the in-process peer group)
     int32_t rank = 0, world = 1;
@@ -57,6 +58,10 @@ struct lda_ctx {
     size_t stat_log_cap = 0;
     std::vector<double> log_ms, log_ms_sample, log_ms_recount, log_ms_theta, log_ms_comm;
     std::vector<int64_t> log_nnz_tok, log_nnz_doc;
+    // f1: recount work items grouped by word range; range p = items
+    // [rc_begin[p], rc_begin[p+1]), rows [w_begin[p], w_begin[p+1]) of n_wk
+    std::vector<int64_t> rc_begin, w_begin;
+    std::vector<cudaEvent_t> range_ev;
     // option loglik_every: LL/token after every n-th sweep of lda_iterate
     int64_t loglik_every = 0;
     double *d_ll_log = nullptr;
@@ -222,6 +227,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
+    } else if (k == "comm_pipeline") {
+        if (value < 1 || value > 64) return fail(ctx, LDA_EINVAL, "comm_pipeline must be in [1, 64]");
+        ctx->comm_pipeline = value;
     } else if (k == "loglik_every") {
         if (value < 0 || value > (int64_t(1) << 31)) return fail(ctx, LDA_EINVAL, "loglik_every must be >= 0");
         ctx->loglik_every = value;
@@ -500,6 +508,28 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                    : std::string("token table copy: ") + cudaGetErrorString(copy_err));
     }
     if (pre_rows32 != H.rows32) return fail(ctx, LDA_ECUDA, "internal: θ row storage size mismatch");
+    {
+        // f1: with world > 1 and the recount kernel, the n_wk rows are
+        // exchanged word range by word range as soon as each range is
+        // recounted (overlapping the rest of the recount and the θ rebuild);
+        // range p holds words [ceil(pV/P), ceil((p+1)V/P)).  Heavy-first
+        // inside a range.  Results do not depend on P.
+        const int64_t P = (ctx->world > 1 && !S.sweep_fused) ? std::min<int64_t>(ctx->comm_pipeline, V) : 1;
+        auto range_of = [&](const lda::RecountChunk &c) {
+            return static_cast<int64_t>(c.word & 0x7FFFFFFFu) * P / V;
+        };
+        std::stable_sort(H.rchunks.begin(), H.rchunks.end(),
+                         [&](const lda::RecountChunk &a, const lda::RecountChunk &b) { return range_of(a) < range_of(b); });
+        ctx->rc_begin.assign(P + 1, 0);
+        ctx->w_begin.assign(P + 1, 0);
+        for (int64_t p = 0; p <= P; ++p) ctx->w_begin[p] = (p * V + P - 1) / P;
+        size_t i = 0;
+        for (int64_t p = 0; p < P; ++p) {
+            ctx->rc_begin[p] = static_cast<int64_t>(i);
+            while (i < H.rchunks.size() && range_of(H.rchunks[i]) == p) ++i;
+        }
+        ctx->rc_begin[P] = static_cast<int64_t>(H.rchunks.size());
+    }
     lda::tmark("layout done, token tables on the device");
 
     S.V = V;
@@ -507,6 +537,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.D = Dg;
     S.T = Tg;
     S.ntiles = H.ntiles;
+    S.rows32 = H.rows32;
     S.alpha = ctx->alpha;
     S.beta = ctx->beta;
     S.seed = seed;
@@ -587,9 +618,14 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     if (n < 0) return fail(ctx, LDA_EINVAL, "negative sweep count");
     CU(cudaSetDevice(ctx->device));
     lda::DevState &S = ctx->S;
-    const int per = 7;
+    const int per = 8;
     int r = ensure_events(ctx, static_cast<size_t>(per) * std::max(n, 1));
     if (r != LDA_OK) return r;
+    while (ctx->range_ev.size() + 1 < ctx->rc_begin.size()) {
+        cudaEvent_t e;
+        CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        ctx->range_ev.push_back(e);
+    }
     if (ctx->stat_log_cap < static_cast<size_t>(n)) {
         if (ctx->d_stat_log) {
             CU(cudaFree(ctx->d_stat_log));
@@ -615,16 +651,37 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventRecord(E[0], ctx->stream));
         KL(lda::launch_sweep(S, t, ctx->stream, &launches, E[6]));
         CU(cudaEventRecord(E[1], ctx->stream));
-        if (S.sweep_fused) std::swap(S.nwk, S.nwk_alt);  // the sampler wrote the next counts
-        else KL(lda::launch_recount(S, ctx->stream, &launches));
+        const int64_t P = static_cast<int64_t>(ctx->rc_begin.size()) - 1;
+        if (S.sweep_fused) {
+            std::swap(S.nwk, S.nwk_alt);  // the sampler wrote the next counts
+        } else {
+            // the ϕ update (L1273-1285), word range by word range (f1)
+            for (int64_t p = 0; p < P; ++p) {
+                KL(lda::launch_recount(S, ctx->stream, &launches, ctx->rc_begin[p], ctx->rc_begin[p + 1], p == 0));
+                if (ctx->world > 1 && P > 1) CU(cudaEventRecord(ctx->range_ev[p], ctx->stream));
+            }
+        }
         CU(cudaEventRecord(E[2], ctx->stream));
         // θ update (depends only on z) on the compute stream while ϕ is
         // summed over the ranks on the comm stream (§6.2)
         KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches));
         CU(cudaEventRecord(E[3], ctx->stream));
         if (ctx->world > 1) {
-            CU(cudaStreamWaitEvent(ctx->comm_stream, E[2], 0));
-            COMM(allreduce_i32(S.nwk, static_cast<size_t>(S.V) * S.K + S.K, ctx->comm_stream, e_));
+            const size_t K = static_cast<size_t>(S.K);
+            if (S.sweep_fused || P == 1) {
+                CU(cudaStreamWaitEvent(ctx->comm_stream, E[2], 0));
+                CU(cudaEventRecord(E[7], ctx->comm_stream));
+                COMM(allreduce_i32(S.nwk, static_cast<size_t>(S.V) * K + K, ctx->comm_stream, e_));
+            } else {
+                for (int64_t p = 0; p < P; ++p) {
+                    // rows of range p; the last range carries n_k (complete after every range's recount)
+                    const size_t r0 = static_cast<size_t>(ctx->w_begin[p]) * K;
+                    const size_t r1 = static_cast<size_t>(ctx->w_begin[p + 1]) * K + (p == P - 1 ? K : 0);
+                    CU(cudaStreamWaitEvent(ctx->comm_stream, ctx->range_ev[p], 0));
+                    if (p == 0) CU(cudaEventRecord(E[7], ctx->comm_stream));
+                    if (r1 > r0) COMM(allreduce_i32(S.nwk + r0, r1 - r0, ctx->comm_stream, e_));
+                }
+            }
             CU(cudaEventRecord(E[4], ctx->comm_stream));
             CU(cudaStreamWaitEvent(ctx->stream, E[4], 0));
         }
@@ -681,7 +738,8 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventElapsedTime(&tot, E[0], E[5]));
         float x = 0;
         if (ctx->world > 1) {
-            CU(cudaEventElapsedTime(&d, E[2], E[4]));
+            // raw exchange time: from the first range's start to the end (includes waits for later ranges)
+            CU(cudaEventElapsedTime(&d, E[7], E[4]));
             // exposed: the compute stream's wait for the allreduce after the θ rebuild
             CU(cudaEventElapsedTime(&x, E[3], E[5]));
         }
@@ -859,6 +917,7 @@ void lda_destroy(lda_ctx *ctx) {
         if (ctx->stream) cudaStreamSynchronize(ctx->stream);
         for (void *p : ctx->allocs) cudaFree(p);
         for (cudaEvent_t e : ctx->ev) cudaEventDestroy(e);
+        for (cudaEvent_t e : ctx->range_ev) cudaEventDestroy(e);
         if (ctx->stream) cudaStreamDestroy(ctx->stream);
         if (ctx->comm_stream) cudaStreamDestroy(ctx->comm_stream);
     }

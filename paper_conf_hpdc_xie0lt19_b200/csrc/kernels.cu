@@ -481,6 +481,7 @@ struct TileArgs {
     uint32_t wt_bytes;
     int nbuf;                  // sweep_tile_cta_kernel: table buffers per CTA
     int recount;               // 1: the ϕ update fused here; 0: recount_kernel after the sweep
+    uint32_t zero_line;        // offset (32-byte units) of an all-zero 128-byte line of `rows`
     uint32_t t;
     uint32_t key0[10], key1[10];
 };
@@ -797,11 +798,15 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
             s1 = entry_mass32(ring[s2].w[7], p32, s1);
             bs[s2] = s0 + s1;
         }
+        // refill for the next step (if any): a quad past the batch's last
+        // line loads the all-zero line instead, so that its lookups go to
+        // p32[0] (one broadcast) rather than to the stale entries' random
+        // topics (bank conflicts)
+        if (base + 8u * R < lsum) {
 #pragma unroll
-        for (int s2 = 0; s2 < R; ++s2) {
-            const uint32_t Ln = base + 8u * (s2 + R) + q;
-            if (Ln < lsum) {
-                const uint32_t lr = lrow[Ln];
+            for (int s2 = 0; s2 < R; ++s2) {
+                const uint32_t Ln = base + 8u * (s2 + R) + q;
+                const uint32_t lr = Ln < lsum ? lrow[Ln] : a.zero_line;
                 ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
                 hdr[s2] = sub == 0 && (lr >> 31);
             }
@@ -1800,19 +1805,28 @@ int launch_init(const DevState &s, void *stream) {
     return cudaGetLastError();
 }
 
-int launch_recount(const DevState &s, void *stream, int *launches) {
+// Recount work items [rc0, rc1) (rc1 < 0: all).  `first`: the launch that
+// opens the sweep's recount (n_k and the rows of split words zeroed).  The
+// word-range pipeline (f1) calls it once per word range, each followed by
+// the exchange of that range's rows.
+int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0, int64_t rc1, bool first) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
+    if (rc1 < 0) rc1 = s.n_rchunks;
     int32_t *nk = s.nwk + static_cast<size_t>(s.V) * s.K;
-    if ((e = cudaMemsetAsync(nk, 0, sizeof(int32_t) * s.K, st)) != cudaSuccess) return e;
-    if ((e = cudaMemsetAsync(s.counter + 1, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
-    if (s.n_split > 0) {
-        zero_rows_kernel<<<static_cast<int>(std::min<int64_t>(s.n_split, 65535)), 256, 0, st>>>(
-            s.split_words, s.n_split, s.nwk, s.K);
-        ++*launches;
+    if (first) {
+        if ((e = cudaMemsetAsync(nk, 0, sizeof(int32_t) * s.K, st)) != cudaSuccess) return e;
+        if (s.n_split > 0) {
+            zero_rows_kernel<<<static_cast<int>(std::min<int64_t>(s.n_split, 65535)), 256, 0, st>>>(
+                s.split_words, s.n_split, s.nwk, s.K);
+            ++*launches;
+        }
     }
-    recount_kernel<<<s.sweep_grid > 0 ? s.num_sms * 4 : 1, 256, 8 * s.K, st>>>(
-        s.rchunks, s.n_rchunks, s.segs, s.K, s.tok_z, s.nwk, nk, s.counter + 1);
+    if (rc1 <= rc0) return cudaGetLastError();
+    if ((e = cudaMemsetAsync(s.counter + 1, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
+    const int grid = static_cast<int>(std::min<int64_t>(rc1 - rc0, static_cast<int64_t>(s.num_sms) * 4));
+    recount_kernel<<<grid, 256, 8 * s.K, st>>>(s.rchunks + rc0, rc1 - rc0, s.segs, s.K, s.tok_z, s.nwk, nk,
+                                               s.counter + 1);
     ++*launches;
     return cudaGetLastError();
 }
@@ -1924,6 +1938,7 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
         ta.nbuf = s.tile_nbuf;
         ta.recount = s.tile_fused ? 1 : 0;
+        ta.zero_line = static_cast<uint32_t>(s.rows32 - 4);  // the tail pad (zeroed at load, never written)
         ta.t = t;
         uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
         for (int r = 0; r < 10; ++r) {

@@ -164,6 +164,7 @@ struct DevState {
     uint64_t *cbase = nullptr;      // V: canonical index of the rank's first token of each word
     // model
     uint32_t *rows = nullptr;       // θ rows, rows32*8 words
+    uint64_t rows32 = 0;            // θ row storage in 32-byte units; the last 4 (one 128-byte line) stay zero
     int32_t *nwk = nullptr;         // V*K + K (n_k at offset V*K), the current counts
     int32_t *nwk_alt = nullptr;     // the other buffer: the sampler's fused recount writes here
     int32_t *zero_words = nullptr;  // words whose next-n_wk row is zeroed before the sweep
@@ -198,7 +199,8 @@ int configure_kernels(DevState &s);
 int launch_init(const DevState &s, void *stream);
 // tok_row[doc_map[i]] = row_off32[d(i)] on the device (the tile layout's host pass leaves it out)
 int launch_tok_row(const DevState &s, void *stream);
-int launch_recount(const DevState &s, void *stream, int *launches);
+int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0 = 0, int64_t rc1 = -1,
+                   bool first = true);
 int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches);
 // z in document order <-> word-major, through doc_map (device buffers of T entries; zd 16-byte aligned)
 int launch_gather_z(const DevState &s, uint16_t *zd, void *stream);

@@ -107,6 +107,8 @@ def _check_equal_to_one_rank(one, many, world):
     (3, "nytimes1pct", 1024, dict(fused_recount=1, tile_tokens=100_000)),
     (2, "nytimes1pct", 128, dict(sampler=3)),
     (4, "nytimes1pct", 1024, dict(sampler=0)),
+    (2, "nytimes1pct", 1024, dict(comm_pipeline=1)),
+    (3, "nytimes1pct", 1024, dict(comm_pipeline=17, recount_tokens=300)),
 ])
 def test_world_equals_one_gpu_bitwise(world, corpus, K, opts):
     D, V, doc_ptr, words = _corpus(corpus)

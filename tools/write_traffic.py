@@ -1,5 +1,7 @@
-"""Write profiles/latest_traffic.json from an ncu --set full report of the
-sampling kernel: dram__bytes_read.sum + dram__bytes_write.sum per launch.
+"""Record, in profiles/traffic.json (one entry per bench config), the DRAM
+traffic of the sampling kernel from an ncu --set full report:
+dram__bytes_read.sum + dram__bytes_write.sum per launch (bench.py reports it
+as roofline.traffic for that config).
 Usage: python tools/write_traffic.py <report.ncu-rep> <config-name> <round-tag>"""
 import csv
 import io
@@ -25,8 +27,11 @@ def main(rep, config, tag):
                "sweep_kernel_dram_bytes_per_launch": rd + wr, "dram_read": rd, "dram_write": wr,
                "ncu_duration_" + units[ix["gpu__time_duration.sum"]]: t, "report": os.path.basename(rep)}
         os.makedirs("profiles", exist_ok=True)
-        with open(os.path.join("profiles", "latest_traffic.json"), "w") as f:
-            json.dump(doc, f, indent=1)
+        path = os.path.join("profiles", "traffic.json")
+        allc = json.load(open(path)) if os.path.exists(path) else {}
+        allc[config] = doc
+        with open(path, "w") as f:
+            json.dump(allc, f, indent=1, sort_keys=True)
         print(json.dumps(doc))
         return
 
