@@ -91,15 +91,18 @@ typedef struct lda_stats {
                                + 4·Σ_d nnz'_d + 8·D_g */
     double bytes_sample;    /* the sampling kernel's share of it:
                                14·T_g + 4·Σ_t nnz_d(t) + 4·V·K */
+    int64_t n_stream_chunks;/* M: chunks streamed per sweep (option stream_chunks;
+                               1 = the corpus stays resident, WorkSchedule1) */
 } lda_stats;
 
 /* Create a context.  D = global number of documents, V = vocabulary size,
  * K = number of topics, α, β = Dirichlet hyper-parameters (Eq. 1; the paper
  * uses α = 50/K, β = 0.01 at L1339, X1).  No device work is done.
  * Errors: LDA_EINVAL unless D >= 1, V >= 1, 1 <= K <= 65536 (topic ids are
- * uint16, L1239-1243), α and β finite and > 0; LDA_ERANGE for
- * 16384 < K <= 65536 (this build packs a θ entry as topic << 18 | count and
- * keeps K-length histograms in shared memory).  *out is set to NULL on error. */
+ * uint16, L1239-1243), α and β finite and > 0.  For K > 16384 θ entries are
+ * packed topic << 16 | count, the K-length histograms of the recount and the
+ * θ rebuild live in global scratch, and the sampler is the lane-per-token
+ * one (sampler 0).  *out is set to NULL on error. */
 int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_ctx **out);
 
 /* Set an integer option before lda_load_corpus (LDA_ESTATE after).  Keys:
@@ -144,6 +147,16 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   2.7 % faster per sweep at PubMed shape); 1 = accumulated
  *                   by the sampler itself (warp-aggregated reductions).  Same
  *                   counts.
+ *   "stream_chunks" M >= 1 (default 1).  M > 1: out-of-HBM streaming (Alg. 1
+ *                   WorkSchedule2, L835-859, §5.1): the rank's
+ *                   documents are cut into M token-balanced chunks whose
+ *                   token tables, z and θ rows stay in page-locked host
+ *                   memory; every sweep streams each chunk through one of two
+ *                   device slots (the transfer of chunk m+1 overlaps the
+ *                   sampling of chunk m, L925-931), n_wk and the word tables
+ *                   stay resident.  Needs sampler 2 or 3 (exclude_self = 0).
+ *                   Same draws as M = 1.  With M > 1 ms_sample holds the
+ *                   whole chunk loop (recount and θ inside it).
  *   "comm_pipeline" world > 1 with the recount kernel (fused_recount = 0):
  *                   recount n_wk in this many word ranges (default 4) and
  *                   start the exchange (Eq. 4) of each range's rows as soon

@@ -19,6 +19,27 @@
 #include "../../include/lda.h"
 #include "lda_internal.h"
 
+// f3 (Alg. 1 WorkSchedule2, L835-859; §5.1): with M > 1 a rank's
+// documents are cut into M chunks whose per-token state lives in pinned host
+// memory and is streamed through two device slots every sweep (the transfer
+// of chunk m+1 overlaps the computation of chunk m, L925-931).
+namespace lda_stream {
+struct Chunk {
+    lda::HostLayout H;                // token tables (tok_row, doc_map: host, page-locked), items, runs
+    lda::DevState R;                  // device-resident small tables of the chunk (offsets, runs, items)
+    int64_t doc_begin = 0, D = 0;     // rank-local documents [doc_begin, doc_begin + D)
+    int64_t tok_begin = 0, T = 0;     // rank-local tokens
+    uint16_t *hz = nullptr;           // pinned: z, word-major (the chunk's layout)
+    uint32_t *hrows = nullptr;        // pinned: θ rows, rows32 * 8 words
+    bool registered = false;
+};
+struct Slot {
+    uint32_t *tok_row = nullptr, *doc_map = nullptr, *rows = nullptr;
+    uint16_t *z = nullptr, *z_doc = nullptr;
+    cudaEvent_t in = nullptr, done = nullptr, free_ = nullptr;
+};
+}  // namespace lda_stream
+
 struct lda_ctx {
     int64_t D = 0;
     int32_t V = 0, K = 0;
@@ -62,11 +83,15 @@ struct lda_ctx {
     // [rc_begin[p], rc_begin[p+1]), rows [w_begin[p], w_begin[p+1]) of n_wk
     std::vector<int64_t> rc_begin, w_begin;
     std::vector<cudaEvent_t> range_ev;
+    // f3: out-of-HBM streaming (option stream_chunks = M)
+    int64_t stream_chunks = 1;
+    std::vector<std::unique_ptr<lda_stream::Chunk>> chunks;
+    lda_stream::Slot slot[2];
+    cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
     // option loglik_every: LL/token after every n-th sweep of lda_iterate
     int64_t loglik_every = 0;
-    double *d_ll_log = nullptr;
     std::vector<int64_t> ll_sweep;
-    std::vector<double> ll_value;
+    std::vector<double> ll_value, ll_pending;
 };
 
 // Handle of an in-process peer group (shared by its ranks' contexts).
@@ -76,7 +101,7 @@ struct lda_peer_group {
 
 namespace {
 
-constexpr int32_t kMaxK = 16384;
+constexpr int32_t kMaxK = 65536;  // u16 topic ids (L1239-1243)
 
 int fail(lda_ctx *c, int code, const std::string &msg) {
     if (c) {
@@ -164,6 +189,326 @@ int rebuild_counts(lda_ctx *ctx, int *launches) {
     return LDA_OK;
 }
 
+
+// ---------------------------------------------------------------------------
+// f3: out-of-HBM streaming (Alg. 1 WorkSchedule2, L835-859, §5.1)
+// ---------------------------------------------------------------------------
+// The device view of chunk m in slot sl: the configured kernels and model
+// buffers of ctx->S, the chunk's resident tables, the slot's token buffers.
+lda::DevState chunk_view(lda_ctx *ctx, int64_t m, int sl) {
+    const lda_stream::Chunk &c = *ctx->chunks[m];
+    const lda_stream::Slot &b = ctx->slot[sl];
+    lda::DevState v = ctx->S;
+    v.D = c.D;
+    v.T = c.T;
+    v.ntiles = c.H.ntiles;
+    v.rows32 = c.H.rows32;
+    v.doc_ptr32 = c.R.doc_ptr32;
+    v.row_off32 = c.R.row_off32;
+    v.segs = c.R.segs;
+    v.rchunks = c.R.rchunks;
+    v.n_rchunks = c.R.n_rchunks;
+    v.split_words = nullptr;
+    v.n_split = 0;
+    v.titems = c.R.titems;
+    v.n_titems = c.R.n_titems;
+    v.cbase = c.R.cbase;
+    v.tok_row = b.tok_row;
+    v.doc_map = b.doc_map;
+    v.tok_z = b.z;
+    v.z_doc = b.z_doc;
+    v.rows = b.rows;
+    return v;
+}
+
+// DataTransfer(Chunk, θ: CPU -> GPU) of Alg. 1 lines 26-27
+int chunk_h2d(lda_ctx *ctx, int64_t m, int sl, cudaStream_t st, bool with_z) {
+    const lda_stream::Chunk &c = *ctx->chunks[m];
+    const lda_stream::Slot &b = ctx->slot[sl];
+    const size_t T = static_cast<size_t>(c.T);
+    if (T) {
+        CU(cudaMemcpyAsync(b.tok_row, c.H.tok_row.data(), 4 * T, cudaMemcpyHostToDevice, st));
+        CU(cudaMemcpyAsync(b.doc_map, c.H.doc_map.data(), 4 * T, cudaMemcpyHostToDevice, st));
+        if (with_z) CU(cudaMemcpyAsync(b.z, c.hz, 2 * T, cudaMemcpyHostToDevice, st));
+    }
+    CU(cudaMemcpyAsync(b.rows, c.hrows, 32 * c.H.rows32, cudaMemcpyHostToDevice, st));
+    return LDA_OK;
+}
+
+// DataTransfer(θ: GPU -> CPU) of Alg. 1 line 29 (and the chunk's new z)
+int chunk_d2h(lda_ctx *ctx, int64_t m, int sl, cudaStream_t st) {
+    const lda_stream::Chunk &c = *ctx->chunks[m];
+    const lda_stream::Slot &b = ctx->slot[sl];
+    if (c.T) CU(cudaMemcpyAsync(c.hz, b.z, 2 * static_cast<size_t>(c.T), cudaMemcpyDeviceToHost, st));
+    CU(cudaMemcpyAsync(c.hrows, b.rows, 32 * c.H.rows32, cudaMemcpyDeviceToHost, st));
+    return LDA_OK;
+}
+
+// n_wk, n_k (accumulated over the chunks, then exchanged) and every chunk's θ
+// from z; init = true draws the random initial z first (t = 0, X10).
+int chunked_rebuild(lda_ctx *ctx, bool init, int *launches) {
+    lda::DevState &S = ctx->S;
+    const size_t nwk_n = static_cast<size_t>(S.V) * S.K + S.K;
+    CU(cudaMemsetAsync(S.nwk, 0, nwk_n * sizeof(int32_t), ctx->stream));
+    int64_t lnnz = 0, nnz = 0;
+    for (int64_t m = 0; m < static_cast<int64_t>(ctx->chunks.size()); ++m) {
+        int r = chunk_h2d(ctx, m, 0, ctx->stream, !init);
+        if (r != LDA_OK) return r;
+        lda::DevState v = chunk_view(ctx, m, 0);
+        if (init) KL(lda::launch_init(v, ctx->stream));
+        KL(lda::launch_recount(v, ctx->stream, launches, 0, -1, false));
+        KL(lda::launch_theta(v, S.stat, ctx->stream, launches));
+        r = chunk_d2h(ctx, m, 0, ctx->stream);
+        if (r != LDA_OK) return r;
+        unsigned long long hs[2] = {0, 0};
+        CU(cudaMemcpyAsync(hs, S.stat, sizeof(hs), cudaMemcpyDeviceToHost, ctx->stream));
+        CU(cudaStreamSynchronize(ctx->stream));
+        lnnz += static_cast<int64_t>(hs[0]);
+        nnz += static_cast<int64_t>(hs[1]);
+    }
+    if (ctx->world > 1) COMM(allreduce_i32(S.nwk, nwk_n, ctx->stream, e_));
+    CU(cudaStreamSynchronize(ctx->stream));
+    ctx->cur_lnnz = lnnz;
+    ctx->cur_nnz = nnz;
+    return LDA_OK;
+}
+
+int load_chunked(lda_ctx *ctx, const int64_t *doc_ptr, const int32_t *words, int64_t Dg, int64_t Tg,
+                 const std::vector<int64_t> &cbase_rank, uint64_t seed) {
+    lda::DevState &S = ctx->S;
+    const int32_t V = ctx->V, K = ctx->K;
+    const int64_t M = std::max<int64_t>(1, std::min<int64_t>(ctx->stream_chunks, std::max<int64_t>(Dg, 1)));
+    std::vector<int64_t> bounds(M + 1);
+    if (lda_partition_docs(Dg, doc_ptr, static_cast<int32_t>(M), bounds.data()) != LDA_OK)
+        return fail(ctx, LDA_EINVAL, "chunk partition failed");
+    const int64_t kscale = S.sweep_tile_cta ? std::max<int64_t>(1, K / 1024) : 1;
+    int l2 = 0;
+    CU(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, ctx->device));
+    std::vector<int64_t> seen(V, 0);
+    size_t max_T = 1, max_rows32 = 4;
+    for (int64_t m = 0; m < M; ++m) {
+        auto c = std::make_unique<lda_stream::Chunk>();
+        const int64_t d0 = bounds[m], d1 = bounds[m + 1], t0 = doc_ptr[d0], t1 = doc_ptr[d1];
+        c->doc_begin = d0;
+        c->D = d1 - d0;
+        c->tok_begin = t0;
+        c->T = t1 - t0;
+        std::vector<int64_t> dp(c->D + 1);
+        for (int64_t d = 0; d <= c->D; ++d) dp[d] = doc_ptr[d0 + d] - t0;
+        std::vector<int64_t> wc(V, 0), cb(V);
+        lda::word_histogram(words + t0, c->T, V, ctx->threads, wc.data());
+        // canonical bases: the chunk's tokens of word w follow those of the
+        // rank's earlier chunks (documents stay in order, X18)
+        for (int32_t w = 0; w < V; ++w) {
+            cb[w] = cbase_rank[w] + seen[w];
+            seen[w] += wc[w];
+        }
+        uint64_t r32 = 4;
+        for (int64_t d = 0; d < c->D; ++d)
+            r32 += 4 * static_cast<uint64_t>((std::min<int64_t>(dp[d + 1] - dp[d], K) + 1 + 31) / 32);
+        int64_t tile = ctx->tile_tokens;
+        if (tile < 0) {
+            const double target = 0.5 * static_cast<double>(l2 > 0 ? l2 : (126 << 20));
+            tile = 32.0 * r32 <= target ? 0
+                                         : std::max<int64_t>(int64_t(1) << 20,
+                                                             static_cast<int64_t>(c->T * (target / (32.0 * r32))));
+        }
+        std::string e = lda::build_layout(dp.data(), words + t0, c->D, V, K, cb.data(), tile * kscale,
+                                          ctx->chunk_tokens, ctx->recount_tokens, ctx->threads, 2,
+                                          ctx->tail_per_tile * kscale, c->H, {}, wc.data(), /*host_tok_row=*/true);
+        if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
+        lda::HostLayout &H = c->H;
+        // every chunk adds into the same n_wk rows: all recount items accumulate
+        for (auto &rc : H.rchunks) rc.word |= 0x80000000u;
+        // page-lock the streamed host tables (async DataTransfer)
+        if (c->T) {
+            CU(cudaHostRegister(H.tok_row.data(), 4 * static_cast<size_t>(c->T), cudaHostRegisterDefault));
+            cudaError_t ce = cudaHostRegister(H.doc_map.data(), 4 * static_cast<size_t>(c->T), cudaHostRegisterDefault);
+            if (ce != cudaSuccess) {
+                cudaHostUnregister(H.tok_row.data());
+                return fail(ctx, LDA_ECUDA, std::string("cudaHostRegister: ") + cudaGetErrorString(ce));
+            }
+            c->registered = true;
+        }
+        CU(cudaMallocHost(&c->hz, 2 * std::max<size_t>(1, c->T)));
+        CU(cudaMallocHost(&c->hrows, 32 * H.rows32));
+        std::memset(c->hrows, 0, 32 * H.rows32);
+        lda::DevState &R = c->R;
+        DA(R.doc_ptr32, c->D + 1);
+        DA(R.row_off32, std::max<int64_t>(c->D, 1));
+        DA(R.segs, H.segs.size());
+        DA(R.rchunks, H.rchunks.size());
+        DA(R.titems, H.titems.size());
+        DA(R.cbase, V);
+        R.n_rchunks = static_cast<int64_t>(H.rchunks.size());
+        R.n_titems = static_cast<int64_t>(H.titems.size());
+        std::vector<uint64_t> cb64(cb.begin(), cb.end());
+        CU(cudaMemcpy(R.doc_ptr32, H.doc_ptr32.data(), 4 * (c->D + 1), cudaMemcpyHostToDevice));
+        if (c->D) CU(cudaMemcpy(R.row_off32, H.row_off32.data(), 4 * c->D, cudaMemcpyHostToDevice));
+        if (!H.segs.empty())
+            CU(cudaMemcpy(R.segs, H.segs.data(), sizeof(lda::Seg) * H.segs.size(), cudaMemcpyHostToDevice));
+        if (!H.rchunks.empty())
+            CU(cudaMemcpy(R.rchunks, H.rchunks.data(), sizeof(lda::RecountChunk) * H.rchunks.size(),
+                          cudaMemcpyHostToDevice));
+        if (!H.titems.empty())
+            CU(cudaMemcpy(R.titems, H.titems.data(), sizeof(lda::TileItem) * H.titems.size(), cudaMemcpyHostToDevice));
+        CU(cudaMemcpy(R.cbase, cb64.data(), 8 * static_cast<size_t>(V), cudaMemcpyHostToDevice));
+        max_T = std::max<size_t>(max_T, static_cast<size_t>(c->T));
+        max_rows32 = std::max<size_t>(max_rows32, H.rows32);
+        ctx->chunks.push_back(std::move(c));
+    }
+    // two device slots (chunk m+1's transfer overlaps chunk m's sweep) and the
+    // resident model
+    for (auto &b : ctx->slot) {
+        DA(b.tok_row, max_T);
+        DA(b.doc_map, max_T);
+        DA(b.z, max_T + 8);
+        DA(b.z_doc, max_T + 8);
+        DA(b.rows, 8 * max_rows32);
+        CU(cudaEventCreateWithFlags(&b.in, cudaEventDisableTiming));
+        CU(cudaEventCreateWithFlags(&b.done, cudaEventDisableTiming));
+        CU(cudaEventCreateWithFlags(&b.free_, cudaEventDisableTiming));
+    }
+    CU(cudaStreamCreateWithFlags(&ctx->h2d_stream, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&ctx->d2h_stream, cudaStreamNonBlocking));
+    for (auto &b : ctx->slot) CU(cudaEventRecord(b.free_, ctx->d2h_stream));
+    const size_t nwk_n = static_cast<size_t>(V) * K + K;
+    DA(S.nwk, nwk_n);
+    DA(S.nwk_alt, nwk_n);
+    DA(S.wtab, S.wt_bytes * static_cast<size_t>(V));
+    DA(S.denom, K);
+    DA(S.counter, 4);
+    DA(S.stat, 4);
+    DA(S.ll_part, 2 * S.ll_blocks + 2);
+    DA(S.ll_out, 2);
+    S.V = V;
+    S.K = K;
+    S.D = Dg;
+    S.T = Tg;
+    S.alpha = ctx->alpha;
+    S.beta = ctx->beta;
+    S.seed = seed;
+    S.ntiles = 0;
+    for (auto &c : ctx->chunks) S.ntiles += c->H.ntiles;
+    int launches = 0;
+    int r = chunked_rebuild(ctx, true, &launches);
+    if (r != LDA_OK) return r;
+    ctx->loaded = true;
+    ctx->sweeps = 0;
+    ctx->stats.local_tokens = Tg;
+    ctx->stats.local_docs = Dg;
+    ctx->stats.global_tokens = ctx->T_global;
+    ctx->stats.world = ctx->world;
+    int64_t items = 0;
+    for (auto &c : ctx->chunks) items += c->R.n_titems;
+    ctx->stats.n_sample_chunks = items;
+    ctx->stats.tile_tokens = ctx->tile_tokens_used;
+    ctx->stats.n_tiles = S.ntiles;
+    ctx->stats.sampler = S.sweep_tile ? 2 : 3;
+    ctx->stats.n_stream_chunks = M;
+    ctx->stats.sum_nnz_doc = ctx->cur_nnz;
+    return LDA_OK;
+}
+
+// One sweep over M streamed chunks (Alg. 1 lines 24-33): per-word tables once,
+// then for every chunk: H2D (h2d stream) -> sample + recount into the next
+// n_wk + θ rebuild (compute stream) -> D2H of z and θ (d2h stream), two slots
+// in flight; then the exchange of the accumulated counts.  E: the sweep's 8
+// events; stat: 2·M θ statistics of the sweep.
+int sweep_chunked(lda_ctx *ctx, uint32_t t, cudaEvent_t *E, unsigned long long *stat, int *launches) {
+    lda::DevState &S = ctx->S;
+    const size_t nwk_n = static_cast<size_t>(S.V) * S.K + S.K;
+    CU(cudaEventRecord(E[0], ctx->stream));
+    KL(lda::launch_sweep(S, t, ctx->stream, launches, E[6], 1));  // prologue + word tables (a2, a3)
+    CU(cudaMemsetAsync(S.nwk_alt, 0, nwk_n * sizeof(int32_t), ctx->stream));
+    const int64_t M = static_cast<int64_t>(ctx->chunks.size());
+    for (int64_t m = 0; m < M; ++m) {
+        const int sl = static_cast<int>(m & 1);
+        lda_stream::Slot &b = ctx->slot[sl];
+        CU(cudaStreamWaitEvent(ctx->h2d_stream, b.free_, 0));  // the slot's previous chunk is back on the host
+        int r = chunk_h2d(ctx, m, sl, ctx->h2d_stream, true);
+        if (r != LDA_OK) return r;
+        CU(cudaEventRecord(b.in, ctx->h2d_stream));
+        CU(cudaStreamWaitEvent(ctx->stream, b.in, 0));
+        lda::DevState v = chunk_view(ctx, m, sl);
+        KL(lda::launch_sweep(v, t, ctx->stream, launches, nullptr, 2));  // a4 against the frozen n_wk
+        lda::DevState vr = v;
+        vr.nwk = S.nwk_alt;                                              // ϕ update: accumulate
+        KL(lda::launch_recount(vr, ctx->stream, launches, 0, -1, false));
+        KL(lda::launch_theta(v, stat + 2 * m, ctx->stream, launches));   // a5
+        CU(cudaEventRecord(b.done, ctx->stream));
+        CU(cudaStreamWaitEvent(ctx->d2h_stream, b.done, 0));
+        r = chunk_d2h(ctx, m, sl, ctx->d2h_stream);
+        if (r != LDA_OK) return r;
+        CU(cudaEventRecord(b.free_, ctx->d2h_stream));
+    }
+    std::swap(S.nwk, S.nwk_alt);
+    CU(cudaEventRecord(E[1], ctx->stream));
+    CU(cudaEventRecord(E[2], ctx->stream));
+    CU(cudaEventRecord(E[3], ctx->stream));
+    if (ctx->world > 1) {
+        CU(cudaStreamWaitEvent(ctx->comm_stream, E[2], 0));
+        CU(cudaEventRecord(E[7], ctx->comm_stream));
+        COMM(allreduce_i32(S.nwk, nwk_n, ctx->comm_stream, e_));
+        CU(cudaEventRecord(E[4], ctx->comm_stream));
+        CU(cudaStreamWaitEvent(ctx->stream, E[4], 0));
+    }
+    CU(cudaEventRecord(E[5], ctx->stream));
+    return LDA_OK;
+}
+
+// LL over the chunks: the word part once (rank 0), the doc part chunk by chunk
+int chunked_loglik(lda_ctx *ctx, double h[2]) {
+    h[0] = h[1] = 0.0;
+    CU(cudaStreamSynchronize(ctx->d2h_stream));
+    for (int64_t m = 0; m < static_cast<int64_t>(ctx->chunks.size()); ++m) {
+        const lda_stream::Chunk &c = *ctx->chunks[m];
+        CU(cudaMemcpyAsync(ctx->slot[0].rows, c.hrows, 32 * c.H.rows32, cudaMemcpyHostToDevice, ctx->stream));
+        lda::DevState v = chunk_view(ctx, m, 0);
+        int launches = 0;
+        KL(lda::launch_loglik(v, m == 0 && ctx->rank == 0, ctx->stream, &launches));
+        double p[2];
+        CU(cudaMemcpyAsync(p, ctx->S.ll_out, sizeof(p), cudaMemcpyDeviceToHost, ctx->stream));
+        CU(cudaStreamSynchronize(ctx->stream));
+        h[0] += p[0];
+        h[1] += p[1];
+    }
+    return LDA_OK;
+}
+
+// LL sums (word part, doc part) of the current state, summed over the ranks
+int loglik_pair(lda_ctx *ctx, double h[2]) {
+    lda::DevState &S = ctx->S;
+    if (!ctx->chunks.empty()) {
+        int r = chunked_loglik(ctx, h);
+        if (r != LDA_OK) return r;
+        if (ctx->world > 1) {
+            CU(cudaMemcpyAsync(S.ll_out, h, 2 * sizeof(double), cudaMemcpyHostToDevice, ctx->stream));
+            COMM(allreduce_f64(S.ll_out, 2, ctx->stream, e_));
+            CU(cudaMemcpyAsync(h, S.ll_out, 2 * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+        }
+        CU(cudaStreamSynchronize(ctx->stream));
+        return LDA_OK;
+    }
+    int launches = 0;
+    KL(lda::launch_loglik(S, ctx->rank == 0, ctx->stream, &launches));
+    if (ctx->world > 1) COMM(allreduce_f64(S.ll_out, 2, ctx->stream, e_));
+    CU(cudaMemcpyAsync(h, S.ll_out, 2 * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    CU(cudaStreamSynchronize(ctx->stream));
+    return LDA_OK;
+}
+
+// option loglik_every: the LL after sweep t, outside the sweep's events (X23)
+int log_loglik(lda_ctx *ctx, uint32_t t, std::vector<int64_t> &ll_at) {
+    if (ctx->loglik_every <= 0 || t % static_cast<uint64_t>(ctx->loglik_every) != 0) return LDA_OK;
+    double h[2];
+    int r = loglik_pair(ctx, h);
+    if (r != LDA_OK) return r;
+    ll_at.push_back(static_cast<int64_t>(t));
+    ctx->ll_pending.push_back(h[0] + h[1]);
+    return LDA_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -180,8 +525,6 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
     *out = nullptr;
     if (D < 1 || V < 1 || K < 1 || K > 65536) return LDA_EINVAL;
     if (!std::isfinite(alpha) || !std::isfinite(beta) || !(alpha > 0) || !(beta > 0)) return LDA_EINVAL;
-    // u16 topic ids allow K <= 65536 (L1239-1243); this build's θ entry
-    // (topic << 18 | count) and shared-memory histograms stop at 16384
     if (K > kMaxK) return LDA_ERANGE;
     lda_ctx *c = new (std::nothrow) lda_ctx();
     if (!c) return LDA_ENOMEM;
@@ -227,6 +570,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
+    } else if (k == "stream_chunks") {
+        if (value < 1 || value > 4096) return fail(ctx, LDA_EINVAL, "stream_chunks must be in [1, 4096]");
+        ctx->stream_chunks = value;
     } else if (k == "comm_pipeline") {
         if (value < 1 || value > 64) return fail(ctx, LDA_EINVAL, "comm_pipeline must be in [1, 64]");
         ctx->comm_pipeline = value;
@@ -383,7 +729,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.exclude_self = ctx->exclude_self;
     S.sampler = ctx->sampler;
     S.certify_slack = static_cast<double>(ctx->certify_slack);
-    S.tile_fused = ctx->fused_recount != 0;
+    S.tile_fused = ctx->fused_recount != 0 && ctx->stream_chunks == 1;  // chunks: the recount kernel accumulates
     KL(lda::configure_kernels(S));
 
     lda::HostLayout &H = ctx->H;
@@ -409,6 +755,11 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     }
     ctx->tile_tokens_used = tile_tokens;
     lda::tmark("histogram, streams, configure");
+    if (ctx->stream_chunks > 1) {
+        if (!tile_layout)
+            return fail(ctx, LDA_EINVAL, "stream_chunks > 1 needs a tile sampler (2 or 3) and exclude_self = 0");
+        return load_chunked(ctx, doc_ptr, words, Dg, Tg, cbase, seed);
+    }
     // The device buffers are allocated by the copier thread below while the
     // host builds the layout (cudaMalloc of ~10 GB takes ~0.3-0.5 s, all of
     // it otherwise on the load path): first the per-token tables it copies
@@ -564,6 +915,16 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     DA(S.ll_part, 2 * S.ll_blocks + 2);
     DA(S.ll_out, 2);
     if (!S.sweep_fused) DA(S.sweep_scratch, static_cast<size_t>(S.sweep_grid) * 2 * K);
+    if (S.recount_gmem) {
+        DA(S.recount_scratch, static_cast<size_t>(S.num_sms) * 4 * 2 * K);
+        CU(cudaMemsetAsync(S.recount_scratch, 0, sizeof(int) * S.num_sms * 4 * 2 * static_cast<size_t>(K),
+                           ctx->stream));
+    }
+    if (S.theta_gmem) {
+        const size_t n = static_cast<size_t>(S.theta_grid) * (S.theta_block / 32) * (K + (K + 31) / 32);
+        DA(S.theta_scratch, n);
+        CU(cudaMemsetAsync(S.theta_scratch, 0, sizeof(uint32_t) * n, ctx->stream));
+    }
 
     auto h2d = [&](void *dst, const void *src, size_t bytes) {
         return bytes ? cudaMemcpyAsync(dst, src, bytes, cudaMemcpyHostToDevice, ctx->stream) : cudaSuccess;
@@ -608,6 +969,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     ctx->stats.tile_tokens = ctx->tile_tokens_used;
     ctx->stats.n_tiles = S.ntiles;
     ctx->stats.sampler = S.sweep_tile ? 2 : (S.sweep_tile_cta ? 3 : 0);
+    ctx->stats.n_stream_chunks = 1;
     ctx->stats.sum_nnz_doc = ctx->cur_nnz;
     return LDA_OK;
 }
@@ -626,6 +988,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         ctx->range_ev.push_back(e);
     }
+    const int64_t M = std::max<int64_t>(1, static_cast<int64_t>(ctx->chunks.size()));  // θ stats per sweep
     if (ctx->stat_log_cap < static_cast<size_t>(n)) {
         if (ctx->d_stat_log) {
             CU(cudaFree(ctx->d_stat_log));
@@ -633,13 +996,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
                                         static_cast<void *>(ctx->d_stat_log)));
             ctx->d_stat_log = nullptr;
         }
-        DA(ctx->d_stat_log, 2 * static_cast<size_t>(n));
-        if (ctx->d_ll_log) {
-            CU(cudaFree(ctx->d_ll_log));
-            ctx->allocs.erase(std::find(ctx->allocs.begin(), ctx->allocs.end(), static_cast<void *>(ctx->d_ll_log)));
-            ctx->d_ll_log = nullptr;
-        }
-        DA(ctx->d_ll_log, 2 * static_cast<size_t>(n));
+        DA(ctx->d_stat_log, 2 * static_cast<size_t>(n) * M);
         ctx->stat_log_cap = n;
     }
     std::vector<int64_t> ll_at;  // sweeps after which the LL is logged
@@ -648,6 +1005,14 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
     for (int32_t s = 0; s < n; ++s) {
         cudaEvent_t *E = ctx->ev.data() + static_cast<size_t>(per) * s;
         const uint32_t t = static_cast<uint32_t>(++ctx->sweeps);
+        if (!ctx->chunks.empty()) {
+            // f3: M > 1 chunks streamed through the device (WorkSchedule2)
+            r = sweep_chunked(ctx, t, E, ctx->d_stat_log + 2 * static_cast<size_t>(M) * s, &launches);
+            if (r != LDA_OK) return r;
+            r = log_loglik(ctx, t, ll_at);
+            if (r != LDA_OK) return r;
+            continue;
+        }
         CU(cudaEventRecord(E[0], ctx->stream));
         KL(lda::launch_sweep(S, t, ctx->stream, &launches, E[6]));
         CU(cudaEventRecord(E[1], ctx->stream));
@@ -686,33 +1051,30 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
             CU(cudaStreamWaitEvent(ctx->stream, E[4], 0));
         }
         CU(cudaEventRecord(E[5], ctx->stream));
-        if (ctx->loglik_every > 0 && t % static_cast<uint64_t>(ctx->loglik_every) == 0) {
-            // after the sweep's events: not part of its time (X23)
-            int ll_launches = 0;
-            KL(lda::launch_loglik(S, ctx->rank == 0, ctx->stream, &ll_launches));
-            if (ctx->world > 1) COMM(allreduce_f64(S.ll_out, 2, ctx->stream, e_));
-            CU(cudaMemcpyAsync(ctx->d_ll_log + 2 * ll_at.size(), S.ll_out, 2 * sizeof(double),
-                               cudaMemcpyDeviceToDevice, ctx->stream));
-            ll_at.push_back(static_cast<int64_t>(t));
-        }
+        r = log_loglik(ctx, t, ll_at);
+        if (r != LDA_OK) return r;
     }
     CU(cudaStreamSynchronize(ctx->stream));
-    {
-        std::vector<double> hl(2 * ll_at.size());
-        if (!hl.empty())
-            CU(cudaMemcpy(hl.data(), ctx->d_ll_log, hl.size() * sizeof(double), cudaMemcpyDeviceToHost));
-        ctx->ll_sweep = ll_at;
-        ctx->ll_value.assign(ll_at.size(), 0.0);
-        for (size_t i = 0; i < ll_at.size(); ++i)
-            ctx->ll_value[i] = (hl[2 * i] + hl[2 * i + 1]) / static_cast<double>(ctx->T_global > 0 ? ctx->T_global : 1);
-    }
+    if (ctx->h2d_stream) CU(cudaStreamSynchronize(ctx->h2d_stream));
+    if (ctx->d2h_stream) CU(cudaStreamSynchronize(ctx->d2h_stream));
+    ctx->ll_sweep = ll_at;
+    ctx->ll_value.assign(ll_at.size(), 0.0);
+    for (size_t i = 0; i < ll_at.size(); ++i)
+        ctx->ll_value[i] = ctx->ll_pending[i] / static_cast<double>(ctx->T_global > 0 ? ctx->T_global : 1);
+    ctx->ll_pending.clear();
     unsigned long long n_exact = 0;
     CU(cudaMemcpy(&n_exact, S.stat + 2, sizeof(n_exact), cudaMemcpyDeviceToHost));
     ctx->stats.n_exact_redraws = static_cast<int64_t>(n_exact);
     std::vector<unsigned long long> hs(2 * static_cast<size_t>(n));
-    if (n)
-        CU(cudaMemcpy(hs.data(), ctx->d_stat_log, hs.size() * sizeof(unsigned long long),
-                      cudaMemcpyDeviceToHost));
+    if (n) {
+        std::vector<unsigned long long> hm(2 * static_cast<size_t>(n) * M);
+        CU(cudaMemcpy(hm.data(), ctx->d_stat_log, hm.size() * sizeof(unsigned long long), cudaMemcpyDeviceToHost));
+        for (size_t i = 0; i < static_cast<size_t>(n); ++i)
+            for (int64_t m = 0; m < M; ++m) {
+                hs[2 * i] += hm[2 * (i * M + m)];
+                hs[2 * i + 1] += hm[2 * (i * M + m) + 1];
+            }
+    }
     lda_stats &st = ctx->stats;
     st.last_n = n;
     st.sweeps_done = static_cast<int64_t>(ctx->sweeps);
@@ -815,12 +1177,9 @@ int lda_loglik(lda_ctx *ctx, double *ll) {
     if (!ll) return fail(ctx, LDA_EINVAL, "null output");
     if (!ctx->loaded) return fail(ctx, LDA_ESTATE, "no corpus loaded");
     CU(cudaSetDevice(ctx->device));
-    int launches = 0;
-    KL(lda::launch_loglik(ctx->S, ctx->rank == 0, ctx->stream, &launches));
-    if (ctx->world > 1) COMM(allreduce_f64(ctx->S.ll_out, 2, ctx->stream, e_));
     double h[2];
-    CU(cudaMemcpyAsync(h, ctx->S.ll_out, sizeof(h), cudaMemcpyDeviceToHost, ctx->stream));
-    CU(cudaStreamSynchronize(ctx->stream));
+    int r = loglik_pair(ctx, h);
+    if (r != LDA_OK) return r;
     *ll = (h[0] + h[1]) / static_cast<double>(ctx->T_global > 0 ? ctx->T_global : 1);
     return LDA_OK;
 }
@@ -837,23 +1196,46 @@ int lda_get_counts(lda_ctx *ctx, int32_t *n_wk, int32_t *n_k, int64_t *ndk_ptr, 
     if (n_k) CU(cudaMemcpy(n_k, S.nwk + static_cast<size_t>(S.V) * S.K, sizeof(int32_t) * S.K,
                            cudaMemcpyDeviceToHost));
     if (ndk_ptr || ndk_topic || ndk_count || ndk_nnz_out) {
-        std::vector<uint32_t> rows(H.rows32 * 8);
-        CU(cudaMemcpy(rows.data(), S.rows, rows.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+        // θ rows: the device copy, or (M > 1 chunks) the chunks' host copies
+        struct Src {
+            const uint32_t *rows;
+            const std::vector<uint32_t> *off;
+            int64_t D;
+        };
+        std::vector<Src> src;
+        std::vector<uint32_t> rows;
+        if (ctx->chunks.empty()) {
+            rows.resize(H.rows32 * 8);
+            CU(cudaMemcpy(rows.data(), S.rows, rows.size() * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+            src.push_back({rows.data(), &H.row_off32, S.D});
+        } else {
+            if (ctx->d2h_stream) CU(cudaStreamSynchronize(ctx->d2h_stream));
+            for (auto &c : ctx->chunks) src.push_back({c->hrows, &c->H.row_off32, c->D});
+        }
         int64_t nnz = 0;
-        for (int64_t d = 0; d < S.D; ++d) nnz += rows[static_cast<size_t>(H.row_off32[d]) * 8];
+        for (const Src &q : src)
+            for (int64_t d = 0; d < q.D; ++d) nnz += q.rows[static_cast<size_t>((*q.off)[d]) * 8];
         if (ndk_nnz_out) *ndk_nnz_out = nnz;
         if ((ndk_topic || ndk_count) && ndk_capacity < nnz)
             return fail(ctx, LDA_ERANGE, "ndk_capacity smaller than nnz");
-        int64_t pos = 0;
-        for (int64_t d = 0; d < S.D; ++d) {
-            const uint32_t *row = rows.data() + static_cast<size_t>(H.row_off32[d]) * 8;
-            if (ndk_ptr) ndk_ptr[d] = pos;
-            for (uint32_t j = 0; j < row[0]; ++j, ++pos) {
-                if (ndk_topic) ndk_topic[pos] = static_cast<uint16_t>(row[1 + j] >> 18);
-                if (ndk_count) ndk_count[pos] = static_cast<int32_t>(row[1 + j] & 0xFFFFu);
+        int64_t pos = 0, dg = 0;
+        for (const Src &q : src)
+            for (int64_t d = 0; d < q.D; ++d, ++dg) {
+                const uint32_t *row = q.rows + static_cast<size_t>((*q.off)[d]) * 8;
+                if (ndk_ptr) ndk_ptr[dg] = pos;
+                for (uint32_t j = 0; j < row[0]; ++j, ++pos) {
+                    if (ndk_topic) ndk_topic[pos] = static_cast<uint16_t>(row[1 + j] >> (S.K > 16384 ? 16 : 18));
+                    if (ndk_count) ndk_count[pos] = static_cast<int32_t>(row[1 + j] & 0xFFFFu);
+                }
             }
-        }
-        if (ndk_ptr) ndk_ptr[S.D] = pos;
+        if (ndk_ptr) ndk_ptr[dg] = pos;
+    }
+    if (z && S.T && !ctx->chunks.empty()) {
+        // M > 1: the chunks' word-major host copies, into document order
+        if (ctx->d2h_stream) CU(cudaStreamSynchronize(ctx->d2h_stream));
+        for (auto &c : ctx->chunks)
+            for (int64_t i = 0; i < c->T; ++i) z[c->tok_begin + i] = c->hz[c->H.doc_map[i]];
+        return LDA_OK;
     }
     if (z && S.T) {
         // z into document order on the device (the θ rebuild's gather), then D2H
@@ -878,6 +1260,14 @@ int lda_set_z(lda_ctx *ctx, const uint16_t *z) {
     for (int64_t i = 0; i < S.T; ++i)
         if (z[i] >= S.K) return fail(ctx, LDA_EINVAL, "topic id >= K");
     CU(cudaSetDevice(ctx->device));
+    if (!ctx->chunks.empty()) {
+        // M > 1: into the chunks' word-major host copies, then the rebuild
+        CU(cudaStreamSynchronize(ctx->d2h_stream));
+        for (auto &c : ctx->chunks)
+            for (int64_t i = 0; i < c->T; ++i) c->hz[c->H.doc_map[i]] = z[c->tok_begin + i];
+        int launches = 0;
+        return chunked_rebuild(ctx, false, &launches);
+    }
     if (S.T) {
         // H2D in document order, scattered to word-major positions on the device
         uint16_t *zd = nullptr;
@@ -915,6 +1305,23 @@ void lda_destroy(lda_ctx *ctx) {
     if (ctx->stream || !ctx->allocs.empty()) {
         cudaSetDevice(ctx->device);
         if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+        for (cudaStream_t st : {ctx->h2d_stream, ctx->d2h_stream})
+            if (st) {
+                cudaStreamSynchronize(st);
+                cudaStreamDestroy(st);
+            }
+        for (auto &b : ctx->slot)
+            for (cudaEvent_t e : {b.in, b.done, b.free_})
+                if (e) cudaEventDestroy(e);
+        for (auto &c : ctx->chunks) {
+            if (c->registered) {
+                cudaHostUnregister(c->H.tok_row.data());
+                cudaHostUnregister(c->H.doc_map.data());
+            }
+            if (c->hz) cudaFreeHost(c->hz);
+            if (c->hrows) cudaFreeHost(c->hrows);
+        }
+        ctx->chunks.clear();
         for (void *p : ctx->allocs) cudaFree(p);
         for (cudaEvent_t e : ctx->ev) cudaEventDestroy(e);
         for (cudaEvent_t e : ctx->range_ev) cudaEventDestroy(e);

@@ -29,8 +29,11 @@ namespace lda {
 constexpr unsigned kFull = 0xffffffffu;
 // θ row entry: topic << kTS | count (count < 2^16 in bits 0-15, bits 16-17
 // zero), so that e >> 16 is the byte offset 4·topic of the topic in an fp32
-// table.  K <= 16384 (14 topic bits).
+// table.  K <= 16384 (14 topic bits).  Wide entries for 16384 < K <= 65536
+// (u16 topic ids, L1239-1243): topic << kTSWide | count (sampler 0 only).
 constexpr int kTS = 18;
+constexpr int kTSWide = 16;
+__host__ __device__ constexpr int entry_shift(int K) { return K > 16384 ? kTSWide : kTS; }
 constexpr int kSweepThreads = 256;
 constexpr int kMaxBlk = 16;  // block-end prefixes kept per token for the sparse rescan
 #ifndef LDA_RING
@@ -85,6 +88,66 @@ __device__ __forceinline__ uint4 ld_nc_v4(const uint4 *p) {
     return v;
 }
 
+// L2 residency hints of the tile samplers (createpolicy + .L2::cache_hint):
+// θ rows evict_last, the once-per-tile streams (tok_row, the per-item word
+// tables) evict_first.  Measured on B200 at PubMed shape: 2.5 % SLOWER
+// (policy registers at the 128-register limit; the kernel is bound by
+// issue and load latency, not by DRAM bandwidth) -- off by default.
+#ifndef LDA_L2HINT
+#define LDA_L2HINT 0
+#endif
+#ifndef LDA_WALK2
+#define LDA_WALK2 1
+#endif
+#ifndef LDA_HOOK
+#define LDA_HOOK 0
+#endif
+__device__ __forceinline__ uint64_t pol_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t pol_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// a θ row line block (kept in L2)
+__device__ __forceinline__ Blk8 ld_row_v8(const uint32_t *p) {
+#if LDA_L2HINT
+    Blk8 b;
+    asm volatile("ld.global.nc.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+                 : "=r"(b.w[0]), "=r"(b.w[1]), "=r"(b.w[2]), "=r"(b.w[3]), "=r"(b.w[4]), "=r"(b.w[5]),
+                   "=r"(b.w[6]), "=r"(b.w[7])
+                 : "l"(p), "l"(pol_evict_last()));
+    return b;
+#else
+    return ld_nc_v8(p);
+#endif
+}
+// a θ row header word (kept in L2)
+__device__ __forceinline__ uint32_t ld_row_u32(const uint32_t *p) {
+#if LDA_L2HINT
+    uint32_t v;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol_evict_last()));
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+// a streamed word (tok_row: read once per sweep)
+__device__ __forceinline__ uint32_t ld_stream_u32(const uint32_t *p) {
+#if LDA_L2HINT
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"
+                 : "=r"(v)
+                 : "l"(p), "l"(pol_evict_first()));
+    return v;
+#else
+    return __ldg(p);
+#endif
+}
+
 // Bring the 32-byte sector at p into L2 (no register, no scoreboard).
 __device__ __forceinline__ void prefetch_l2(const void *p) {
     asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
@@ -94,6 +157,16 @@ __device__ __forceinline__ void prefetch_l2(const void *p) {
 // bulk-prefetch instruction per θ row; bytes a multiple of 16).
 __device__ __forceinline__ void prefetch_l2_bulk(const void *p, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+}
+// ... for a word table (streamed: evict_first)
+__device__ __forceinline__ void prefetch_l2_table(const void *p, uint32_t bytes) {
+#if LDA_L2HINT
+    asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p), "r"(bytes),
+                 "l"(pol_evict_first())
+                 : "memory");
+#else
+    prefetch_l2_bulk(p, bytes);
+#endif
 }
 
 // Word-major position of virtual index v of a word whose item spans runs
@@ -201,12 +274,12 @@ __device__ __forceinline__ uint32_t philox_x0_sched(uint64_t c, uint32_t t, cons
     return c0;
 }
 
-template <bool EXCL>
+template <bool EXCL, int TS>
 struct Mass {
-    // mass of one θ entry e = topic << 18 | count under the word's p*
+    // mass of one θ entry e = topic << TS | count under the word's p*
     __device__ __forceinline__ static double fma_into(uint32_t e, const double *__restrict__ pstar, int zo,
                                                       double po_new, double acc) {
-        const uint32_t tp = e >> kTS;
+        const uint32_t tp = e >> TS;
         uint32_t cn = e & 0xFFFFu;
         double p = pstar[tp];
         if (EXCL && static_cast<int>(tp) == zo && cn != 0u) {
@@ -219,7 +292,7 @@ struct Mass {
 
 // SMEMP: p*/P in shared memory (LDS addressing); else in a global scratch
 // slice per CTA (large K).
-template <bool EXCL, bool SMEMP>
+template <bool EXCL, bool SMEMP, int TS = kTS>
 __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(SweepArgs a) {
     extern __shared__ double smem_d[];
     __shared__ int s_ci;
@@ -319,7 +392,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
             // pass 1: S over the row, block-end prefixes to smem
             double S = 0.0;
 #pragma unroll
-            for (int e = 1; e < 8; ++e) S = Mass<EXCL>::fma_into(q[0].w[e], pstar, zo, po_new, S);
+            for (int e = 1; e < 8; ++e) S = Mass<EXCL, TS>::fma_into(q[0].w[e], pstar, zo, po_new, S);
             blkC[tid] = S;
             if (static_cast<uint32_t>(kRing) < nblk) q[0] = ld_nc_v8(rw + 8 * kRing);
             // blocks 1 .. nblk-1, ring slot (b % kRing)
@@ -333,7 +406,7 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                     const uint32_t nx = b + kRing;
                     if (nx < nblk) q[i] = ld_nc_v8(rw + 8 * nx);
 #pragma unroll
-                    for (int e = 0; e < 8; ++e) S = Mass<EXCL>::fma_into(u.w[e], pstar, zo, po_new, S);
+                    for (int e = 0; e < 8; ++e) S = Mass<EXCL, TS>::fma_into(u.w[e], pstar, zo, po_new, S);
                     if (b < kMaxBlk) blkC[b * kSweepThreads + tid] = S;
                 }
             }
@@ -349,8 +422,8 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
                 z = -1;
 #define LDA_STEP(e)                                                   \
     {                                                                 \
-        C = Mass<EXCL>::fma_into((e), pstar, zo, po_new, C);          \
-        if (z < 0 && C > x) z = static_cast<int>((e) >> kTS);          \
+        C = Mass<EXCL, TS>::fma_into((e), pstar, zo, po_new, C);      \
+        if (z < 0 && C > x) z = static_cast<int>((e) >> TS);           \
     }
                 for (; z < 0 && b < nblk; ++b) {  // one block, or a linear tail past kMaxBlk
                     const Blk8 u = ld_nc_v8(rw + 8 * b);
@@ -481,7 +554,6 @@ struct TileArgs {
     uint32_t wt_bytes;
     int nbuf;                  // sweep_tile_cta_kernel: table buffers per CTA
     int recount;               // 1: the ϕ update fused here; 0: recount_kernel after the sweep
-    uint32_t zero_line;        // offset (32-byte units) of an all-zero 128-byte line of `rows`
     uint32_t t;
     uint32_t key0[10], key1[10];
 };
@@ -704,11 +776,20 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
 // Bulk copy (TMA engine, no LSU wavefronts) global -> this CTA's smem,
 // completion counted on the mbarrier.
 __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, uint64_t *bar) {
+#if LDA_L2HINT
+    // word tables are streamed (read once per tile): evict_first in L2
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], "
+        "%4;" ::"r"(smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol_evict_first())
+        : "memory");
+#else
     asm volatile(
         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
             smem_u32(dst)),
         "l"(src), "r"(bytes), "r"(smem_u32(bar))
         : "memory");
+#endif
 }
 
 // Per-warp shared memory of the tile sampler (bytes): the word table, block
@@ -751,8 +832,9 @@ __device__ __forceinline__ TileHead tile_head(const TileArgs &a, uint32_t row, u
     const unsigned heads = __ballot_sync(kFull, !h.dup);
     const int hl = 31 - __clz(heads & (0xFFFFFFFFu >> (31 - lane)));
     h.c0 = __shfl_sync(kFull, c0, hl);
-    if (h.take && !h.dup)
+    if (h.take && !h.dup) {
         for (uint32_t i = 0; i < h.nl; ++i) lrow[h.c0 + i] = (row + 4u * i) | (i == 0 ? 0x80000000u : 0u);
+    }
     __syncwarp();
 #pragma unroll
     for (int s2 = 0; s2 < R; ++s2) {
@@ -762,7 +844,7 @@ __device__ __forceinline__ TileHead tile_head(const TileArgs &a, uint32_t row, u
         hdr[s2] = false;
         if (L < h.lsum) {
             const uint32_t lr = lrow[L];
-            ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+            ring[s2] = ld_row_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
             hdr[s2] = sub == 0 && (lr >> 31);
         }
     }
@@ -780,10 +862,46 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
     const int lane = threadIdx.x & 31, q = lane >> 2, sub = lane & 3;
     bool hooked = false;
     for (uint32_t base = 0; base < lsum; base += 8u * R) {
+#if LDA_HOOK == 1
+        // the caller's prefetch hook at the start of the last step (after step 1)
+        if (base > 0 && base + 8u * R >= lsum) {
+#else
         if (base == 8u * R) {
+#endif
             at_step2();
             hooked = true;
         }
+#if LDA_WALK2
+        // slot by slot: sum the slot's line, refill the slot for the next
+        // step at once (its load then has the other slots' work to land),
+        // then the slot's line sum
+#pragma unroll
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
+            float s0 = count_f32(w0) * tab32(p32, w0);
+            float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
+            s0 = entry_mass32(ring[s2].w[2], p32, s0);
+            s1 = entry_mass32(ring[s2].w[3], p32, s1);
+            s0 = entry_mass32(ring[s2].w[4], p32, s0);
+            s1 = entry_mass32(ring[s2].w[5], p32, s1);
+            s0 = entry_mass32(ring[s2].w[6], p32, s0);
+            s1 = entry_mass32(ring[s2].w[7], p32, s1);
+            const float bs = s0 + s1;
+            const uint32_t Ln = base + 8u * (s2 + R) + q;
+            if (Ln < lsum) {
+                const uint32_t lr = lrow[Ln];
+                ring[s2] = ld_row_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+                hdr[s2] = sub == 0 && (lr >> 31);
+            }
+            const uint32_t L = base + 8u * s2 + q;
+            float ls = bs + __shfl_xor_sync(kFull, bs, 1);
+            ls += __shfl_xor_sync(kFull, ls, 2);
+            if (L < lsum) {
+                blk[4 * L + sub] = bs;
+                if (sub == 0) lsm[L] = ls;
+            }
+        }
+#else
         float bs[R];
 #pragma unroll
         for (int s2 = 0; s2 < R; ++s2) {
@@ -798,16 +916,12 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
             s1 = entry_mass32(ring[s2].w[7], p32, s1);
             bs[s2] = s0 + s1;
         }
-        // refill for the next step (if any): a quad past the batch's last
-        // line loads the all-zero line instead, so that its lookups go to
-        // p32[0] (one broadcast) rather than to the stale entries' random
-        // topics (bank conflicts)
-        if (base + 8u * R < lsum) {
 #pragma unroll
-            for (int s2 = 0; s2 < R; ++s2) {
-                const uint32_t Ln = base + 8u * (s2 + R) + q;
-                const uint32_t lr = Ln < lsum ? lrow[Ln] : a.zero_line;
-                ring[s2] = ld_nc_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
+        for (int s2 = 0; s2 < R; ++s2) {
+            const uint32_t Ln = base + 8u * (s2 + R) + q;
+            if (Ln < lsum) {
+                const uint32_t lr = lrow[Ln];
+                ring[s2] = ld_row_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
                 hdr[s2] = sub == 0 && (lr >> 31);
             }
         }
@@ -821,6 +935,7 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
                 if (sub == 0) lsm[L] = ls;
             }
         }
+#endif
     }
     if (!hooked) at_step2();
 }
@@ -881,7 +996,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             // first e with local prefix s_e > r; certify s_{e-1}, s_e
             const float r32 = static_cast<float>(x - C);
             const float eR = static_cast<float>((eX + gS * C + u * (x - C)) * 1.0001 + 1e-30);
-            Blk8 w = ld_nc_v8(a.rows + (static_cast<size_t>(row) + b) * 8);
+            Blk8 w = ld_row_v8(a.rows + (static_cast<size_t>(row) + b) * 8);
             if (b == 0) w.w[0] = 0u;
             float sl = 0.0f, sp = 0.0f, se = 0.0f;
             int ez = -1;
@@ -1055,7 +1170,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
     uint32_t cn = ci != 0xFFFFFFFFu ? claim() : 0xFFFFFFFFu;
     TileItem itn = cn < a.n_items ? a.items[cn] : none;
     if (lane == 0 && cn < a.n_items && itn.word != it.word)
-        prefetch_l2_bulk(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
+        prefetch_l2_table(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
     // Batch head (up to 32 tokens whose θ rows have at most LM lines in
     // total; consecutive tokens of one document -- a (word, doc) pair --
     // share the walk of its row): line table in smem, first R lines of the
@@ -1069,9 +1184,9 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
     // the first batch
     uint32_t row = 0, crank = 0, nnz = 0;
     if (lane < it.n) {
-        row = __ldg(a.tok_row + it.pos + lane);
+        row = ld_stream_u32(a.tok_row + it.pos + lane);
         crank = it.crank0 + lane;
-        nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
+        nnz = ld_row_u32(a.rows + static_cast<size_t>(row) * 8);
     }
     TileHead hd = head(row, nnz, static_cast<uint32_t>(lane) < it.n);
     uint32_t b0 = 0;
@@ -1115,10 +1230,10 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         const bool nxt_valid = static_cast<uint32_t>(lane) < nxt_n;
         uint32_t n_row = 0, n_nnz = 0;
         const uint32_t n_crank = (more ? it.crank0 + b1 : itn.crank0) + lane;
-        if (nxt_valid) n_row = __ldg(a.tok_row + nxt_pos + lane);
+        if (nxt_valid) n_row = ld_stream_u32(a.tok_row + nxt_pos + lane);
         // ---- walk (the next batch's row headers issued after its first step)
         tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, lsm, [&] {
-            if (nxt_valid) n_nnz = __ldg(a.rows + static_cast<size_t>(n_row) * 8);
+            if (nxt_valid) n_nnz = ld_row_u32(a.rows + static_cast<size_t>(n_row) * 8);
         });
         __syncwarp();
         // ---- the next batch's head: its line table and first lines, in flight during this draw
@@ -1150,7 +1265,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
             cn = claim();
             itn = cn < a.n_items ? a.items[cn] : none;
             if (lane == 0 && cn < a.n_items && itn.word != it.word)
-                prefetch_l2_bulk(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
+                prefetch_l2_table(a.wtab + static_cast<size_t>(itn.word) * a.wt_bytes, a.wt_bytes);
         }
     }
     __syncthreads();
@@ -1271,9 +1386,9 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
                 const uint32_t p = it.pos + b0 + lane;
                 uint32_t row = 0, crank = 0, nnz = 0;
                 if (valid) {
-                    row = __ldg(a.tok_row + p);
+                    row = ld_stream_u32(a.tok_row + p);
                     crank = it.crank0 + b0 + lane;
-                    nnz = __ldg(a.rows + static_cast<size_t>(row) * 8);
+                    nnz = ld_row_u32(a.rows + static_cast<size_t>(row) * 8);
                 }
                 const TileHead hd = tile_head<R>(a, row, nnz, valid, LM, lrow, ring, hdr);
                 tile_walk<R>(a, hd.lsum, lrow, ring, hdr, p32, blk, lsm, [] {});
@@ -1337,15 +1452,19 @@ __global__ void zero_rows_kernel(const int32_t *__restrict__ words, int64_t n, i
 // (each run contiguous in the word-major stream: coalesced z reads, no
 // per-token search), then writes the word's row of n_wk (global atomics only
 // for words split over several items) and accumulates n_k.
+// GMEM (K > 16384): the CTA's two K-length histograms in a global scratch
+// slice (zero on entry, left zero on exit) instead of shared memory.
+template <bool GMEM>
 __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc,
                                const Seg *__restrict__ segs, int K, const uint16_t *__restrict__ z,
                                int32_t *__restrict__ nwk, int32_t *__restrict__ nk,
-                               uint32_t *__restrict__ counter) {
+                               uint32_t *__restrict__ counter, int *__restrict__ gscratch) {
     extern __shared__ int smem_i[];
-    int *hist = smem_i, *nkp = smem_i + K;
+    int *hist = GMEM ? gscratch + static_cast<size_t>(blockIdx.x) * 2 * K : smem_i, *nkp = hist + K;
     __shared__ int s_ci;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarps = blockDim.x >> 5;
-    for (int k = threadIdx.x; k < 2 * K; k += blockDim.x) smem_i[k] = 0;
+    if (!GMEM)
+        for (int k = threadIdx.x; k < 2 * K; k += blockDim.x) smem_i[k] = 0;
     __syncthreads();
     for (;;) {
         if (threadIdx.x == 0) s_ci = static_cast<int>(atomicAdd(counter, 1u));
@@ -1379,7 +1498,10 @@ __global__ void recount_kernel(const RecountChunk *__restrict__ rc, int64_t n_rc
         __syncthreads();
     }
     for (int k = threadIdx.x; k < K; k += blockDim.x)
-        if (nkp[k]) atomicAdd(nk + k, nkp[k]);
+        if (nkp[k]) {
+            atomicAdd(nk + k, nkp[k]);
+            if (GMEM) nkp[k] = 0;
+        }
 }
 
 // ---------------------------------------------------------------------------
@@ -1419,16 +1541,21 @@ __global__ void scatter_z_kernel(const uint32_t *__restrict__ doc_map, const uin
 }
 
 // Phase B: zd is z in document order (gather_z_kernel).
+// GMEM (K > 16384): the warp's histogram + bitmap in a global scratch slice
+// (zero on entry, left zero) instead of shared memory; TS: entry shift.
+template <bool GMEM, int TS>
 __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
                              const uint16_t *__restrict__ zd,
                              uint32_t *__restrict__ rows, int64_t D, int K,
-                             unsigned long long *__restrict__ stat) {
+                             unsigned long long *__restrict__ stat, uint32_t *__restrict__ gscratch) {
     extern __shared__ uint32_t smem_u[];
     const int Kw = (K + 31) >> 5;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;
-    uint32_t *cnt = smem_u + static_cast<size_t>(warp) * (K + Kw);
+    uint32_t *cnt = (GMEM ? gscratch + static_cast<size_t>(blockIdx.x) * wpb * (K + Kw) : smem_u) +
+                    static_cast<size_t>(warp) * (K + Kw);
     uint32_t *bits = cnt + K;
-    for (int k = lane; k < K + Kw; k += 32) cnt[k] = 0u;
+    if (!GMEM)
+        for (int k = lane; k < K + Kw; k += 32) cnt[k] = 0u;
     __syncwarp();
     unsigned long long s_lnnz = 0, s_nnz = 0;
     const int64_t nw = static_cast<int64_t>(gridDim.x) * wpb;
@@ -1482,7 +1609,7 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
                 const int b = __ffs(bw) - 1;
                 bw &= bw - 1;
                 const uint32_t k = static_cast<uint32_t>(qq) * 32 + b;
-                row[1 + pos++] = (k << kTS) | cnt[k];
+                row[1 + pos++] = (k << TS) | cnt[k];
                 cnt[k] = 0u;
             }
             if (qq < Kw) bits[qq] = 0u;
@@ -1585,7 +1712,8 @@ __host__ __device__ inline size_t peer_slice_lo(size_t n, int world, int q, size
 }
 
 template <class T>
-__global__ void peer_rs_kernel(PeerPtrs src, int world, T *__restrict__ own, size_t lo, size_t hi) {
+__global__ void peer_rs_kernel(const __grid_constant__ PeerPtrs src, int world, T *__restrict__ own, size_t lo,
+                               size_t hi) {
     constexpr int VW = 16 / sizeof(T);
     const size_t nv = (hi - lo) / VW;
     const size_t stride = static_cast<size_t>(gridDim.x) * blockDim.x;
@@ -1679,7 +1807,11 @@ int configure_kernels(DevState &s) {
         s.sweep_smem = smemp ? want : blk;
         s.sweep_fused = smemp;
         const void *fn = nullptr;
-        if (s.exclude_self)
+        const bool wide = s.K > 16384;  // wide θ entries; p*/P never fit in smem there
+        if (wide)
+            fn = s.exclude_self ? reinterpret_cast<const void *>(&sweep_kernel<true, false, kTSWide>)
+                                : reinterpret_cast<const void *>(&sweep_kernel<false, false, kTSWide>);
+        else if (s.exclude_self)
             fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<true, true>)
                        : reinterpret_cast<const void *>(&sweep_kernel<true, false>);
         else
@@ -1768,25 +1900,34 @@ int configure_kernels(DevState &s) {
             s.sweep_fused = s.tile_fused;
         }
     }
-    // recount
-    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&recount_kernel),
+    // recount: two K-length histograms per CTA in shared memory, or (wide K)
+    // in a global scratch slice per CTA
+    s.recount_gmem = static_cast<size_t>(8) * s.K + 1024 > static_cast<size_t>(max_optin);
+    if (!s.recount_gmem &&
+        (e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&recount_kernel<false>),
                                   cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) != cudaSuccess)
         return e;
-    // theta: as many warps per block (<= 8) as fit
+    // theta: as many warps per block (<= 8) as fit; wide K: per-warp global scratch
     size_t per_warp = static_cast<size_t>(4) * (s.K + (s.K + 31) / 32);
     int wpb = static_cast<int>(std::min<size_t>(8, (static_cast<size_t>(max_optin) - 1024) / per_warp));
-    if (wpb < 1) return cudaErrorInvalidValue;
-    s.theta_block = 32 * wpb;
-    s.theta_smem = per_warp * wpb;
-    if ((e = cudaFuncSetAttribute(reinterpret_cast<const void *>(&theta_kernel),
-                                  cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  static_cast<int>(s.theta_smem))) != cudaSuccess)
-        return e;
-    int tb = 1;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, reinterpret_cast<const void *>(&theta_kernel),
-                                                           s.theta_block, s.theta_smem)) != cudaSuccess)
-        return e;
-    s.theta_grid = s.num_sms * (tb > 0 ? tb : 1);
+    s.theta_gmem = wpb < 1;
+    if (s.theta_gmem) {
+        s.theta_block = 256;
+        s.theta_smem = 0;
+        s.theta_grid = s.num_sms * 4;
+    } else {
+        s.theta_block = 32 * wpb;
+        s.theta_smem = per_warp * wpb;
+        const void *tf = s.K > 16384 ? reinterpret_cast<const void *>(&theta_kernel<false, kTSWide>)
+                                     : reinterpret_cast<const void *>(&theta_kernel<false, kTS>);
+        if ((e = cudaFuncSetAttribute(tf, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      static_cast<int>(s.theta_smem))) != cudaSuccess)
+            return e;
+        int tb = 1;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, tf, s.theta_block, s.theta_smem)) != cudaSuccess)
+            return e;
+        s.theta_grid = s.num_sms * (tb > 0 ? tb : 1);
+    }
     s.ll_blocks = 2 * s.num_sms;
     return cudaSuccess;
 }
@@ -1825,8 +1966,12 @@ int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0, 
     if (rc1 <= rc0) return cudaGetLastError();
     if ((e = cudaMemsetAsync(s.counter + 1, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
     const int grid = static_cast<int>(std::min<int64_t>(rc1 - rc0, static_cast<int64_t>(s.num_sms) * 4));
-    recount_kernel<<<grid, 256, 8 * s.K, st>>>(s.rchunks + rc0, rc1 - rc0, s.segs, s.K, s.tok_z, s.nwk, nk,
-                                               s.counter + 1);
+    if (s.recount_gmem)
+        recount_kernel<true><<<grid, 256, 0, st>>>(s.rchunks + rc0, rc1 - rc0, s.segs, s.K, s.tok_z, s.nwk, nk,
+                                                  s.counter + 1, s.recount_scratch);
+    else
+        recount_kernel<false><<<grid, 256, 8 * s.K, st>>>(s.rchunks + rc0, rc1 - rc0, s.segs, s.K, s.tok_z, s.nwk,
+                                                          nk, s.counter + 1, nullptr);
     ++*launches;
     return cudaGetLastError();
 }
@@ -1861,19 +2006,28 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
         gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, st>>>(s.doc_map, s.tok_z, s.z_doc, s.T);
         ++*launches;
     }
-    theta_kernel<<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(s.doc_ptr32, s.row_off32, s.z_doc, s.rows, s.D,
-                                                                   s.K, stat_out);
+    if (s.theta_gmem)
+        theta_kernel<true, kTSWide><<<s.theta_grid, s.theta_block, 0, st>>>(s.doc_ptr32, s.row_off32, s.z_doc, s.rows,
+                                                                           s.D, s.K, stat_out, s.theta_scratch);
+    else if (s.K > 16384)
+        theta_kernel<false, kTSWide><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(
+            s.doc_ptr32, s.row_off32, s.z_doc, s.rows, s.D, s.K, stat_out, nullptr);
+    else
+        theta_kernel<false, kTS><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(
+            s.doc_ptr32, s.row_off32, s.z_doc, s.rows, s.D, s.K, stat_out, nullptr);
     ++*launches;
     return cudaGetLastError();
 }
 
-int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event) {
+int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event, int parts) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     const double Vbeta = static_cast<double>(s.V) * s.beta;
     const int32_t *nk = s.nwk + static_cast<size_t>(s.V) * s.K;
-    prologue_kernel<<<(s.K + 255) / 256, 256, 0, st>>>(nk, s.K, Vbeta, s.denom);
-    ++*launches;
+    if (parts & 1) {
+        prologue_kernel<<<(s.K + 255) / 256, 256, 0, st>>>(nk, s.K, Vbeta, s.denom);
+        ++*launches;
+    }
     if (!s.sweep_tile && !s.sweep_tile_cta && table_done_event &&
         (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
         return e;
@@ -1895,13 +2049,15 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
     }
     if (s.sweep_tile || s.sweep_tile_cta) {
         // every row of the next n_wk is accumulated (words span tiles)
-        if (s.tile_fused &&
+        if ((parts & 1) && s.tile_fused &&
             (e = cudaMemsetAsync(s.nwk_alt, 0, sizeof(int32_t) * (static_cast<size_t>(s.V) * s.K + s.K), st)) !=
                 cudaSuccess)
             return e;
         const int wtb = static_cast<int>(std::min<int64_t>((static_cast<int64_t>(s.V) + 7) / 8, 8 * s.num_sms));
         const bool compact = s.sweep_tile_cta && s.tile_cta_gnk;
-        if ((s.K & 3) == 0 && compact)
+        if (!(parts & 1)) {
+            // the tables of this sweep are built (out-of-HBM chunks after the first)
+        } else if ((s.K & 3) == 0 && compact)
             word_table_kernel<true, true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
                                                                      s.wtab);
         else if (compact)
@@ -1913,9 +2069,10 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         else
             word_table_kernel<false, false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
                                                                        s.wtab);
-        ++*launches;
+        if (parts & 1) ++*launches;
         if (table_done_event && (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
             return e;
+        if (!(parts & 2)) return cudaGetLastError();
         TileArgs ta;
         ta.items = s.titems;
         ta.n_items = s.n_titems;
@@ -1938,7 +2095,6 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
         ta.nbuf = s.tile_nbuf;
         ta.recount = s.tile_fused ? 1 : 0;
-        ta.zero_line = static_cast<uint32_t>(s.rows32 - 4);  // the tail pad (zeroed at load, never written)
         ta.t = t;
         uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
         for (int r = 0; r < 10; ++r) {
@@ -1980,7 +2136,10 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         k0 += 0x9E3779B9u;
         k1 += 0xBB67AE85u;
     }
-    if (s.exclude_self) {
+    if (s.K > 16384) {
+        if (s.exclude_self) sweep_kernel<true, false, kTSWide><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+        else sweep_kernel<false, false, kTSWide><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
+    } else if (s.exclude_self) {
         if (s.sweep_fused) sweep_kernel<true, true><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
         else sweep_kernel<true, false><<<s.sweep_grid, kSweepThreads, s.sweep_smem, st>>>(a);
     } else {

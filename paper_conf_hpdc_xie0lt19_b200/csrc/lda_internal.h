@@ -191,6 +191,9 @@ struct DevState {
     int num_sms = 148;
     int sweep_grid = 0, sweep_block = 0;
     int theta_grid = 0, theta_block = 0;
+    bool recount_gmem = false, theta_gmem = false;  // K > 16384: K-length histograms in global scratch
+    int *recount_scratch = nullptr;                 // recount_gmem: num_sms*4 CTAs x 2K
+    uint32_t *theta_scratch = nullptr;              // theta_gmem: theta_grid*8 warps x (K + K/32)
     size_t sweep_smem = 0, theta_smem = 0;
     int ll_blocks = 0;
 };
@@ -205,7 +208,10 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
 // z in document order <-> word-major, through doc_map (device buffers of T entries; zd 16-byte aligned)
 int launch_gather_z(const DevState &s, uint16_t *zd, void *stream);
 int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream);
-int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event);
+// parts: bit 0 = prologue + per-word tables (once per sweep), bit 1 = the
+// sampling kernel (tile samplers; sampler 0 always runs both)
+int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event,
+                 int parts = 3);
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches);
 
 // ---------------------------------------------------------------------------

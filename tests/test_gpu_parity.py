@@ -132,6 +132,25 @@ def test_k8192_small(opts):
     assert unexc == 0
 
 
+@pytest.mark.parametrize("K,opts", [(20000, {}), (65536, {}), (30000, dict(exclude_self=1))])
+def test_wide_k_lockstep(K, opts):
+    """16384 < K <= 65536 (u16 topic ids, L1239-1243): wide θ entries
+    (topic << 16 | count), K-length histograms in global scratch, the
+    lane-per-token sampler -- against the oracle in lock step."""
+    doc_ptr, words = _corpus(60, 150, 6_000, 0.7, 16, 41)
+    a, b = 50.0 / K, 0.01
+    excl = opts.get("exclude_self", 0)
+    o = U.oracle_for(60, 150, K, a, b, doc_ptr, words, 4)
+    g = U.gpu_model(60, 150, K, a, b, doc_ptr, words, 4, **opts)
+    assert g.stats()["sampler"] == 0
+    assert np.array_equal(g.z(), o.z)
+    U.check_counts_equal(g, o)
+    bad, unexc = U.lockstep(g, o, 3, exclude_self=excl)
+    assert unexc == 0
+    assert g.loglik() == pytest.approx(o.loglik(), rel=1e-9)
+    U.check_invariants_gpu(g, doc_ptr, words)
+
+
 def test_nytimes_shaped_midsize_many_chunks():
     """A downscaled NYTimes-shaped corpus at K=1024 that spans many sampler
     chunks, split words and ragged tails; options that only change the work
