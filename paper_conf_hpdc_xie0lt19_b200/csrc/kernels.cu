@@ -96,12 +96,6 @@ __device__ __forceinline__ uint4 ld_nc_v4(const uint4 *p) {
 #ifndef LDA_L2HINT
 #define LDA_L2HINT 0
 #endif
-#ifndef LDA_WALK2
-#define LDA_WALK2 1
-#endif
-#ifndef LDA_HOOK
-#define LDA_HOOK 0
-#endif
 __device__ __forceinline__ uint64_t pol_evict_last() {
     uint64_t p;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
@@ -474,9 +468,33 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
     }
 }
 
+#ifndef LDA_I2FP
+#define LDA_I2FP 1
+#endif
 // count (low 16 bits of a θ entry) as float, exactly: bits 0x4B00:count = 2^23 + c
 __device__ __forceinline__ float count_f32(uint32_t e) {
     return __uint_as_float(__byte_perm(e, 0x4B00u, 0x5410)) - 8388608.0f;
+}
+// the same with the byte selector 0x5410 in a register the caller made once
+// (opaque_u32): a constant selector is rematerialised before every PRMT
+// (one extra IMAD per θ entry in the walk, measured in the SASS)
+__device__ __forceinline__ float count_f32(uint32_t e, uint32_t sel) {
+#if LDA_I2FP
+    // LOP3 + I2FP.F32.U32 (bits 16-17 of an entry are zero)
+    return __uint2float_rn(e & 0x1FFFFu);
+#else
+    return __uint_as_float(__byte_perm(e, 0x4B00u, sel)) - 8388608.0f;
+#endif
+}
+__device__ __forceinline__ uint32_t opaque_u32(uint32_t v) {
+    uint32_t r;
+    asm volatile("mov.b32 %0, %1;" : "=r"(r) : "r"(v));
+    return r;
+}
+// the line sum of line L from its four block sums (the quad's order)
+__device__ __forceinline__ float line_sum(const float *blk, uint32_t L) {
+    const float4 b = *reinterpret_cast<const float4 *>(blk + 4 * L);
+    return (b.x + b.y) + (b.z + b.w);
 }
 // the entry's topic in an fp32 table: byte offset e >> 16 = 4·topic
 __device__ __forceinline__ float tab32(const float *__restrict__ p32, uint32_t e) {
@@ -484,6 +502,9 @@ __device__ __forceinline__ float tab32(const float *__restrict__ p32, uint32_t e
 }
 __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc) {
     return fmaf(count_f32(e), tab32(p32, e), acc);
+}
+__device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc, uint32_t sel) {
+    return fmaf(count_f32(e, sel), tab32(p32, e), acc);
 }
 
 // ---------------------------------------------------------------------------
@@ -533,6 +554,21 @@ __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restric
 #endif
 constexpr int kTileMaxK = LDA_TILE_MAXK;
 
+#ifndef LDA_TILE_STATS
+#define LDA_TILE_STATS 0
+#endif
+#if LDA_TILE_STATS
+// diagnostics build only: batches, tokens, θ-row lines walked, distinct rows, walk steps
+__device__ unsigned long long g_tile_stats[8];
+extern "C" int lda_debug_tile_stats(unsigned long long *out, int reset) {
+    cudaError_t e = cudaMemcpyFromSymbol(out, g_tile_stats, sizeof(g_tile_stats));
+    if (e == cudaSuccess && reset) {
+        unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        e = cudaMemcpyToSymbol(g_tile_stats, z, sizeof(z));
+    }
+    return e;
+}
+#endif
 struct TileArgs {
     const TileItem *items;
     int64_t n_items;
@@ -855,65 +891,34 @@ __device__ __forceinline__ TileHead tile_head(const TileArgs &a, uint32_t row, u
 // `sub` sums entries 8·sub .. 8·sub+7 of the line (two FFMA chains); the
 // quad's line sum by two xor-shuffles.  Branch-free over the R lines in
 // flight (a lane past the end sums stale entries and discards them).
-// at_step2() runs once, after the first step (the caller's prefetch hook).
+// at_step2() runs once, at the start of the last step (the caller's prefetch hook).
 template <int R, class F>
 __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, const uint32_t *lrow, Blk8 (&ring)[R],
-                                          bool (&hdr)[R], const float *p32, float *blk, float *lsm, F &&at_step2) {
+                                          bool (&hdr)[R], const float *p32, float *blk, uint32_t sel,
+                                          F &&at_step2) {
     const int lane = threadIdx.x & 31, q = lane >> 2, sub = lane & 3;
     bool hooked = false;
     for (uint32_t base = 0; base < lsum; base += 8u * R) {
-#if LDA_HOOK == 1
-        // the caller's prefetch hook at the start of the last step (after step 1)
+        // the caller's prefetch hook at the start of the last step (or after
+        // a single step): the loads it issues (the next batch's θ row
+        // headers) depend on loads issued before the walk, which then have
+        // all earlier steps to land (measured +1 % over the second step)
         if (base > 0 && base + 8u * R >= lsum) {
-#else
-        if (base == 8u * R) {
-#endif
             at_step2();
             hooked = true;
         }
-#if LDA_WALK2
-        // slot by slot: sum the slot's line, refill the slot for the next
-        // step at once (its load then has the other slots' work to land),
-        // then the slot's line sum
-#pragma unroll
-        for (int s2 = 0; s2 < R; ++s2) {
-            const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
-            float s0 = count_f32(w0) * tab32(p32, w0);
-            float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
-            s0 = entry_mass32(ring[s2].w[2], p32, s0);
-            s1 = entry_mass32(ring[s2].w[3], p32, s1);
-            s0 = entry_mass32(ring[s2].w[4], p32, s0);
-            s1 = entry_mass32(ring[s2].w[5], p32, s1);
-            s0 = entry_mass32(ring[s2].w[6], p32, s0);
-            s1 = entry_mass32(ring[s2].w[7], p32, s1);
-            const float bs = s0 + s1;
-            const uint32_t Ln = base + 8u * (s2 + R) + q;
-            if (Ln < lsum) {
-                const uint32_t lr = lrow[Ln];
-                ring[s2] = ld_row_v8(a.rows + (static_cast<size_t>(lr & 0x7FFFFFFFu) + sub) * 8);
-                hdr[s2] = sub == 0 && (lr >> 31);
-            }
-            const uint32_t L = base + 8u * s2 + q;
-            float ls = bs + __shfl_xor_sync(kFull, bs, 1);
-            ls += __shfl_xor_sync(kFull, ls, 2);
-            if (L < lsum) {
-                blk[4 * L + sub] = bs;
-                if (sub == 0) lsm[L] = ls;
-            }
-        }
-#else
         float bs[R];
 #pragma unroll
         for (int s2 = 0; s2 < R; ++s2) {
             const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
-            float s0 = count_f32(w0) * tab32(p32, w0);
-            float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
-            s0 = entry_mass32(ring[s2].w[2], p32, s0);
-            s1 = entry_mass32(ring[s2].w[3], p32, s1);
-            s0 = entry_mass32(ring[s2].w[4], p32, s0);
-            s1 = entry_mass32(ring[s2].w[5], p32, s1);
-            s0 = entry_mass32(ring[s2].w[6], p32, s0);
-            s1 = entry_mass32(ring[s2].w[7], p32, s1);
+            float s0 = count_f32(w0, sel) * tab32(p32, w0);
+            float s1 = count_f32(ring[s2].w[1], sel) * tab32(p32, ring[s2].w[1]);
+            s0 = entry_mass32(ring[s2].w[2], p32, s0, sel);
+            s1 = entry_mass32(ring[s2].w[3], p32, s1, sel);
+            s0 = entry_mass32(ring[s2].w[4], p32, s0, sel);
+            s1 = entry_mass32(ring[s2].w[5], p32, s1, sel);
+            s0 = entry_mass32(ring[s2].w[6], p32, s0, sel);
+            s1 = entry_mass32(ring[s2].w[7], p32, s1, sel);
             bs[s2] = s0 + s1;
         }
 #pragma unroll
@@ -925,17 +930,12 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
                 hdr[s2] = sub == 0 && (lr >> 31);
             }
         }
+        // block sums to smem, unconditionally: a lane past the batch's last
+        // line writes into the scratch past it (L < lsum + 8R <= LM + 8R,
+        // inside the warp's blk + pad region); the draw forms line sums
+        // from the four block sums of a line
 #pragma unroll
-        for (int s2 = 0; s2 < R; ++s2) {
-            const uint32_t L = base + 8u * s2 + q;
-            float ls = bs[s2] + __shfl_xor_sync(kFull, bs[s2], 1);
-            ls += __shfl_xor_sync(kFull, ls, 2);
-            if (L < lsum) {
-                blk[4 * L + sub] = bs[s2];
-                if (sub == 0) lsm[L] = ls;
-            }
-        }
-#endif
+        for (int s2 = 0; s2 < R; ++s2) blk[4 * (base + 8u * s2 + q) + sub] = bs[s2];
     }
     if (!hooked) at_step2();
 }
@@ -947,7 +947,7 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
 // prefixes are farther from x by monotonicity); uncertain -> flag.
 template <bool COMPACT = false>
 __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t c0, uint32_t nl, uint32_t row,
-                                          uint32_t crank, uint64_t cb, double Q64, double gS, const float *lsm,
+                                          uint32_t crank, uint64_t cb, double Q64, double gS,
                                           const float *blk, const float *p32, const float *L32, const double *Pc,
                                           int NC, int &z, bool &flag, uint32_t &x0) {
     const int K = a.K;
@@ -956,9 +956,8 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
     flag = false;
     x0 = 0;
     if (take) {
-        const float *ln = lsm + c0;
         double S = 0.0;
-        for (uint32_t i = 0; i < nl; ++i) S += f2d_pos(ln[i]);
+        for (uint32_t i = 0; i < nl; ++i) S += f2d_pos(line_sum(blk, c0 + i));
         x0 = philox_x0_sched(cb + crank, a.t, a.key0, a.key1);
         const double U = (__hiloint2double(0x43300000, static_cast<int>(x0)) - 4503599627370496.0) *
                          2.3283064365386962890625e-10;  // x0·2^-32, exact
@@ -975,7 +974,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             double C = 0.0, Cn = 0.0;
             uint32_t i = 0;
             for (;; ++i) {
-                Cn = C + f2d_pos(ln[i]);
+                Cn = C + f2d_pos(line_sum(blk, c0 + i));
                 if (Cn > x || i + 1 >= nl) break;
                 C = Cn;
             }
@@ -1142,8 +1141,10 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
     float *p32 = reinterpret_cast<float *>(Pc + tab_nc2(K));
     float *L32 = p32 + K4;
     float *blk = L32 + 128 * NC;           // 4 block sums per line
-    float *lsm = blk + 4 * LM;             // line sums
-    uint32_t *lrow = reinterpret_cast<uint32_t *>(lsm + LM);
+    // blk: 4 block sums per line; the next LM floats pad it for the walk's
+    // unconditional stores past the batch's last line (LM >= 8R)
+    uint32_t *lrow = reinterpret_cast<uint32_t *>(blk + 5 * LM);
+    const uint32_t sel = opaque_u32(0x5410u);
     uint32_t *tcum = lrow + LM;
     uint64_t *bar = reinterpret_cast<uint64_t *>(tcum + 32);
     for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
@@ -1153,6 +1154,9 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
     unsigned n_exact = 0;
     int cur_word = -1;
     uint32_t phase = 0;
+#if LDA_TILE_STATS
+    unsigned long long st_batches = 0, st_tokens = 0, st_lines = 0, st_rows = 0, st_steps = 0;
+#endif
     const double u = 5.9604644775390625e-08;  // fp32 unit roundoff 2^-24
     // rounding bound of every prefix of the walk: p32 2u + 4-FFMA chain + 1
     // (block sum) + 2 (quad line sum), accumulated in fp64
@@ -1220,6 +1224,18 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         // ---- this batch
         const uint32_t p = it.pos + b0 + lane;
         const bool take = hd.take;
+#if LDA_TILE_STATS
+        {
+            const unsigned nd = __popc(__ballot_sync(kFull, take && !hd.dup));
+            if (lane == 0) {
+                st_batches += 1;
+                st_tokens += hd.nb;
+                st_lines += hd.lsum;
+                st_rows += nd;
+                st_steps += (hd.lsum + 8u * LDA_TRING - 1) / (8u * LDA_TRING);
+            }
+        }
+#endif
         const int nb = hd.nb;
         const uint32_t lsum = hd.lsum, c0 = hd.c0, nl = hd.nl;
         // ---- the next batch: this item's next tokens, else the next item's first
@@ -1232,7 +1248,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         const uint32_t n_crank = (more ? it.crank0 + b1 : itn.crank0) + lane;
         if (nxt_valid) n_row = ld_stream_u32(a.tok_row + nxt_pos + lane);
         // ---- walk (the next batch's row headers issued after its first step)
-        tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, lsm, [&] {
+        tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, sel, [&] {
             if (nxt_valid) n_nnz = ld_row_u32(a.rows + static_cast<size_t>(n_row) * 8);
         });
         __syncwarp();
@@ -1247,7 +1263,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         int z;
         bool flag;
         uint32_t x0;
-        tile_draw(a, take, c0, nl, row, crank, cb, Q64, gS, lsm, blk, p32, L32, Pc, NC, z, flag, x0);
+        tile_draw(a, take, c0, nl, row, crank, cb, Q64, gS, blk, p32, L32, Pc, NC, z, flag, x0);
         tile_finish(a, take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q, n_exact);
         // ---- advance
         row = n_row;
@@ -1273,6 +1289,15 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         for (int k = threadIdx.x; k < K; k += blockDim.x)
             if (nkh[k]) atomicAdd(a.nk_next + k, nkh[k]);
     if (a.n_exact && lane == 0 && n_exact) atomicAdd(a.n_exact, static_cast<unsigned long long>(n_exact));
+#if LDA_TILE_STATS
+    if (lane == 0) {
+        atomicAdd(&g_tile_stats[0], st_batches);
+        atomicAdd(&g_tile_stats[1], st_tokens);
+        atomicAdd(&g_tile_stats[2], st_lines);
+        atomicAdd(&g_tile_stats[3], st_rows);
+        atomicAdd(&g_tile_stats[4], st_steps);
+    }
+#endif
 }
 
 
@@ -1317,8 +1342,8 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     char *tabs = reinterpret_cast<char *>(smem_dd) + (GNK ? 0 : 4 * K4);
     char *wb = tabs + NB * wt + static_cast<size_t>(warp) * tile_cta_warp_bytes(LM);
     float *blk = reinterpret_cast<float *>(wb);
-    float *lsm = blk + 4 * LM;
-    uint32_t *lrow = reinterpret_cast<uint32_t *>(lsm + LM);
+    uint32_t *lrow = reinterpret_cast<uint32_t *>(blk + 5 * LM);  // blk + pad (see sweep_tile_kernel)
+    const uint32_t sel = opaque_u32(0x5410u);
     char *ctrl = tabs + NB * wt + static_cast<size_t>(nwarps) * tile_cta_warp_bytes(LM);
     uint64_t *bar = reinterpret_cast<uint64_t *>(ctrl);         // [4]
     TileItem *items = reinterpret_cast<TileItem *>(ctrl + 32);  // [4]
@@ -1391,12 +1416,12 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
                     nnz = ld_row_u32(a.rows + static_cast<size_t>(row) * 8);
                 }
                 const TileHead hd = tile_head<R>(a, row, nnz, valid, LM, lrow, ring, hdr);
-                tile_walk<R>(a, hd.lsum, lrow, ring, hdr, p32, blk, lsm, [] {});
+                tile_walk<R>(a, hd.lsum, lrow, ring, hdr, p32, blk, sel, [] {});
                 __syncwarp();
                 int z;
                 bool flag;
                 uint32_t x0;
-                tile_draw<GNK>(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, lsm, blk, p32, L32, Pc, NC, z,
+                tile_draw<GNK>(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, blk, p32, L32, Pc, NC, z,
                                flag, x0);
                 tile_finish(a, hd.take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q,
                             n_exact);
@@ -1837,7 +1862,7 @@ int configure_kernels(DevState &s) {
         // per-warp tables of 8·K bytes leave too few warps per SM (measured at
         // K = 8192 on the NYTimes shape: sampler 0 is faster)
         if (s.sampler < 0) s.sampler = s.K <= kTileMaxK ? 2 : 3;
-        s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1;
+        s.sweep_tile = s.sampler == 2 && !s.exclude_self && LDA_FUSE && wpc >= 1 && s.K <= 16384;
         // large K: CTA-shared double-buffered tables (sweep_tile_cta_kernel)
         s.tile_cta_gnk = s.K > kTileMaxK;
         // large K: one CTA per SM with up to 4 compact table buffers, keeping
@@ -1859,7 +1884,8 @@ int configure_kernels(DevState &s) {
                 }
         const int cwarps = fit(s.tile_nbuf);
         const size_t cta_bytes = tile_cta_bytes(s.K, s.tile_lmax, cwarps, s.tile_cta_gnk, s.tile_nbuf);
-        s.sweep_tile_cta = s.sampler == 3 && !s.exclude_self && LDA_FUSE && cwarps >= 2;
+        // the tile samplers read θ entries as topic << 18 | count (K <= 16384)
+        s.sweep_tile_cta = s.sampler == 3 && !s.exclude_self && LDA_FUSE && cwarps >= 2 && s.K <= 16384;
         if (s.sampler == 3 && !s.sweep_tile_cta) s.sampler = 0;
         if (s.sweep_tile_cta) {
             const void *fn = s.tile_cta_gnk ? reinterpret_cast<const void *>(&sweep_tile_cta_kernel<LDA_TRING, true>)
