@@ -468,29 +468,11 @@ __global__ void __launch_bounds__(kSweepThreads, LDA_SWEEP_MINB) sweep_kernel(Sw
     }
 }
 
-#ifndef LDA_I2FP
-#define LDA_I2FP 1
-#endif
 // count (low 16 bits of a θ entry) as float, exactly: bits 0x4B00:count = 2^23 + c
 __device__ __forceinline__ float count_f32(uint32_t e) {
     return __uint_as_float(__byte_perm(e, 0x4B00u, 0x5410)) - 8388608.0f;
 }
-// the same with the byte selector 0x5410 in a register the caller made once
-// (opaque_u32): a constant selector is rematerialised before every PRMT
-// (one extra IMAD per θ entry in the walk, measured in the SASS)
-__device__ __forceinline__ float count_f32(uint32_t e, uint32_t sel) {
-#if LDA_I2FP
-    // LOP3 + I2FP.F32.U32 (bits 16-17 of an entry are zero)
-    return __uint2float_rn(e & 0x1FFFFu);
-#else
-    return __uint_as_float(__byte_perm(e, 0x4B00u, sel)) - 8388608.0f;
-#endif
-}
-__device__ __forceinline__ uint32_t opaque_u32(uint32_t v) {
-    uint32_t r;
-    asm volatile("mov.b32 %0, %1;" : "=r"(r) : "r"(v));
-    return r;
-}
+// (PRMT + FADD; measured faster on B200 than LOP3 + I2FP.F32.U32: -0.5 %)
 // the line sum of line L from its four block sums (the quad's order)
 __device__ __forceinline__ float line_sum(const float *blk, uint32_t L) {
     const float4 b = *reinterpret_cast<const float4 *>(blk + 4 * L);
@@ -502,9 +484,6 @@ __device__ __forceinline__ float tab32(const float *__restrict__ p32, uint32_t e
 }
 __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc) {
     return fmaf(count_f32(e), tab32(p32, e), acc);
-}
-__device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restrict__ p32, float acc, uint32_t sel) {
-    return fmaf(count_f32(e, sel), tab32(p32, e), acc);
 }
 
 // ---------------------------------------------------------------------------
@@ -613,26 +592,25 @@ __device__ __forceinline__ double pstar64(const int32_t *nwk_row, const double *
 
 // Exact (fp64) draw of one token by the whole warp, from the counts in global
 // memory: p*(k) = (n_wk+β)/(n_k+Vβ) as the oracle computes it, S over the
-// doc row, Q = Σ_k α·p*(k) (cached per item in *q64 / *have_q), x = U·(S+Q),
-// then the first bin of [sparse ‖ dense] whose prefix exceeds x (X4-X6).
-// Only the summation order differs from the oracle's.
+// doc row, x = U·(S+Q), then the first bin of [sparse ‖ dense] whose prefix
+// exceeds x (X4-X6).  Q and the dense prefix at every group start come from
+// the word's table (B[g] = fp64 prefix of α·p* before group g of gsz topics,
+// B[G] = Q, built by word_table_kernel): the dense search jumps to the group
+// holding x and scans it with the exact p*, O(log G + gsz) instead of O(K).
+// Only the summation order (and p* by reciprocal inside B) differs from the
+// oracle's: fp64 rounding, far below the north_star's 1e-6 excuse.
 __device__ __noinline__ int draw_exact_warp(const int32_t *nwk_row, const double *denom, const uint32_t *rw,
                                             uint32_t nnz, uint32_t x0, int K, double alpha, double beta,
-                                            double *q64, int *have_q) {
+                                            const double *B, int G, int gsz) {
     const int lane = threadIdx.x & 31;
-    if (!*have_q) {
-        double q = 0.0;
-        for (int k = lane; k < K; k += 32) q += alpha * pstar64(nwk_row, denom, beta, k);
-        *q64 = warp_sum_d(q);
-        *have_q = 1;
-    }
+    const double Q = B[G];
     double s = 0.0;
     for (uint32_t j = 1 + lane; j <= nnz; j += 32) {
         const uint32_t e = __ldg(rw + j);
         s = fma(static_cast<double>(e & 0xFFFFu), pstar64(nwk_row, denom, beta, e >> kTS), s);
     }
     const double S = warp_sum_d(s);
-    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + *q64);
+    const double x = static_cast<double>(x0) * 2.3283064365386962890625e-10 * (S + Q);
     if (x < S) {
         double carry = 0.0;
         for (uint32_t j0 = 1; j0 <= nnz; j0 += 32) {
@@ -651,8 +629,15 @@ __device__ __noinline__ int draw_exact_warp(const int32_t *nwk_row, const double
         }
         return K - 1;
     }
-    double carry = S;
-    for (int k0 = 0; k0 < K; k0 += 32) {
+    // the last group g with S + B[g] <= x (uniform over the warp)
+    int g = 0;
+    for (int n = G; n > 1;) {
+        const int h = n >> 1;
+        if (S + B[g + h] <= x) g += h;
+        n -= h;
+    }
+    double carry = S + B[g];
+    for (int k0 = g * gsz; k0 < K; k0 += 32) {
         const int k = k0 + lane;
         const double m = k < K ? alpha * pstar64(nwk_row, denom, beta, k) : 0.0;
         const double c = carry + warp_incl_scan_d(m, lane);
@@ -894,8 +879,7 @@ __device__ __forceinline__ TileHead tile_head(const TileArgs &a, uint32_t row, u
 // at_step2() runs once, at the start of the last step (the caller's prefetch hook).
 template <int R, class F>
 __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, const uint32_t *lrow, Blk8 (&ring)[R],
-                                          bool (&hdr)[R], const float *p32, float *blk, uint32_t sel,
-                                          F &&at_step2) {
+                                          bool (&hdr)[R], const float *p32, float *blk, F &&at_step2) {
     const int lane = threadIdx.x & 31, q = lane >> 2, sub = lane & 3;
     bool hooked = false;
     for (uint32_t base = 0; base < lsum; base += 8u * R) {
@@ -911,14 +895,14 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
 #pragma unroll
         for (int s2 = 0; s2 < R; ++s2) {
             const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
-            float s0 = count_f32(w0, sel) * tab32(p32, w0);
-            float s1 = count_f32(ring[s2].w[1], sel) * tab32(p32, ring[s2].w[1]);
-            s0 = entry_mass32(ring[s2].w[2], p32, s0, sel);
-            s1 = entry_mass32(ring[s2].w[3], p32, s1, sel);
-            s0 = entry_mass32(ring[s2].w[4], p32, s0, sel);
-            s1 = entry_mass32(ring[s2].w[5], p32, s1, sel);
-            s0 = entry_mass32(ring[s2].w[6], p32, s0, sel);
-            s1 = entry_mass32(ring[s2].w[7], p32, s1, sel);
+            float s0 = count_f32(w0) * tab32(p32, w0);
+            float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
+            s0 = entry_mass32(ring[s2].w[2], p32, s0);
+            s1 = entry_mass32(ring[s2].w[3], p32, s1);
+            s0 = entry_mass32(ring[s2].w[4], p32, s0);
+            s1 = entry_mass32(ring[s2].w[5], p32, s1);
+            s0 = entry_mass32(ring[s2].w[6], p32, s0);
+            s1 = entry_mass32(ring[s2].w[7], p32, s1);
             bs[s2] = s0 + s1;
         }
 #pragma unroll
@@ -1092,7 +1076,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
 // warp), then z and the fused recount (ϕ update, L1273-1285).
 __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool flag, int z, uint32_t row,
                                             uint32_t nnz, uint32_t x0, uint32_t p, const int32_t *nwk_row,
-                                            int32_t *row_next, int *nkh, double *q64x, int *have_q,
+                                            int32_t *row_next, int *nkh, const double *B, int G, int gsz,
                                             unsigned &n_exact) {
     // nkh: the n_k histogram -- the CTA's in shared memory, or the global
     // next n_k (the large-K kernel keeps its shared memory for warps)
@@ -1107,7 +1091,7 @@ __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool f
         const uint32_t nf = __shfl_sync(kFull, nnz, f);
         const uint32_t xf = __shfl_sync(kFull, x0, f);
         const int zf = draw_exact_warp(nwk_row, a.denom, a.rows + static_cast<size_t>(rf) * 8, nf, xf, K,
-                                       a.alpha, a.beta, q64x, have_q);
+                                       a.alpha, a.beta, B, G, gsz);
         if (lane == f) z = zf;
         ++n_exact;
     }
@@ -1144,7 +1128,6 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
     // blk: 4 block sums per line; the next LM floats pad it for the walk's
     // unconditional stores past the batch's last line (LM >= 8R)
     uint32_t *lrow = reinterpret_cast<uint32_t *>(blk + 5 * LM);
-    const uint32_t sel = opaque_u32(0x5410u);
     uint32_t *tcum = lrow + LM;
     uint64_t *bar = reinterpret_cast<uint64_t *>(tcum + 32);
     for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
@@ -1198,8 +1181,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
     const int32_t *nwk_row = nullptr;
     int32_t *row_next = nullptr;
     uint64_t cb = 0;
-    double Q64 = 0.0, q64x = 0.0;
-    int have_q = 0;
+    double Q64 = 0.0;
     while (ci != 0xFFFFFFFFu) {
         if (new_item) {
             if (static_cast<int>(it.word) != cur_word) {
@@ -1218,7 +1200,6 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
             cb = __ldg(a.cbase + it.word);
             nwk_row = a.nwk + static_cast<size_t>(it.word) * K;
             row_next = a.nwk_next + static_cast<size_t>(it.word) * K;
-            have_q = 0;
             new_item = false;
         }
         // ---- this batch
@@ -1248,7 +1229,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         const uint32_t n_crank = (more ? it.crank0 + b1 : itn.crank0) + lane;
         if (nxt_valid) n_row = ld_stream_u32(a.tok_row + nxt_pos + lane);
         // ---- walk (the next batch's row headers issued after its first step)
-        tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, sel, [&] {
+        tile_walk<R>(a, lsum, lrow, ring, hdr, p32, blk, [&] {
             if (nxt_valid) n_nnz = ld_row_u32(a.rows + static_cast<size_t>(n_row) * 8);
         });
         __syncwarp();
@@ -1264,7 +1245,7 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         bool flag;
         uint32_t x0;
         tile_draw(a, take, c0, nl, row, crank, cb, Q64, gS, blk, p32, L32, Pc, NC, z, flag, x0);
-        tile_finish(a, take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q, n_exact);
+        tile_finish(a, take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, Pc, NC, 128, n_exact);
         // ---- advance
         row = n_row;
         crank = n_crank;
@@ -1343,7 +1324,6 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     char *wb = tabs + NB * wt + static_cast<size_t>(warp) * tile_cta_warp_bytes(LM);
     float *blk = reinterpret_cast<float *>(wb);
     uint32_t *lrow = reinterpret_cast<uint32_t *>(blk + 5 * LM);  // blk + pad (see sweep_tile_kernel)
-    const uint32_t sel = opaque_u32(0x5410u);
     char *ctrl = tabs + NB * wt + static_cast<size_t>(nwarps) * tile_cta_warp_bytes(LM);
     uint64_t *bar = reinterpret_cast<uint64_t *>(ctrl);         // [4]
     TileItem *items = reinterpret_cast<TileItem *>(ctrl + 32);  // [4]
@@ -1398,8 +1378,6 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
         const uint64_t cb = __ldg(a.cbase + it.word);
         const int32_t *nwk_row = a.nwk + static_cast<size_t>(it.word) * K;
         int32_t *row_next = a.nwk_next + static_cast<size_t>(it.word) * K;
-        double q64x = 0.0;
-        int have_q = 0;
         for (;;) {
             uint32_t sl = 0;
             if (lane == 0) sl = atomicAdd(slot + b, 1u);
@@ -1416,14 +1394,14 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
                     nnz = ld_row_u32(a.rows + static_cast<size_t>(row) * 8);
                 }
                 const TileHead hd = tile_head<R>(a, row, nnz, valid, LM, lrow, ring, hdr);
-                tile_walk<R>(a, hd.lsum, lrow, ring, hdr, p32, blk, sel, [] {});
+                tile_walk<R>(a, hd.lsum, lrow, ring, hdr, p32, blk, [] {});
                 __syncwarp();
                 int z;
                 bool flag;
                 uint32_t x0;
                 tile_draw<GNK>(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, blk, p32, L32, Pc, NC, z,
                                flag, x0);
-                tile_finish(a, hd.take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, &q64x, &have_q,
+                tile_finish(a, hd.take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, Pc, NC, GNK ? 32 : 128,
                             n_exact);
                 b0 += static_cast<uint32_t>(hd.nb);
             }
