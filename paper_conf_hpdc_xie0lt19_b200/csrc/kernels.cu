@@ -536,9 +536,7 @@ constexpr int kTileMaxK = LDA_TILE_MAXK;
 #ifndef LDA_TILE_STATS
 #define LDA_TILE_STATS 0
 #endif
-#ifndef LDA_CTA_PF
-#define LDA_CTA_PF 1
-#endif
+
 #if LDA_TILE_STATS
 // diagnostics build only: batches, tokens, θ-row lines walked, distinct rows, walk steps
 __device__ unsigned long long g_tile_stats[8];
@@ -1302,7 +1300,7 @@ __host__ __device__ constexpr size_t tile_cta_warp_bytes(int lmax) {
 __host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps, bool gnk, int nb) {
     return (gnk ? 0 : static_cast<size_t>(4) * ((K + 3) & ~3)) +
            static_cast<size_t>(nb) * (gnk ? tab_bytes_compact(K) : tab_bytes(K)) +
-           nwarps * tile_cta_warp_bytes(lmax) + 192;
+           nwarps * tile_cta_warp_bytes(lmax) + 128;
 }
 
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
@@ -1332,7 +1330,6 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     TileItem *items = reinterpret_cast<TileItem *>(ctrl + 32);  // [4]
     uint32_t *slot = reinterpret_cast<uint32_t *>(ctrl + 96);   // [4]
     uint32_t *left = slot + 4;                                  // [4]
-    TileItem *nxt = reinterpret_cast<TileItem *>(ctrl + 128);   // [4]: each buffer's next item (claimed ahead)
     const double gS = 9.5 * 5.9604644775390625e-08 * a.slack;
 
     // buffer b <- the CTA's next work item (its table by bulk copy); the end
@@ -1342,25 +1339,10 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     // compute-sanitizer's racecheck does not model mbarrier ordering and
     // reports this handoff as a hazard (memcheck is clean).  The loader runs
     // only after every warp has left the buffer (left[b] reached 0).
-    // each buffer's next work item is claimed one use ahead and its table
-    // prefetched into L2 then, so that the buffer's refill (the bulk copy
-    // into shared memory) reads L2 instead of HBM
-    auto claim = [&]() {
+    auto load = [&](int b) {
         const uint32_t ci = atomicAdd(a.counter, 1u);
         TileItem it = {0u, 0u, 0u, 0u};
         if (ci < a.n_items) it = a.items[ci];
-#if LDA_CTA_PF
-        if (it.n) prefetch_l2_bulk(a.wtab + static_cast<size_t>(it.word) * a.wt_bytes, a.wt_bytes);
-#endif
-        return it;
-    };
-    auto load = [&](int b) {
-#if LDA_CTA_PF
-        const TileItem it = nxt[b];
-        nxt[b] = it.n ? claim() : it;
-#else
-        const TileItem it = claim();
-#endif
         items[b] = it;
         slot[b] = 0u;
         left[b] = static_cast<uint32_t>(nwarps);
@@ -1377,9 +1359,6 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     if (threadIdx.x == 0) {
         for (int b = 0; b < NB; ++b) mbar_init(bar + b, 1);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-#if LDA_CTA_PF
-        for (int b = 0; b < NB; ++b) nxt[b] = claim();
-#endif
         for (int b = 0; b < NB; ++b) load(b);
     }
     __syncthreads();
