@@ -266,7 +266,88 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     std::vector<std::vector<uint32_t>> cnext(nthreads, std::vector<uint32_t>(V));
 
     uint64_t pos = 0;  // start of the current tile's segment
-    for (int b = 0; b < ndt; ++b) {
+    if (tile_layout && ndt >= 2 * nthreads) {
+        // Many tiles (PubMed shape: 54 on 16 host threads): one thread per
+        // tile instead of every tile split over all threads, so the per-word
+        // work (V-length count arrays, their sums and prefixes) is done once
+        // per tile instead of once per tile and thread.
+        //   1. counts of every tile (head and tail words)
+        //   2. canonical ranks of the runs (prefix over the tiles, per word),
+        //      the tiles' segment starts and the head words' run starts
+        //   3. the scatter, tile by tile, each tile's part announced to the
+        //      copier (on_final) as soon as it is written
+        std::vector<int64_t> headT(ndt, 0);
+        std::atomic<int> next_tile{0};
+        auto tile_threads = [&](auto &&f) {
+            std::vector<std::thread> th;
+            for (int t = 1; t < nthreads; ++t) th.emplace_back(f);
+            f();
+            for (auto &x : th) x.join();
+        };
+        tile_threads([&] {
+            for (int b; (b = next_tile.fetch_add(1)) < ndt;) {
+                auto &tc = tile_cnt[b];
+                tc.assign(V, 0);
+                const int64_t i0 = doc_ptr[tile_doc[b]], i1 = doc_ptr[tile_doc[b + 1]];
+                for (int64_t i = i0; i < i1; ++i) tc[words[i]]++;
+                int64_t tt = 0;
+                for (int32_t w = 0; w < V; ++w)
+                    if (tail[w]) tt += tc[w];
+                headT[b] = (i1 - i0) - tt;
+            }
+        });
+        std::vector<uint64_t> pos_tile(ndt + 1, 0);
+        for (int b = 0; b < ndt; ++b) pos_tile[b + 1] = pos_tile[b] + static_cast<uint64_t>(headT[b]);
+        // per word: the run's canonical rank in each tile = tokens of the word in earlier tiles
+        parallel_for(nthreads, V, [&](int, int64_t w0, int64_t w1) {
+            for (int64_t w = w0; w < w1; ++w) {
+                uint32_t run_c = 0;
+                for (int b = 0; b < ndt; ++b) {
+                    tcrank[static_cast<size_t>(b) * V + w] = run_c;
+                    run_c += tile_cnt[b][w];
+                }
+            }
+        });
+        next_tile = 0;
+        tile_threads([&] {
+            std::vector<uint32_t> next(V);
+            for (int b; (b = next_tile.fetch_add(1)) < ndt;) {
+                auto &tc = tile_cnt[b];
+                uint32_t *tseg_b = tseg.data() + static_cast<size_t>(b) * V;
+                const uint32_t *tcr_b = tcrank.data() + static_cast<size_t>(b) * V;
+                uint64_t p = pos_tile[b];
+                for (int32_t w = 0; w < V; ++w) {
+                    if (tail[w]) {
+                        // the tail word's tokens of this tile continue its tail run
+                        next[w] = tail_next[w] + tcr_b[w];
+                        tc[w] = 0;  // counted in the tail tile only
+                    } else {
+                        tseg_b[w] = static_cast<uint32_t>(p);
+                        next[w] = static_cast<uint32_t>(p);
+                        p += tc[w];
+                    }
+                }
+                const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
+                if (want_row) {
+                    for (int64_t d = d0; d < d1; ++d) {
+                        const uint32_t row = L.row_off32[d];
+                        for (int64_t i = doc_ptr[d]; i < doc_ptr[d + 1]; ++i) {
+                            const uint32_t q = next[words[i]]++;
+                            L.doc_map[i] = q;
+                            L.tok_row[q] = row;
+                        }
+                    }
+                } else {
+                    for (int64_t i = doc_ptr[d0]; i < doc_ptr[d1]; ++i) L.doc_map[i] = next[words[i]]++;
+                }
+                if (on_final)
+                    on_final(pos_tile[b], pos_tile[b + 1], static_cast<uint64_t>(doc_ptr[d0]),
+                             static_cast<uint64_t>(doc_ptr[d1]));
+            }
+        });
+        pos = pos_tile[ndt];
+    }
+    for (int b = 0; b < ndt && !(tile_layout && ndt >= 2 * nthreads); ++b) {
         const uint64_t pos_tile = pos;
         const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
         // the tile's documents in nth contiguous parts (original order), balanced by tokens

@@ -221,3 +221,17 @@ def test_python_binding_checks_buffer_lengths():
         assert e.value.code == L.LDA_EINVAL
     finally:
         L.lda_destroy(ctx)
+
+
+@pytest.mark.parametrize("sampler", [2, 3])
+def test_layout_invariants_many_tiles(sampler):
+    """At least twice as many tiles as host threads (PubMed shape: 54 tiles):
+    the host pass runs one thread per tile (counts, run ranks, scatter);
+    the same brute-force invariants must hold."""
+    import os
+    doc_ptr, words = _corpus(6000, 3000, 17, max_len=40)
+    tiles_wanted = 2 * (os.cpu_count() or 8) + 3
+    tile_tokens = max(50, int(doc_ptr[-1]) // tiles_wanted)
+    st = L.lda_layout_selfcheck(doc_ptr, words, 3000, 24, sampler=sampler, tile_tokens=tile_tokens,
+                                chunk_tokens=64, tail_per_tile=8)
+    assert st["tiles"] >= tiles_wanted and st["tail_words"] > 0
