@@ -117,7 +117,10 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int sampler, int64_t tail_per_tile, HostLayout &out,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {},
                          const int64_t *word_counts = nullptr,  // V local tokens per word, if known
-                         bool host_tok_row = true);  // tile layout: false = tok_row left to the device (launch_tok_row)
+                         bool host_tok_row = true,  // tile layout: false = tok_row left to the device (launch_tok_row)
+                         // called with the host doc_map buffer right after its allocation (the
+                         // caller may page-lock it in the background for fast H2D copies)
+                         const std::function<void(void *, size_t)> &on_host_alloc = {});
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
