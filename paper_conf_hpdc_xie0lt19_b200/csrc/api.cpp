@@ -6,6 +6,8 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
 #include <condition_variable>
 #include <mutex>
 #include <thread>
@@ -55,6 +57,7 @@ struct lda_ctx {
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int64_t comm_pipeline = 4;  // world > 1: word ranges whose rows are exchanged as soon as recounted (f1)
+    int zdoc = 0;               // the tile sampler writes z in document order too (skips the θ gather)
     int threads = 0;
     // distribution: the exchange of Eq. 4 (NCCL or the in-process peer group)
     int32_t rank = 0, world = 1;
@@ -570,6 +573,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
+    } else if (k == "zdoc") {
+        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "zdoc must be 0 or 1");
+        ctx->zdoc = static_cast<int>(value);
     } else if (k == "stream_chunks") {
         if (value < 1 || value > 4096) return fail(ctx, LDA_EINVAL, "stream_chunks must be in [1, 4096]");
         ctx->stream_chunks = value;
@@ -769,6 +775,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         if (t) pre.push_back({reinterpret_cast<void **>(t), sizeof(uint32_t) * Tg});
     pre.push_back({reinterpret_cast<void **>(&S.tok_z), sizeof(uint16_t) * Tg});
     pre.push_back({reinterpret_cast<void **>(&S.z_doc), sizeof(uint16_t) * (Tg + 8)});
+    if (tile_layout && ctx->zdoc) pre.push_back({reinterpret_cast<void **>(&S.tok_doc), sizeof(uint32_t) * Tg});
     const size_t nwk_bytes = sizeof(int32_t) * (static_cast<size_t>(V) * K + K);
     pre.push_back({reinterpret_cast<void **>(&S.nwk), nwk_bytes});
     if (S.sweep_fused) pre.push_back({reinterpret_cast<void **>(&S.nwk_alt), nwk_bytes});
@@ -789,6 +796,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         cudaStream_t cs = nullptr;
         cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
         pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
+        const auto c0 = std::chrono::steady_clock::now();
         for (auto &pa : pre) {
             if (copy_err != cudaSuccess) break;
             void *q = nullptr;
@@ -800,6 +808,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             *pa.first = q;
             pre_done.push_back(q);
         }
+        const auto c1 = std::chrono::steady_clock::now();
+        double copy_ms = 0.0;
         for (;;) {
             Job j;
             {
@@ -818,10 +828,15 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                 r = cudaMemcpyAsync(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
             if (nt && r == cudaSuccess)
                 r = cudaMemcpyAsync(S.doc_map + j.t0, H.doc_map.data() + j.t0, nt, cudaMemcpyHostToDevice, cs);
+            const auto j0 = std::chrono::steady_clock::now();
             if (r == cudaSuccess) r = cudaStreamSynchronize(cs);
+            copy_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - j0).count();
             if (r != cudaSuccess && copy_err == cudaSuccess) copy_err = r;
         }
         if (cs) cudaStreamDestroy(cs);
+        if (std::getenv("LDA_TIMING"))
+            std::fprintf(stderr, "[lda]   copier: device allocation %.1f ms, H2D waits %.1f ms\n",
+                         std::chrono::duration<double, std::milli>(c1 - c0).count(), copy_ms);
     });
     auto on_final = [&](uint64_t p0, uint64_t p1, uint64_t t0, uint64_t t1) {
         {
@@ -829,19 +844,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             jobs.push_back(Job{p0, p1, t0, t1});
         }
         cv.notify_one();
-    };
-    // page-lock the host doc_map (3 GB at PubMed shape) in the background as
-    // soon as the layout allocates it: the copier's H2D copies then run at
-    // DMA speed instead of through the driver's pageable staging, and the
-    // pages are faulted in here rather than by the tile pass's first writes
-    void *pin_ptr = nullptr;
-    std::thread pinner;
-    auto on_host_alloc = [&](void *ptr, size_t bytes) {
-        pinner = std::thread([&pin_ptr, ptr, bytes, dev = ctx->device] {
-            cudaSetDevice(dev);
-            if (cudaHostRegister(ptr, bytes, cudaHostRegisterDefault) == cudaSuccess) pin_ptr = ptr;
-            else cudaGetLastError();
-        });
     };
     // the large-K sampler copies a table of 8·K bytes per work item: its items
     // grow with K (tiles and the tail threshold scaled by K/1024; measured at
@@ -851,15 +853,13 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
                                       tile_layout ? 2 : 0,
                                       ctx->tail_per_tile * kscale, H,
-                                      on_final, local.data(), /*host_tok_row=*/!tile_layout, on_host_alloc);
-    if (pinner.joinable()) pinner.join();
+                                      on_final, local.data(), /*host_tok_row=*/!tile_layout);
     {
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
     }
     cv.notify_one();
     copier.join();
-    if (pin_ptr) cudaHostUnregister(pin_ptr);  // every H2D copy from it is done
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
     // a range error of the layout takes precedence over an allocation error
     if (!e.empty()) {
@@ -977,6 +977,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
     if (tile_layout) KL(lda::launch_tok_row(S, ctx->stream));
+    KL(lda::launch_inv_map(S, ctx->stream));
     // a1: random init (t = 0), then the count rebuild.
     CU(cudaStreamSynchronize(ctx->stream));
     lda::tmark("H2D copies");
@@ -1062,7 +1063,8 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventRecord(E[2], ctx->stream));
         // θ update (depends only on z) on the compute stream while ϕ is
         // summed over the ranks on the comm stream (§6.2)
-        KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches));
+        KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches,
+                             /*gathered=*/S.tok_doc != nullptr));
         CU(cudaEventRecord(E[3], ctx->stream));
         if (ctx->world > 1) {
             const size_t K = static_cast<size_t>(S.K);

@@ -146,8 +146,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &L,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final,
-                         const int64_t *word_counts, bool host_tok_row,
-                         const std::function<void(void *, size_t)> &on_host_alloc) {
+                         const int64_t *word_counts, bool host_tok_row) {
     const int64_t T = doc_ptr[D];
     L.D = D;
     L.T = T;
@@ -225,7 +224,6 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     if ((want_row && !L.tok_row.allocate(T)) || !L.doc_map.allocate(T) ||
         (!tile_layout && !L.tok_crank.allocate(T)))
         return "host allocation of the token tables failed";
-    if (on_host_alloc && T > 0) on_host_alloc(L.doc_map.data(), sizeof(uint32_t) * static_cast<size_t>(T));
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
     if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";
     // first touch in parallel, one store per 4 KB page (the kernel zeroes

@@ -117,10 +117,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int sampler, int64_t tail_per_tile, HostLayout &out,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {},
                          const int64_t *word_counts = nullptr,  // V local tokens per word, if known
-                         bool host_tok_row = true,  // tile layout: false = tok_row left to the device (launch_tok_row)
-                         // called with the host doc_map buffer right after its allocation (the
-                         // caller may page-lock it in the background for fast H2D copies)
-                         const std::function<void(void *, size_t)> &on_host_alloc = {});
+                         bool host_tok_row = true);  // tile layout: false = tok_row left to the device (launch_tok_row)
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
@@ -153,6 +150,7 @@ struct DevState {
     uint32_t *doc_map = nullptr;    // T
     uint32_t *tok_crank = nullptr;  // T (word-major); null for the tile samplers (ranks from the items)
     uint16_t *z_doc = nullptr;      // T, z in document order (θ rebuild, phase A)
+    uint32_t *tok_doc = nullptr;    // option zdoc (tile samplers): word-major -> document-order index
     uint32_t *doc_ptr32 = nullptr;  // D+1
     uint32_t *row_off32 = nullptr;  // D
     Seg *segs = nullptr;
@@ -207,7 +205,10 @@ int launch_init(const DevState &s, void *stream);
 int launch_tok_row(const DevState &s, void *stream);
 int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0 = 0, int64_t rc1 = -1,
                    bool first = true);
-int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches);
+// gathered: z_doc already holds this sweep's z in document order (option zdoc)
+int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches,
+                 bool gathered = false);
+int launch_inv_map(const DevState &s, void *stream);
 // z in document order <-> word-major, through doc_map (device buffers of T entries; zd 16-byte aligned)
 int launch_gather_z(const DevState &s, uint16_t *zd, void *stream);
 int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream);
