@@ -57,7 +57,6 @@ struct lda_ctx {
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int64_t comm_pipeline = 4;  // world > 1: word ranges whose rows are exchanged as soon as recounted (f1)
-    int zdoc = 0;               // the tile sampler writes z in document order too (skips the θ gather)
     int threads = 0;
     // distribution: the exchange of Eq. 4 (NCCL or the in-process peer group)
     int32_t rank = 0, world = 1;
@@ -573,9 +572,6 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
-    } else if (k == "zdoc") {
-        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "zdoc must be 0 or 1");
-        ctx->zdoc = static_cast<int>(value);
     } else if (k == "stream_chunks") {
         if (value < 1 || value > 4096) return fail(ctx, LDA_EINVAL, "stream_chunks must be in [1, 4096]");
         ctx->stream_chunks = value;
@@ -775,7 +771,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         if (t) pre.push_back({reinterpret_cast<void **>(t), sizeof(uint32_t) * Tg});
     pre.push_back({reinterpret_cast<void **>(&S.tok_z), sizeof(uint16_t) * Tg});
     pre.push_back({reinterpret_cast<void **>(&S.z_doc), sizeof(uint16_t) * (Tg + 8)});
-    if (tile_layout && ctx->zdoc) pre.push_back({reinterpret_cast<void **>(&S.tok_doc), sizeof(uint32_t) * Tg});
     const size_t nwk_bytes = sizeof(int32_t) * (static_cast<size_t>(V) * K + K);
     pre.push_back({reinterpret_cast<void **>(&S.nwk), nwk_bytes});
     if (S.sweep_fused) pre.push_back({reinterpret_cast<void **>(&S.nwk_alt), nwk_bytes});
@@ -791,35 +786,46 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     std::condition_variable cv;
     bool jobs_done = false;
     cudaError_t copy_err = cudaSuccess;
-    std::thread copier([&] {
+    // the device buffers are allocated by copier 0; then all copiers move the
+    // finished parts of the token tables (pageable host memory: the driver
+    // stages each copy, so several copies run at once from several threads)
+    bool alloc_done = false;
+    double copy_ms_total = 0.0, alloc_ms = 0.0;
+    auto copier_main = [&](int id) {
         cudaSetDevice(ctx->device);
         cudaStream_t cs = nullptr;
         cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
-        pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
-        const auto c0 = std::chrono::steady_clock::now();
-        for (auto &pa : pre) {
-            if (copy_err != cudaSuccess) break;
-            void *q = nullptr;
-            copy_err = cudaMalloc(&q, std::max<size_t>(pa.second, 1));
-            if (copy_err != cudaSuccess) {
-                pre_fail_bytes = pa.second;
-                break;
+        if (id == 0) {
+            const auto c0 = std::chrono::steady_clock::now();
+            cudaError_t err = cudaSuccess;
+            for (auto &pa : pre) {
+                void *q = nullptr;
+                err = cudaMalloc(&q, std::max<size_t>(pa.second, 1));
+                if (err != cudaSuccess) {
+                    pre_fail_bytes = pa.second;
+                    break;
+                }
+                *pa.first = q;
+                pre_done.push_back(q);
             }
-            *pa.first = q;
-            pre_done.push_back(q);
+            std::lock_guard<std::mutex> lk(mu);
+            if (err != cudaSuccess && copy_err == cudaSuccess) copy_err = err;
+            alloc_done = true;
+            alloc_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - c0).count();
+            cv.notify_all();
         }
-        const auto c1 = std::chrono::steady_clock::now();
         double copy_ms = 0.0;
         for (;;) {
             Job j;
             {
                 std::unique_lock<std::mutex> lk(mu);
-                cv.wait(lk, [&] { return !jobs.empty() || jobs_done; });
+                cv.wait(lk, [&] { return alloc_done && (!jobs.empty() || jobs_done); });
                 if (jobs.empty()) break;
                 j = jobs.front();
                 jobs.erase(jobs.begin());
+                if (copy_err != cudaSuccess) continue;  // drain the queue
             }
-            if (copy_err != cudaSuccess) continue;  // drain the queue
+            const auto j0 = std::chrono::steady_clock::now();
             cudaError_t r = cudaSuccess;
             const size_t np = (j.p1 - j.p0) * sizeof(uint32_t), nt = (j.t1 - j.t0) * sizeof(uint32_t);
             if (np && r == cudaSuccess && H.tok_row.data())
@@ -828,22 +834,32 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                 r = cudaMemcpyAsync(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np, cudaMemcpyHostToDevice, cs);
             if (nt && r == cudaSuccess)
                 r = cudaMemcpyAsync(S.doc_map + j.t0, H.doc_map.data() + j.t0, nt, cudaMemcpyHostToDevice, cs);
-            const auto j0 = std::chrono::steady_clock::now();
             if (r == cudaSuccess) r = cudaStreamSynchronize(cs);
             copy_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - j0).count();
-            if (r != cudaSuccess && copy_err == cudaSuccess) copy_err = r;
+            if (r != cudaSuccess) {
+                std::lock_guard<std::mutex> lk(mu);
+                if (copy_err == cudaSuccess) copy_err = r;
+            }
         }
         if (cs) cudaStreamDestroy(cs);
-        if (std::getenv("LDA_TIMING"))
-            std::fprintf(stderr, "[lda]   copier: device allocation %.1f ms, H2D waits %.1f ms\n",
-                         std::chrono::duration<double, std::milli>(c1 - c0).count(), copy_ms);
-    });
+        std::lock_guard<std::mutex> lk(mu);
+        copy_ms_total += copy_ms;
+    };
+    pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
+    constexpr int kCopiers = 4;
+    std::vector<std::thread> copiers;
+    for (int id = 0; id < kCopiers; ++id) copiers.emplace_back(copier_main, id);
     auto on_final = [&](uint64_t p0, uint64_t p1, uint64_t t0, uint64_t t1) {
         {
+            // in pieces of <= 4 M tokens (16 MB), so that the copiers share a tile
             std::lock_guard<std::mutex> lk(mu);
-            jobs.push_back(Job{p0, p1, t0, t1});
+            const uint64_t piece = uint64_t(1) << 22;
+            const uint64_t n = std::max<uint64_t>(1, std::max((p1 - p0 + piece - 1) / piece, (t1 - t0 + piece - 1) / piece));
+            for (uint64_t q = 0; q < n; ++q)
+                jobs.push_back(Job{p0 + (p1 - p0) * q / n, p0 + (p1 - p0) * (q + 1) / n, t0 + (t1 - t0) * q / n,
+                                   t0 + (t1 - t0) * (q + 1) / n});
         }
-        cv.notify_one();
+        cv.notify_all();
     };
     // the large-K sampler copies a table of 8·K bytes per work item: its items
     // grow with K (tiles and the tail threshold scaled by K/1024; measured at
@@ -858,8 +874,11 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
     }
-    cv.notify_one();
-    copier.join();
+    cv.notify_all();
+    for (auto &t : copiers) t.join();
+    if (std::getenv("LDA_TIMING"))
+        std::fprintf(stderr, "[lda]   copiers: device allocation %.1f ms, H2D %.1f ms (summed over %d threads)\n",
+                     alloc_ms, copy_ms_total, kCopiers);
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
     // a range error of the layout takes precedence over an allocation error
     if (!e.empty()) {
@@ -977,7 +996,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
     if (tile_layout) KL(lda::launch_tok_row(S, ctx->stream));
-    KL(lda::launch_inv_map(S, ctx->stream));
     // a1: random init (t = 0), then the count rebuild.
     CU(cudaStreamSynchronize(ctx->stream));
     lda::tmark("H2D copies");
@@ -1063,8 +1081,7 @@ int lda_iterate(lda_ctx *ctx, int32_t n) {
         CU(cudaEventRecord(E[2], ctx->stream));
         // θ update (depends only on z) on the compute stream while ϕ is
         // summed over the ranks on the comm stream (§6.2)
-        KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches,
-                             /*gathered=*/S.tok_doc != nullptr));
+        KL(lda::launch_theta(S, ctx->d_stat_log + 2 * static_cast<size_t>(s), ctx->stream, &launches));
         CU(cudaEventRecord(E[3], ctx->stream));
         if (ctx->world > 1) {
             const size_t K = static_cast<size_t>(S.K);

@@ -555,8 +555,6 @@ struct TileArgs {
     const uint64_t *cbase;     // V: canonical index of the rank's first token of each word
     const uint32_t *tok_row;   // word-major: θ row of the token's doc (32-byte units, 128-byte aligned)
     uint16_t *z;
-    const uint32_t *tok_doc;   // option zdoc: word-major -> document-order token index (doc_map's inverse), or null
-    uint16_t *z_doc;           // ... and z in document order, written by the sampler (the θ rebuild then skips its gather)
     const uint32_t *rows;
     const int32_t *nwk;        // frozen counts (V*K, n_k after)
     const double *denom;       // K: n_k + Vβ
@@ -1078,7 +1076,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
 // Exact fp64 redraw of a batch's uncertain tokens (one at a time by the
 // warp), then z and the fused recount (ϕ update, L1273-1285).
 __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool flag, int z, uint32_t row,
-                                            uint32_t nnz, uint32_t x0, uint32_t p, uint32_t zi, const int32_t *nwk_row,
+                                            uint32_t nnz, uint32_t x0, uint32_t p, const int32_t *nwk_row,
                                             int32_t *row_next, int *nkh, const double *B, int G, int gsz,
                                             unsigned &n_exact) {
     // nkh: the n_k histogram -- the CTA's in shared memory, or the global
@@ -1101,7 +1099,6 @@ __device__ __forceinline__ void tile_finish(const TileArgs &a, bool take, bool f
     // ---- z and the fused recount
     if (take) {
         a.z[p] = static_cast<uint16_t>(z);
-        if (a.z_doc) a.z_doc[zi] = static_cast<uint16_t>(z);
     }
     if (take && a.recount) {
         const unsigned act = __activemask();
@@ -1248,10 +1245,8 @@ __global__ void __launch_bounds__(32 * LDA_TILE_WPC, LDA_TILE_MINB) sweep_tile_k
         int z;
         bool flag;
         uint32_t x0;
-        // zdoc: the token's document-order index, loaded now so that the draw covers its latency
-        const uint32_t zi = a.tok_doc && take ? ld_stream_u32(a.tok_doc + p) : 0u;
         tile_draw(a, take, c0, nl, row, crank, cb, Q64, gS, blk, p32, L32, Pc, NC, z, flag, x0);
-        tile_finish(a, take, flag, z, row, nnz, x0, p, zi, nwk_row, row_next, nkh, Pc, NC, 128, n_exact);
+        tile_finish(a, take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, Pc, NC, 128, n_exact);
         // ---- advance
         row = n_row;
         crank = n_crank;
@@ -1405,10 +1400,9 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
                 int z;
                 bool flag;
                 uint32_t x0;
-                const uint32_t zi = a.tok_doc && hd.take ? ld_stream_u32(a.tok_doc + p) : 0u;
                 tile_draw<GNK>(a, hd.take, hd.c0, hd.nl, row, crank, cb, Q64, gS, blk, p32, L32, Pc, NC, z,
                                flag, x0);
-                tile_finish(a, hd.take, flag, z, row, nnz, x0, p, zi, nwk_row, row_next, nkh, Pc, NC, GNK ? 32 : 128,
+                tile_finish(a, hd.take, flag, z, row, nnz, x0, p, nwk_row, row_next, nkh, Pc, NC, GNK ? 32 : 128,
                             n_exact);
                 b0 += static_cast<uint32_t>(hd.nb);
             }
@@ -1446,13 +1440,6 @@ __global__ void tok_row_kernel(const uint32_t *__restrict__ doc_ptr32, const uin
         const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1], row = row_off32[d];
         for (uint32_t i = s + lane; i < e; i += 32) tok_row[doc_map[i]] = row;
     }
-}
-
-// option zdoc: tok_doc[doc_map[i]] = i (the inverse of the doc-word map)
-__global__ void inv_map_kernel(const uint32_t *__restrict__ doc_map, uint32_t *__restrict__ tok_doc, int64_t T) {
-    for (int64_t i = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; i < T;
-         i += static_cast<int64_t>(gridDim.x) * blockDim.x)
-        tok_doc[doc_map[i]] = static_cast<uint32_t>(i);
 }
 
 __global__ void zero_rows_kernel(const int32_t *__restrict__ words, int64_t n, int32_t *__restrict__ nwk,
@@ -2001,12 +1988,6 @@ int launch_tok_row(const DevState &s, void *stream) {
     return cudaGetLastError();
 }
 
-int launch_inv_map(const DevState &s, void *stream) {
-    if (s.T > 0 && s.tok_doc)
-        inv_map_kernel<<<s.num_sms * 8, 256, 0, static_cast<cudaStream_t>(stream)>>>(s.doc_map, s.tok_doc, s.T);
-    return cudaGetLastError();
-}
-
 int launch_gather_z(const DevState &s, uint16_t *zd, void *stream) {
     const int64_t thr = (s.T + 7) / 8;
     if (thr > 0)
@@ -2021,12 +2002,12 @@ int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream) {
     return cudaGetLastError();
 }
 
-int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches, bool gathered) {
+int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches) {
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     if ((e = cudaMemsetAsync(stat_out, 0, 2 * sizeof(unsigned long long), st)) != cudaSuccess) return e;
     const int64_t thr = (s.T + 7) / 8;
-    if (thr > 0 && !gathered) {
+    if (thr > 0) {
         gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, st>>>(s.doc_map, s.tok_z, s.z_doc, s.T);
         ++*launches;
     }
@@ -2103,8 +2084,6 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.cbase = s.cbase;
         ta.tok_row = s.tok_row;
         ta.z = s.tok_z;
-        ta.tok_doc = s.tok_doc;
-        ta.z_doc = s.tok_doc ? s.z_doc : nullptr;
         ta.rows = s.rows;
         ta.nwk = s.nwk;
         ta.denom = s.denom;

@@ -150,7 +150,6 @@ struct DevState {
     uint32_t *doc_map = nullptr;    // T
     uint32_t *tok_crank = nullptr;  // T (word-major); null for the tile samplers (ranks from the items)
     uint16_t *z_doc = nullptr;      // T, z in document order (θ rebuild, phase A)
-    uint32_t *tok_doc = nullptr;    // option zdoc (tile samplers): word-major -> document-order index
     uint32_t *doc_ptr32 = nullptr;  // D+1
     uint32_t *row_off32 = nullptr;  // D
     Seg *segs = nullptr;
@@ -205,10 +204,7 @@ int launch_init(const DevState &s, void *stream);
 int launch_tok_row(const DevState &s, void *stream);
 int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0 = 0, int64_t rc1 = -1,
                    bool first = true);
-// gathered: z_doc already holds this sweep's z in document order (option zdoc)
-int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches,
-                 bool gathered = false);
-int launch_inv_map(const DevState &s, void *stream);
+int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, int *launches);
 // z in document order <-> word-major, through doc_map (device buffers of T entries; zd 16-byte aligned)
 int launch_gather_z(const DevState &s, uint16_t *zd, void *stream);
 int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream);

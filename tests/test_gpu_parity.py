@@ -164,8 +164,8 @@ def test_nytimes_shaped_midsize_many_chunks():
     z_ref = g.z()
     for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
                  dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3),
-                 dict(tile_tokens=0), dict(tile_tokens=20_000, fused_recount=1), dict(zdoc=1),
-                 dict(zdoc=1, sampler=3, tile_tokens=30_000)]:
+                 dict(tile_tokens=0), dict(tile_tokens=20_000, fused_recount=1),
+                 dict(sampler=3, tile_tokens=30_000)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
