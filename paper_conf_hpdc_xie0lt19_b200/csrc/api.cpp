@@ -688,11 +688,42 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     const int64_t Dg = doc_end - doc_begin;
     bool range_err = false;
     lda::tmark(nullptr);
-    // one pass over the words: validation + the local word histogram
+    // the CUDA setup (streams, kernel configuration: the process's first
+    // kernel-attribute calls load the module, ~80 ms) runs in a helper thread
+    // while the host validates the words
+    lda::DevState &S = ctx->S;
+    S.K = ctx->K;
+    S.exclude_self = ctx->exclude_self;
+    S.sampler = ctx->sampler;
+    S.certify_slack = static_cast<double>(ctx->certify_slack);
+    S.tile_fused = ctx->fused_recount != 0 && ctx->stream_chunks == 1;  // chunks: the recount kernel accumulates
+    cudaError_t setup_err = cudaSuccess;
+    std::thread setup([&] {
+        cudaError_t e = cudaSetDevice(ctx->device);
+        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking);
+        if (e == cudaSuccess) e = static_cast<cudaError_t>(lda::configure_kernels(S));
+        setup_err = e;
+    });
+    // the document offsets first; the words (one pass: validation + the
+    // local word histogram) here too unless the layout's own per-tile count
+    // pass does both (one rank, tile samplers, resident corpus)
     std::vector<int64_t> local(ctx->V, 0);
-    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, local.data(), ctx->threads);
-    lda::tmark("validate + word histogram");
+    std::string v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, nullptr, ctx->threads, false);
+    setup.join();
     if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
+    if (setup_err != cudaSuccess) {
+        // an invalid corpus is reported as such even without a device
+        v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, nullptr, ctx->threads);
+        if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
+        return fail(ctx, LDA_ECUDA, std::string("CUDA setup: ") + cudaGetErrorString(setup_err));
+    }
+    const bool words_in_layout = ctx->world == 1 && ctx->stream_chunks == 1 && (S.sweep_tile || S.sweep_tile_cta);
+    if (!words_in_layout) {
+        v = lda::validate_corpus(doc_ptr, words, Dg, ctx->V, &range_err, local.data(), ctx->threads);
+        if (!v.empty()) return fail(ctx, range_err ? LDA_ERANGE : LDA_EINVAL, v);
+    }
+    lda::tmark("validate (+ word histogram) || CUDA setup");
     const int64_t Tg = doc_ptr[Dg];
     // θ row storage: 128-byte aligned rows of min(L_d, K) + 1 words, in
     // 32-byte units (the layout's row_off32; checked against H.rows32 after
@@ -704,8 +735,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     const int32_t V = ctx->V, K = ctx->K;
 
     CU(cudaSetDevice(ctx->device));
-    CU(cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking));
-    CU(cudaStreamCreateWithFlags(&ctx->comm_stream, cudaStreamNonBlocking));
 
     // Local word histogram -> canonical bases.  c for rank g's tokens of word
     // w starts at Σ_{w'<w} T(w') + Σ_{g'<g} T_{g'}(w)   (X18, §8(c) step 2).
@@ -722,17 +751,11 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         std::copy(local.begin(), local.end(), all.begin());
     }
     std::vector<int64_t> cbase(V);
-    int64_t run = 0;
-    lda_canonical_bases(V, ctx->world, ctx->rank, all.data(), cbase.data(), &run);
-    ctx->T_global = run;
-
-    lda::DevState &S = ctx->S;
-    S.K = K;
-    S.exclude_self = ctx->exclude_self;
-    S.sampler = ctx->sampler;
-    S.certify_slack = static_cast<double>(ctx->certify_slack);
-    S.tile_fused = ctx->fused_recount != 0 && ctx->stream_chunks == 1;  // chunks: the recount kernel accumulates
-    KL(lda::configure_kernels(S));
+    if (!words_in_layout) {
+        int64_t run = 0;
+        lda_canonical_bases(V, ctx->world, ctx->rank, all.data(), cbase.data(), &run);
+        ctx->T_global = run;
+    }
 
     lda::HostLayout &H = ctx->H;
     // the per-token tables go to the device tile by tile, copied by a helper
@@ -901,7 +924,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
                                       tile_layout ? 2 : 0,
                                       ctx->tail_per_tile * kscale, H,
-                                      on_final, local.data(), /*host_tok_row=*/!tile_layout);
+                                      on_final, words_in_layout ? nullptr : local.data(),
+                                      /*host_tok_row=*/!tile_layout);
     {
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
@@ -913,10 +937,17 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         std::fprintf(stderr, "[lda]   copiers: device allocation %.1f ms, H2D %.1f ms (summed over %d threads)\n",
                      alloc_ms, copy_ms_total, kCopiers);
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
-    // a range error of the layout takes precedence over an allocation error
+    // a layout error (invalid word id, or a range) takes precedence over an allocation error
     if (!e.empty()) {
         cudaGetLastError();
+        if (e.rfind("invalid: ", 0) == 0) return fail(ctx, LDA_EINVAL, e.substr(9));
         return fail(ctx, LDA_ERANGE, e);
+    }
+    if (words_in_layout) {
+        // one rank: canonical bases from the layout's word counts (X18)
+        int64_t run = 0;
+        lda_canonical_bases(V, 1, 0, H.word_count.data(), cbase.data(), &run);
+        ctx->T_global = run;
     }
     if (copy_err != cudaSuccess) {
         cudaGetLastError();

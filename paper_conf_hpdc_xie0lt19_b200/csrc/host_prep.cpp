@@ -92,7 +92,7 @@ void word_histogram(const int32_t *words, int64_t T, int32_t V, int nthreads, in
 }
 
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
-                            bool *range_error, int64_t *word_counts, int nthreads) {
+                            bool *range_error, int64_t *word_counts, int nthreads, bool check_words) {
     *range_error = false;
     if (D < 0) return "negative document count";
     if (!doc_ptr) return "doc_ptr is NULL";
@@ -112,6 +112,7 @@ std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_
         return "more than 2^32-1 tokens on one rank";
     }
     if (T > 0 && !words) return "words is NULL";
+    if (!check_words) return "";
     int nth = host_threads(nthreads);
     std::vector<int64_t> bad(nth, -1);
     // with word_counts: the same pass counts the tokens of every word
@@ -191,10 +192,53 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     tile_doc.push_back(D);
     const int ndt = static_cast<int>(tile_doc.size()) - 1;  // document tiles
 
-    // Word counts of the shard (parallel histogram).
+    // Word counts of the shard.  Without word_counts the word ids are also
+    // validated here (the caller skipped its own pass over the words): by
+    // the per-tile counts of the thread-per-tile pass below, or one parallel
+    // histogram.
+    const bool tile_fast = sampler == 2 && ndt >= 2 * nthreads;  // one host thread per tile (see below)
     std::vector<int64_t> wc(V, 0);
-    if (word_counts) std::copy(word_counts, word_counts + V, wc.begin());
-    else word_histogram(words, T, V, nthreads, wc.data());
+    std::vector<std::vector<uint32_t>> pre_cnt;  // tile_fast: the doc tiles' word counts
+    if (word_counts) {
+        std::copy(word_counts, word_counts + V, wc.begin());
+    } else if (tile_fast) {
+        pre_cnt.resize(ndt);
+        std::atomic<int> next_tile{0};
+        std::atomic<int64_t> bad{-1};
+        std::vector<std::thread> th;
+        auto count = [&] {
+            for (int b; (b = next_tile.fetch_add(1)) < ndt;) {
+                auto &tc = pre_cnt[b];
+                tc.assign(V, 0);
+                const int64_t i1 = doc_ptr[tile_doc[b + 1]];
+                for (int64_t i = doc_ptr[tile_doc[b]]; i < i1; ++i) {
+                    const uint32_t w = static_cast<uint32_t>(words[i]);
+                    if (w >= static_cast<uint32_t>(V)) {
+                        bad = i;
+                        break;
+                    }
+                    tc[w]++;
+                }
+            }
+        };
+        for (int t = 1; t < nthreads; ++t) th.emplace_back(count);
+        count();
+        for (auto &x : th) x.join();
+        if (bad >= 0)
+            return "invalid: word id " + std::to_string(words[bad.load()]) + " at token " +
+                   std::to_string(bad.load()) + " outside [0, V)";
+        parallel_for(nthreads, V, [&](int, int64_t w0, int64_t w1) {
+            for (int64_t w = w0; w < w1; ++w) {
+                int64_t c = 0;
+                for (int b = 0; b < ndt; ++b) c += pre_cnt[b][w];
+                wc[w] = c;
+            }
+        });
+    } else {
+        bool range_err = false;
+        std::string v = validate_corpus(doc_ptr, words, D, V, &range_err, wc.data(), nthreads);
+        if (!v.empty()) return "invalid: " + v;
+    }
     L.word_count = wc;
 
     // Tail words (tile sampler only): words with too few tokens per document
@@ -266,7 +310,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     std::vector<std::vector<uint32_t>> cnext(nthreads, std::vector<uint32_t>(V));
 
     uint64_t pos = 0;  // start of the current tile's segment
-    if (tile_layout && ndt >= 2 * nthreads) {
+    if (tile_fast) {
         // Many tiles (PubMed shape: 54 on 16 host threads): one thread per
         // tile instead of every tile split over all threads, so the per-word
         // work (V-length count arrays, their sums and prefixes) is done once
@@ -287,9 +331,13 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         tile_threads([&] {
             for (int b; (b = next_tile.fetch_add(1)) < ndt;) {
                 auto &tc = tile_cnt[b];
-                tc.assign(V, 0);
                 const int64_t i0 = doc_ptr[tile_doc[b]], i1 = doc_ptr[tile_doc[b + 1]];
-                for (int64_t i = i0; i < i1; ++i) tc[words[i]]++;
+                if (!pre_cnt.empty()) {
+                    tc.swap(pre_cnt[b]);  // counted (and validated) above
+                } else {
+                    tc.assign(V, 0);
+                    for (int64_t i = i0; i < i1; ++i) tc[words[i]]++;
+                }
                 int64_t tt = 0;
                 for (int32_t w = 0; w < V; ++w)
                     if (tail[w]) tt += tc[w];
@@ -347,7 +395,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         });
         pos = pos_tile[ndt];
     }
-    for (int b = 0; b < ndt && !(tile_layout && ndt >= 2 * nthreads); ++b) {
+    for (int b = 0; b < ndt && !tile_fast; ++b) {
         const uint64_t pos_tile = pos;
         const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
         // the tile's documents in nth contiguous parts (original order), balanced by tokens

@@ -110,7 +110,9 @@ struct HostLayout {
 // doc_map over document-major tokens [tok_begin, tok_end) are final (after
 // each document tile, and for the tail region at the end) -- the caller can
 // start their host->device copies while the next tile is prepared.
-// Returns "" on success, else an error message.
+// Returns "" on success, else an error message ("invalid: ..." for an invalid
+// corpus: a word id outside [0, V) when word_counts is null and the layout
+// validated the ids itself; anything else is a range error).
 std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                          int32_t K, const int64_t *cbase, int64_t tile_tokens,
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
@@ -123,7 +125,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
 // doc exceeds 65535 tokens.
 std::string validate_corpus(const int64_t *doc_ptr, const int32_t *words, int64_t D, int32_t V,
                             bool *range_error, int64_t *word_counts = nullptr,  // V counts, if wanted
-                            int nthreads = 0);                                    // 0: all host threads
+                            int nthreads = 0,                                     // 0: all host threads
+                            bool check_words = true);  // false: offsets and sizes only (the layout checks the ids)
 
 int host_threads(int requested);
 

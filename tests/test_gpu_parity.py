@@ -308,3 +308,21 @@ def test_convergence_harness_ll_rises():
     assert [p["sweep"] for p in pts] == [0, 5, 10, 15, 20]
     assert all(b["ms"] > a["ms"] for a, b in zip(pts, pts[1:]))
     assert pts[-1]["ll_per_token"] > pts[0]["ll_per_token"] + 0.05
+
+
+@pytest.mark.parametrize("tile_tokens", [0, 500])
+def test_invalid_word_ids_rejected_on_device(tile_tokens):
+    """With one rank and a tile sampler the word ids are validated by the
+    layout's own count pass (no separate pass over the words): an id outside
+    [0, V) must still fail with LDA_EINVAL -- with one tile and with many
+    (the thread-per-tile pass)."""
+    import paper_conf_hpdc_xie0lt19_b200 as L
+    doc_ptr, words = _corpus(400, 300, 30_000, 0.5, 16, 3)
+    for bad in (300, -1, 1 << 20):
+        w = words.copy()
+        w[len(w) // 2] = bad
+        with pytest.raises(L.LDAError) as e:
+            U.gpu_model(400, 300, 16, 0.5, 0.01, doc_ptr, w, 1, tile_tokens=tile_tokens)
+        assert e.value.code == L.LDA_EINVAL, e.value
+    g = U.gpu_model(400, 300, 16, 0.5, 0.01, doc_ptr, words, 1, tile_tokens=tile_tokens)
+    U.check_invariants_gpu(g, doc_ptr, words)
