@@ -688,6 +688,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     const int64_t Dg = doc_end - doc_begin;
     bool range_err = false;
     lda::tmark(nullptr);
+    const auto load_t0 = std::chrono::steady_clock::now();
     // the CUDA setup (streams, kernel configuration: the process's first
     // kernel-attribute calls load the module, ~80 ms) runs in a helper thread
     // while the host validates the words
@@ -813,7 +814,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // finished parts of the token tables (pageable host memory: the driver
     // stages each copy, so several copies run at once from several threads)
     bool alloc_done = false;
-    double copy_ms_total = 0.0, alloc_ms = 0.0;
+    double copy_ms_total = 0.0, memcpy_ms_total = 0.0, alloc_ms = 0.0, last_copy_end = 0.0, layout_end = 0.0;
     // page-locked staging ring: the copiers memcpy a finished piece of a token
     // table into a slot (in parallel, from several threads) and DMA it from
     // there -- the driver's own pageable path serialises the copies at ~10 GB/s
@@ -857,7 +858,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             alloc_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - c0).count();
             cv.notify_all();
         }
-        double copy_ms = 0.0;
+        double copy_ms = 0.0, memcpy_ms = 0.0;
         for (;;) {
             Job j;
             {
@@ -887,7 +888,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                     return;
                 }
                 char *buf = stage + static_cast<size_t>(slot) * kSlotBytes;
+                const auto m0 = std::chrono::steady_clock::now();
                 std::memcpy(buf, src, bytes);
+                memcpy_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - m0).count();
                 r = cudaMemcpyAsync(dst, buf, bytes, cudaMemcpyHostToDevice, cs);
                 if (r == cudaSuccess) r = cudaStreamSynchronize(cs);
                 std::lock_guard<std::mutex> lk(mu);
@@ -906,6 +909,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         if (cs) cudaStreamDestroy(cs);
         std::lock_guard<std::mutex> lk(mu);
         copy_ms_total += copy_ms;
+        memcpy_ms_total += memcpy_ms;
+        last_copy_end = std::max(last_copy_end, std::chrono::duration<double, std::milli>(
+                                                    std::chrono::steady_clock::now() - load_t0).count());
     };
     pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
     std::vector<std::thread> copiers;
@@ -935,13 +941,16 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     {
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
+        layout_end = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - load_t0).count();
     }
     cv.notify_all();
     for (auto &t : copiers) t.join();
     if (stage) cudaFreeHost(stage);
     if (std::getenv("LDA_TIMING"))
-        std::fprintf(stderr, "[lda]   copiers: device allocation %.1f ms, H2D %.1f ms (summed over %d threads)\n",
-                     alloc_ms, copy_ms_total, kCopiers);
+        std::fprintf(stderr,
+                     "[lda]   copiers: device allocation %.1f ms, H2D %.1f ms (of which host memcpy %.1f; summed "
+                     "over %d threads); layout end at %.1f ms, last copy end at %.1f ms (from the load start)\n",
+                     alloc_ms, copy_ms_total, memcpy_ms_total, kCopiers, layout_end, last_copy_end);
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
     // a layout error (invalid word id, or a range) takes precedence over an allocation error
     if (!e.empty()) {
