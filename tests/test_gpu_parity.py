@@ -165,7 +165,7 @@ def test_nytimes_shaped_midsize_many_chunks():
     for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
                  dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3),
                  dict(tile_tokens=0), dict(tile_tokens=20_000, fused_recount=1),
-                 dict(sampler=3, tile_tokens=30_000)]:
+                 dict(sampler=3, tile_tokens=30_000), dict(theta_fused=1)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
@@ -187,8 +187,8 @@ def test_exclude_self_lockstep():
     assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
-@pytest.mark.parametrize("sampler", [2, 3, 0])
-def test_edge_cases(sampler):
+@pytest.mark.parametrize("sampler,extra", [(2, {}), (3, {}), (0, {}), (2, dict(theta_fused=1))])
+def test_edge_cases(sampler, extra):
     rng = np.random.default_rng(4)
     # empty docs, single-token docs, a 65535-token doc, absent words, D=1
     L_d = np.array([0, 1, 0, 5, 65535, 1, 0, 3] + list(rng.integers(0, 20, 50)), np.int64)
@@ -197,7 +197,7 @@ def test_edge_cases(sampler):
     words = rng.integers(0, V // 2, size=doc_ptr[-1]).astype(np.int32)   # words >= 150 absent
     D, K = len(L_d), 40
     o = U.oracle_for(D, V, K, 0.3, 0.02, doc_ptr, words, 77)
-    g = U.gpu_model(D, V, K, 0.3, 0.02, doc_ptr, words, 77, chunk_tokens=64, sampler=sampler)
+    g = U.gpu_model(D, V, K, 0.3, 0.02, doc_ptr, words, 77, chunk_tokens=64, sampler=sampler, **extra)
     assert np.array_equal(g.z(), o.z)
     U.check_counts_equal(g, o)
     bad, unexc = U.lockstep(g, o, 3)
