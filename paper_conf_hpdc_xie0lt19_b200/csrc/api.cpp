@@ -57,7 +57,6 @@ struct lda_ctx {
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int64_t comm_pipeline = 4;  // world > 1: word ranges whose rows are exchanged as soon as recounted (f1)
-    int theta_fused = 0;        // θ rebuild reads z through doc_map, software-pipelined (no z_doc gather)
     int threads = 0;
     // distribution: the exchange of Eq. 4 (NCCL or the in-process peer group)
     int32_t rank = 0, world = 1;
@@ -573,9 +572,6 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "certify_slack") {
         if (value < 1 || value > (int64_t(1) << 40)) return fail(ctx, LDA_EINVAL, "certify_slack out of range");
         ctx->certify_slack = value;
-    } else if (k == "theta_fused") {
-        if (value != 0 && value != 1) return fail(ctx, LDA_EINVAL, "theta_fused must be 0 or 1");
-        ctx->theta_fused = static_cast<int>(value);
     } else if (k == "stream_chunks") {
         if (value < 1 || value > 4096) return fail(ctx, LDA_EINVAL, "stream_chunks must be in [1, 4096]");
         ctx->stream_chunks = value;
@@ -702,7 +698,6 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.sampler = ctx->sampler;
     S.certify_slack = static_cast<double>(ctx->certify_slack);
     S.tile_fused = ctx->fused_recount != 0 && ctx->stream_chunks == 1;  // chunks: the recount kernel accumulates
-    S.theta_fused = ctx->theta_fused != 0;
     cudaError_t setup_err = cudaSuccess;
     std::thread setup([&] {
         cudaError_t e = cudaSetDevice(ctx->device);

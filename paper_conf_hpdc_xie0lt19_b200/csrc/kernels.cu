@@ -1635,118 +1635,6 @@ __global__ void theta_kernel(const uint32_t *__restrict__ doc_ptr32, const uint3
     }
 }
 
-// The θ rebuild with the gather fused in (option theta_fused): a warp per
-// document as in theta_kernel, but z is read through the doc-word map
-// directly, software-pipelined over the warp's documents -- while document j
-// is histogrammed, the z of document j+1 (through the map positions loaded
-// one document earlier) and the map positions of document j+2 are in flight
-// (the first 32·kThetaPipe tokens of each document; longer documents finish
-// with direct dependent loads).  Saves the z_doc round trip of
-// gather_z_kernel.
-constexpr int kThetaPipe = 8;
-
-template <int TS>
-__global__ void theta_fused_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
-                                   const uint32_t *__restrict__ doc_map, const uint16_t *__restrict__ z,
-                                   uint32_t *__restrict__ rows, int64_t D, int K,
-                                   unsigned long long *__restrict__ stat) {
-    extern __shared__ uint32_t smem_u[];
-    const int Kw = (K + 31) >> 5;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, wpb = blockDim.x >> 5;
-    uint32_t *cnt = smem_u + static_cast<size_t>(warp) * (K + Kw);
-    uint32_t *bits = cnt + K;
-    for (int k = lane; k < K + Kw; k += 32) cnt[k] = 0u;
-    __syncwarp();
-    unsigned long long s_lnnz = 0, s_nnz = 0;
-    const int64_t nw = static_cast<int64_t>(gridDim.x) * wpb;
-    const int64_t d0 = static_cast<int64_t>(blockIdx.x) * wpb + warp;
-    constexpr uint32_t NONE = 0xFFFFFFFFu;
-    auto bounds = [&](int64_t d, uint32_t &bs, uint32_t &be, uint32_t &bo) {
-        bs = be = bo = 0;
-        if (d < D) {
-            bs = __ldg(doc_ptr32 + d);
-            be = __ldg(doc_ptr32 + d + 1);
-            bo = __ldg(row_off32 + d);
-        }
-    };
-    auto load_map = [&](uint32_t bs, uint32_t be, uint32_t (&pm)[kThetaPipe]) {
-#pragma unroll
-        for (int r = 0; r < kThetaPipe; ++r) {
-            const uint32_t i = bs + 32u * r + lane;
-            pm[r] = i < be ? __ldcs(doc_map + i) : NONE;
-        }
-    };
-    auto load_z = [&](const uint32_t (&pm)[kThetaPipe], uint32_t (&zz)[kThetaPipe]) {
-#pragma unroll
-        for (int r = 0; r < kThetaPipe; ++r) zz[r] = pm[r] != NONE ? static_cast<uint32_t>(z[pm[r]]) : NONE;
-    };
-    // pipeline state: doc j (zc), doc j+1 (pm1 -> z next), doc j+2 (bounds)
-    uint32_t s0, e0, o0, s1, e1, o1, s2, e2, o2;
-    bounds(d0, s0, e0, o0);
-    bounds(d0 + nw, s1, e1, o1);
-    uint32_t pm[kThetaPipe], zc[kThetaPipe], zn[kThetaPipe];
-    load_map(s0, e0, pm);
-    load_z(pm, zc);
-    load_map(s1, e1, pm);
-    for (int64_t d = d0; d < D; d += nw) {
-        bounds(d + 2 * nw, s2, e2, o2);
-        load_z(pm, zn);               // doc j+1's topics
-        load_map(s2, e2, pm);         // doc j+2's map positions
-        uint32_t *row = rows + static_cast<size_t>(o0) * 8;
-        const uint32_t old_nnz = row[0];
-#pragma unroll
-        for (int r = 0; r < kThetaPipe; ++r)
-            if (zc[r] != NONE) {
-                atomicAdd(&cnt[zc[r]], 1u);
-                atomicOr(&bits[zc[r] >> 5], 1u << (zc[r] & 31));
-            }
-        for (uint32_t i = s0 + 32u * kThetaPipe + lane; i < e0; i += 32u) {  // long documents
-            const uint32_t k = z[__ldcs(doc_map + i)];
-            atomicAdd(&cnt[k], 1u);
-            atomicOr(&bits[k >> 5], 1u << (k & 31));
-        }
-        __syncwarp();
-        uint32_t base = 0;
-        for (int qb = 0; qb < Kw; qb += 32) {
-            const int qq = qb + lane;
-            uint32_t bw = qq < Kw ? bits[qq] : 0u;
-            const uint32_t pc = __popc(bw);
-            uint32_t incl = pc;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(kFull, incl, o);
-                if (lane >= o) incl += y;
-            }
-            uint32_t pos = base + incl - pc;
-            while (bw) {
-                const int b = __ffs(bw) - 1;
-                bw &= bw - 1;
-                const uint32_t k = static_cast<uint32_t>(qq) * 32 + b;
-                row[1 + pos++] = (k << TS) | cnt[k];
-                cnt[k] = 0u;
-            }
-            if (qq < Kw) bits[qq] = 0u;
-            base += __shfl_sync(kFull, incl, 31);
-        }
-        for (uint32_t i = 1u + base + lane; i < 1u + old_nnz; i += 32u) row[i] = 0u;
-        if (lane == 0) {
-            row[0] = base;
-            s_nnz += base;
-            s_lnnz += static_cast<unsigned long long>(e0 - s0) * base;
-        }
-        __syncwarp();
-        // rotate
-#pragma unroll
-        for (int r = 0; r < kThetaPipe; ++r) zc[r] = zn[r];
-        s0 = s1; e0 = e1; o0 = o1;
-        s1 = s2; e1 = e2; o1 = o2;
-    }
-    if (lane == 0) {
-        atomicAdd(stat + 0, s_lnnz);
-        atomicAdd(stat + 1, s_nnz);
-    }
-}
-
 // ---------------------------------------------------------------------------
 // Log-likelihood (X11), deterministic two-stage fp64 reductions.
 // ---------------------------------------------------------------------------
@@ -2040,11 +1928,6 @@ int configure_kernels(DevState &s) {
         if ((e = cudaFuncSetAttribute(tf, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       static_cast<int>(s.theta_smem))) != cudaSuccess)
             return e;
-        const void *tff = s.K > 16384 ? reinterpret_cast<const void *>(&theta_fused_kernel<kTSWide>)
-                                      : reinterpret_cast<const void *>(&theta_fused_kernel<kTS>);
-        if ((e = cudaFuncSetAttribute(tff, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      static_cast<int>(s.theta_smem))) != cudaSuccess)
-            return e;
         int tb = 1;
         if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&tb, tf, s.theta_block, s.theta_smem)) != cudaSuccess)
             return e;
@@ -2123,16 +2006,6 @@ int launch_theta(const DevState &s, unsigned long long *stat_out, void *stream, 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     cudaError_t e;
     if ((e = cudaMemsetAsync(stat_out, 0, 2 * sizeof(unsigned long long), st)) != cudaSuccess) return e;
-    if (s.theta_fused && !s.theta_gmem) {
-        if (s.K > 16384)
-            theta_fused_kernel<kTSWide><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(
-                s.doc_ptr32, s.row_off32, s.doc_map, s.tok_z, s.rows, s.D, s.K, stat_out);
-        else
-            theta_fused_kernel<kTS><<<s.theta_grid, s.theta_block, s.theta_smem, st>>>(
-                s.doc_ptr32, s.row_off32, s.doc_map, s.tok_z, s.rows, s.D, s.K, stat_out);
-        ++*launches;
-        return cudaGetLastError();
-    }
     const int64_t thr = (s.T + 7) / 8;
     if (thr > 0) {
         gather_z_kernel<<<static_cast<unsigned>((thr + 255) / 256), 256, 0, st>>>(s.doc_map, s.tok_z, s.z_doc, s.T);

@@ -195,7 +195,6 @@ struct DevState {
     int sweep_grid = 0, sweep_block = 0;
     int theta_grid = 0, theta_block = 0;
     bool recount_gmem = false, theta_gmem = false;  // K > 16384: K-length histograms in global scratch
-    bool theta_fused = false;       // option theta_fused: θ reads z through doc_map (no z_doc gather)
     int *recount_scratch = nullptr;                 // recount_gmem: num_sms*4 CTAs x 2K
     uint32_t *theta_scratch = nullptr;              // theta_gmem: theta_grid*8 warps x (K + K/32)
     size_t sweep_smem = 0, theta_smem = 0;

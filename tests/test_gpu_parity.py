@@ -165,7 +165,7 @@ def test_nytimes_shaped_midsize_many_chunks():
     for opts in [dict(chunk_tokens=100, recount_tokens=300), dict(tile_tokens=30_000),
                  dict(chunk_tokens=33, tile_tokens=7_000, recount_tokens=256, threads=3),
                  dict(tile_tokens=0), dict(tile_tokens=20_000, fused_recount=1),
-                 dict(sampler=3, tile_tokens=30_000), dict(theta_fused=1)]:
+                 dict(sampler=3, tile_tokens=30_000)]:
         h = U.gpu_model(cfg.D, cfg.V, cfg.K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, **opts)
         h.iterate(3)
         assert np.array_equal(h.z(), z_ref), opts
@@ -187,7 +187,7 @@ def test_exclude_self_lockstep():
     assert unexc == 0 and bad <= U.MAX_EXCUSED_FRAC * 30_000 * 3
 
 
-@pytest.mark.parametrize("sampler,extra", [(2, {}), (3, {}), (0, {}), (2, dict(theta_fused=1))])
+@pytest.mark.parametrize("sampler,extra", [(2, {}), (3, {}), (0, {}), (2, dict(tile_tokens=5_000))])
 def test_edge_cases(sampler, extra):
     rng = np.random.default_rng(4)
     # empty docs, single-token docs, a 65535-token doc, absent words, D=1
