@@ -238,6 +238,14 @@ int lda_layout_selfcheck(int64_t D, int32_t V, int32_t K, const int64_t *doc_ptr
                          int32_t sampler, int64_t tile_tokens, int64_t chunk_tokens, int64_t tail_per_tile,
                          int64_t *out_stats, char *msg, int32_t msg_cap);
 
+/* Diagnostic (tests): the library's device radix sort -- a stable LSD sort
+ * of n (key, value) pairs by the low `bits` bits of the keys (8 bits per
+ * pass; lda_load_corpus uses it to build the tile layout's doc-word map on
+ * the device).  Host arrays in, host arrays out; device scratch is
+ * allocated and freed by the call.  Returns 0, LDA_EINVAL or LDA_ECUDA. */
+int lda_debug_radix_sort(const uint32_t *keys, const uint32_t *vals, int64_t n, int32_t bits, uint32_t *out_keys,
+                         uint32_t *out_vals);
+
 /* Load this rank's documents [doc_begin, doc_end) of the global corpus,
  * randomly initialise every token's topic (L377-379; Philox at t = 0, X10)
  * and build n_wk, n_k and θ (allreduced across ranks when world > 1).

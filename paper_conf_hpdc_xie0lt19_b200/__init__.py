@@ -25,7 +25,7 @@ STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4:
 # every symbol include/lda.h declares
 ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_peer_group_create",
                "lda_init_peer", "lda_peer_group_destroy", "lda_partition_docs",
-               "lda_canonical_bases", "lda_layout_selfcheck",
+               "lda_canonical_bases", "lda_layout_selfcheck", "lda_debug_radix_sort",
                "lda_load_corpus", "lda_iterate", "lda_loglik", "lda_get_counts", "lda_get_stats",
                "lda_get_sweep_log", "lda_get_loglik_log", "lda_get_stream", "lda_set_z", "lda_destroy",
                "lda_last_error", "lda_version")
@@ -82,6 +82,7 @@ def lib():
             "lda_layout_selfcheck": ([_i64, _i32, _i32, _vp, _vp, _i32, _i64, _i64, _i64, _vp, ctypes.c_char_p,
                                       _i32], ctypes.c_int),
             "lda_load_corpus": ([_vp, _i64, _i64, _vp, _vp, _u64], ctypes.c_int),
+            "lda_debug_radix_sort": ([_vp, _vp, _i64, _i32, _vp, _vp], ctypes.c_int),
             "lda_iterate": ([_vp, _i32], ctypes.c_int),
             "lda_loglik": ([_vp, ctypes.POINTER(_f64)], ctypes.c_int),
             "lda_get_counts": ([_vp, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp], ctypes.c_int),
@@ -159,6 +160,17 @@ def lda_layout_selfcheck(doc_ptr, words, V, K, sampler=2, tile_tokens=0, chunk_t
     if r != 0:
         raise LDAError(r, f"lda_layout_selfcheck: {buf.value.decode()}")
     return dict(zip(("tiles", "items", "tail_words", "runs"), st.tolist()))
+
+
+def lda_debug_radix_sort(keys, vals, bits):
+    """The library's stable device radix sort (diagnostic): returns (keys, vals) sorted by the low `bits` key bits."""
+    k = np.ascontiguousarray(keys, np.uint32)
+    v = np.ascontiguousarray(vals, np.uint32)
+    if k.shape != v.shape:
+        raise LDAError(LDA_EINVAL, "keys and vals differ in length")
+    ok, ov = np.empty_like(k), np.empty_like(v)
+    _check(lib().lda_debug_radix_sort(_p(k), _p(v), len(k), int(bits), _p(ok), _p(ov)))
+    return ok, ov
 
 
 def lda_canonical_bases(word_counts, rank):

@@ -16,7 +16,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "liblda.so")
-SOURCES = ["api.cpp", "comm.cpp", "host_prep.cpp", "kernels.cu"]
+SOURCES = ["api.cpp", "comm.cpp", "host_prep.cpp", "kernels.cu", "layout_gpu.cu"]
 HEADERS = ["lda_internal.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

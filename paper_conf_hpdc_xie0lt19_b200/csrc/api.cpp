@@ -804,6 +804,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     const uint64_t pre_rows32 = r32;
     struct Job {
         uint64_t p0, p1, t0, t1;
+        int words = 0;  // 1: upload words[t0, t1) into S.tok_row (device layout: the sort's input)
     };
     std::vector<Job> jobs;
     std::mutex mu;
@@ -813,6 +814,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     // the device buffers are allocated by copier 0; then all copiers move the
     // finished parts of the token tables (pageable host memory: the driver
     // stages each copy, so several copies run at once from several threads)
+    const bool dev_scatter = tile_layout;  // doc_map built on the device (see below)
+    bool words_pinned = false;
     bool alloc_done = false;
     double copy_ms_total = 0.0, memcpy_ms_total = 0.0, alloc_ms = 0.0, last_copy_end = 0.0, layout_end = 0.0;
     // page-locked staging ring: the copiers memcpy a finished piece of a token
@@ -897,9 +900,19 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                 free_slots.push_back(slot);
                 cv.notify_all();
             };
-            if (H.tok_row.data()) put(S.tok_row + j.p0, H.tok_row.data() + j.p0, np);
-            if (S.tok_crank) put(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np);
-            put(S.doc_map + j.t0, H.doc_map.data() + j.t0, nt);
+            if (j.words) {
+                // the words (device layout); straight DMA when the caller's buffer is page-locked
+                if (words_pinned) {
+                    r = cudaMemcpyAsync(S.tok_row + j.t0, words + j.t0, nt, cudaMemcpyHostToDevice, cs);
+                    if (r == cudaSuccess) r = cudaStreamSynchronize(cs);
+                } else {
+                    put(S.tok_row + j.t0, words + j.t0, nt);
+                }
+            } else {
+                if (H.tok_row.data()) put(S.tok_row + j.p0, H.tok_row.data() + j.p0, np);
+                if (S.tok_crank) put(S.tok_crank + j.p0, H.tok_crank.data() + j.p0, np);
+                put(S.doc_map + j.t0, H.doc_map.data() + j.t0, nt);
+            }
             copy_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - j0).count();
             if (r != cudaSuccess) {
                 std::lock_guard<std::mutex> lk(mu);
@@ -914,6 +927,21 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                                     std::chrono::steady_clock::now() - load_t0).count());
     };
     pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
+    // the tile layout's doc-word map is built on the device (layout_gpu.cu):
+    // the copiers upload the words into S.tok_row (rebuilt from doc_map
+    // afterwards) while the host computes the counts
+    if (dev_scatter && Tg > 0) {
+        cudaPointerAttributes pa{};
+        if (cudaPointerGetAttributes(&pa, words) == cudaSuccess)
+            words_pinned = pa.type == cudaMemoryTypeHost;
+        cudaGetLastError();
+        const uint64_t piece = uint64_t(1) << 22;
+        for (uint64_t t0 = 0; t0 < static_cast<uint64_t>(Tg); t0 += piece) {
+            Job j{0, 0, t0, std::min<uint64_t>(static_cast<uint64_t>(Tg), t0 + piece)};
+            j.words = 1;
+            jobs.push_back(j);
+        }
+    }
     std::vector<std::thread> copiers;
     for (int id = 0; id < kCopiers; ++id) copiers.emplace_back(copier_main, id);
     auto on_final = [&](uint64_t p0, uint64_t p1, uint64_t t0, uint64_t t1) {
@@ -937,7 +965,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                       tile_layout ? 2 : 0,
                                       ctx->tail_per_tile * kscale, H,
                                       on_final, words_in_layout ? nullptr : local.data(),
-                                      /*host_tok_row=*/!tile_layout);
+                                      /*host_tok_row=*/!tile_layout, /*device_scatter=*/dev_scatter);
     {
         std::lock_guard<std::mutex> lk(mu);
         jobs_done = true;
@@ -1074,6 +1102,42 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     CU(cudaMemsetAsync(S.rows, 0, H.rows32 * 32, ctx->stream));
     CU(cudaMemsetAsync(S.nwk, 0, (static_cast<size_t>(V) * K + K) * sizeof(int32_t), ctx->stream));
 
+    if (dev_scatter && Tg > 0) {
+        // doc_map = the stable sort of the tokens by (tile, word) (layout_gpu.cu)
+        const uint64_t n = static_cast<uint64_t>(Tg);
+        const int ndt = static_cast<int>(H.tile_doc.size()) - 1;
+        const uint64_t maxkey = static_cast<uint64_t>(ndt + 1) * static_cast<uint64_t>(V);
+        if (maxkey > 0xFFFFFFFFull) return fail(ctx, LDA_ERANGE, "too many document tiles for 32-bit layout keys");
+        int bits = 1;
+        while (bits < 32 && (uint64_t(1) << bits) < maxkey) ++bits;
+        const size_t tw = lda::radix_sort_temp_words(n);
+        const size_t words_total = 4 * n + tw + H.tile_doc.size() + (static_cast<size_t>(V) + 3) / 4 + 64;
+        uint32_t *tmp = nullptr;
+        cudaError_t ce = cudaMalloc(&tmp, sizeof(uint32_t) * words_total);
+        if (ce != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ctx, ce == cudaErrorMemoryAllocation ? LDA_ENOMEM : LDA_ECUDA,
+                        std::string("layout sort scratch: ") + cudaGetErrorString(ce));
+        }
+        uint32_t *keys = tmp, *vals = tmp + n, *ktmp = tmp + 2 * n, *vtmp = tmp + 3 * n, *rtmp = tmp + 4 * n;
+        uint32_t *d_tile_doc = rtmp + tw;
+        uint8_t *d_tail = reinterpret_cast<uint8_t *>(d_tile_doc + H.tile_doc.size());
+        bool in_tmp = false;
+        int r = 0;
+        ce = h2d(d_tile_doc, H.tile_doc.data(), sizeof(uint32_t) * H.tile_doc.size());
+        if (ce == cudaSuccess) ce = h2d(d_tail, H.tail.data(), H.tail.size());
+        if (ce == cudaSuccess)
+            r = lda::launch_layout_keys(S.doc_ptr32, reinterpret_cast<const int32_t *>(S.tok_row), d_tail, d_tile_doc,
+                                        ndt, V, Dg, keys, vals, S.num_sms, ctx->stream);
+        if (ce == cudaSuccess && r == 0)
+            r = lda::radix_sort_pairs(keys, vals, ktmp, vtmp, n, bits, rtmp, ctx->stream, &in_tmp);
+        if (ce == cudaSuccess && r == 0) r = lda::launch_invert(in_tmp ? vtmp : vals, S.doc_map, n, S.num_sms, ctx->stream);
+        if (ce == cudaSuccess && r != 0) ce = static_cast<cudaError_t>(r);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(ctx->stream);
+        cudaFree(tmp);
+        if (ce != cudaSuccess) return fail(ctx, LDA_ECUDA, std::string("device layout: ") + cudaGetErrorString(ce));
+        lda::tmark("device layout (keys, radix sort, doc_map)");
+    }
     if (tile_layout) KL(lda::launch_tok_row(S, ctx->stream));
     // a1: random init (t = 0), then the count rebuild.
     CU(cudaStreamSynchronize(ctx->stream));

@@ -147,7 +147,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &L,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final,
-                         const int64_t *word_counts, bool host_tok_row) {
+                         const int64_t *word_counts, bool host_tok_row, bool device_scatter) {
     const int64_t T = doc_ptr[D];
     L.D = D;
     L.T = T;
@@ -265,9 +265,17 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     // word-major stream, the costliest part of the host pass) are left to
     // the device unless asked for (launch_tok_row from doc_map)
     const bool want_row = !tile_layout || host_tok_row;
-    if ((want_row && !L.tok_row.allocate(T)) || !L.doc_map.allocate(T) ||
+    // device_scatter (tile layout): the per-token scatter -- doc_map -- is left
+    // to the device (layout_gpu.cu), which sorts the tokens by the key
+    // tile·V + word (tail words: ndt·V + word); the host keeps the counts
+    const bool dev_scatter = device_scatter && tile_layout && !want_row;
+    if ((want_row && !L.tok_row.allocate(T)) || (!dev_scatter && !L.doc_map.allocate(T)) ||
         (!tile_layout && !L.tok_crank.allocate(T)))
         return "host allocation of the token tables failed";
+    if (dev_scatter) {
+        L.tile_doc.assign(tile_doc.begin(), tile_doc.end());
+        L.tail.assign(tail.begin(), tail.end());
+    }
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
     if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";
     // first touch in parallel, one store per 4 KB page (the kernel zeroes
@@ -376,6 +384,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                     }
                 }
                 const int64_t d0 = tile_doc[b], d1 = tile_doc[b + 1];
+                if (dev_scatter) continue;
                 if (want_row) {
                     for (int64_t d = d0; d < d1; ++d) {
                         const uint32_t row = L.row_off32[d];
@@ -468,7 +477,7 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
         // similar length -> similar θ row lengths -> little SIMT divergence.
         // (The Philox counter does not depend on this order: each token
         // carries its canonical rank.)
-        run_parts([&](int t) {
+        if (!dev_scatter) run_parts([&](int t) {
             auto &next = pnext[t];
             if (tile_layout && !want_row) {
                 for (int64_t i = doc_ptr[tdoc[t]]; i < doc_ptr[tdoc[t + 1]]; ++i) L.doc_map[i] = next[words[i]]++;
@@ -502,10 +511,10 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                 }
             }
         });
-        if (on_final)
+        if (on_final && !dev_scatter)
             on_final(pos_tile, pos, static_cast<uint64_t>(doc_ptr[d0]), static_cast<uint64_t>(doc_ptr[d1]));
     }
-    if (on_final && tail_tokens > 0) on_final(static_cast<uint64_t>(T - tail_tokens), static_cast<uint64_t>(T), 0, 0);
+    if (on_final && !dev_scatter && tail_tokens > 0) on_final(static_cast<uint64_t>(T - tail_tokens), static_cast<uint64_t>(T), 0, 0);
     if (pos != static_cast<uint64_t>(T - tail_tokens)) return "internal: token layout does not cover the corpus";
     ctmp.release();
     tmark("layout: tiles (count, ranks, scatter)");

@@ -1797,6 +1797,7 @@ int launch_peer_all_gather(void *const *ptrs, int world, int rank, void *own, si
 // ---------------------------------------------------------------------------
 int configure_kernels(DevState &s) {
     cudaError_t e;
+    const void *sampler0_fn = nullptr;
     int dev = 0;
     if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
     if ((e = cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
@@ -1821,13 +1822,8 @@ int configure_kernels(DevState &s) {
         else
             fn = smemp ? reinterpret_cast<const void *>(&sweep_kernel<false, true>)
                        : reinterpret_cast<const void *>(&sweep_kernel<false, false>);
-        if ((e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      static_cast<int>(s.sweep_smem))) != cudaSuccess)
-            return e;
-        int bps = 1;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, fn, kSweepThreads, s.sweep_smem)) != cudaSuccess)
-            return e;
-        s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
+        sampler0_fn = fn;  // its attributes are set below only if sampler 0 runs (each first touch of a
+                           // kernel loads it: ~ms per kernel on the load path)
     }
     // tile sampler (default): per CTA the n_k histogram, per warp the word
     // table and the batch scratch; <= 8 warps per CTA
@@ -1882,14 +1878,16 @@ int configure_kernels(DevState &s) {
             s.sweep_fused = s.tile_fused;
         }
         s.wt_bytes = s.sweep_tile_cta && s.tile_cta_gnk ? tab_bytes_compact(s.K) : tab_bytes(s.K);
-        if (s.sweep_tile || s.sweep_tile_cta)
-            for (const void *f : {reinterpret_cast<const void *>(&word_table_kernel<true, false>),
-                                  reinterpret_cast<const void *>(&word_table_kernel<false, false>),
-                                  reinterpret_cast<const void *>(&word_table_kernel<true, true>),
-                                  reinterpret_cast<const void *>(&word_table_kernel<false, true>)})
-                if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) !=
-                    cudaSuccess)
-                    return e;
+        if (s.sweep_tile || s.sweep_tile_cta) {
+            // the variant launch_sweep will use
+            const bool compact = s.sweep_tile_cta && s.tile_cta_gnk, vec = (s.K & 3) == 0;
+            const void *f = compact ? (vec ? reinterpret_cast<const void *>(&word_table_kernel<true, true>)
+                                           : reinterpret_cast<const void *>(&word_table_kernel<false, true>))
+                                    : (vec ? reinterpret_cast<const void *>(&word_table_kernel<true, false>)
+                                           : reinterpret_cast<const void *>(&word_table_kernel<false, false>));
+            if ((e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * s.K)) != cudaSuccess)
+                return e;
+        }
         if (s.sweep_tile) {
             const void *fn = reinterpret_cast<const void *>(&sweep_tile_kernel<LDA_TRING>);
             s.tile_block = 32 * wpc;
@@ -1904,6 +1902,17 @@ int configure_kernels(DevState &s) {
             s.tile_grid = s.num_sms * (bps > 0 ? bps : 1);
             s.sweep_fused = s.tile_fused;
         }
+    }
+    if (!s.sweep_tile && !s.sweep_tile_cta) {
+        // sampler 0 runs
+        if ((e = cudaFuncSetAttribute(sampler0_fn, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      static_cast<int>(s.sweep_smem))) != cudaSuccess)
+            return e;
+        int bps = 1;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, sampler0_fn, kSweepThreads, s.sweep_smem)) !=
+            cudaSuccess)
+            return e;
+        s.sweep_grid = s.num_sms * (bps > 0 ? bps : 1);
     }
     // recount: two K-length histograms per CTA in shared memory, or (wide K)
     // in a global scratch slice per CTA

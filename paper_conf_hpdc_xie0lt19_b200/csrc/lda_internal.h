@@ -102,6 +102,9 @@ struct HostLayout {
     std::vector<int32_t> zero_words;   // words split over sampler chunks or without tokens
     std::vector<int64_t> word_count;   // V local tokens per word
     std::vector<TileItem> titems;      // tile sampler items: tile-major, heavy-first inside a tile
+    // device_scatter only: the document tiles and the tail words (the sort key of layout_gpu.cu)
+    std::vector<uint32_t> tile_doc;    // ndt+1 document boundaries of the document tiles
+    std::vector<uint8_t> tail;         // V: 1 = the word's tokens form one run in the tail tile
 };
 
 // cbase[w] = canonical index of this rank's first token of word w.
@@ -119,7 +122,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int sampler, int64_t tail_per_tile, HostLayout &out,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final = {},
                          const int64_t *word_counts = nullptr,  // V local tokens per word, if known
-                         bool host_tok_row = true);  // tile layout: false = tok_row left to the device (launch_tok_row)
+                         bool host_tok_row = true,   // tile layout: false = tok_row left to the device (launch_tok_row)
+                         bool device_scatter = false);  // tile layout: doc_map left to the device (layout_gpu.cu)
 
 // Host-side validation of a local corpus; "" if valid.  *too_long set when a
 // doc exceeds 65535 tokens.
@@ -216,6 +220,19 @@ int launch_scatter_z(const DevState &s, const uint16_t *zd, void *stream);
 int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, void *table_done_event,
                  int parts = 3);
 int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches);
+
+// layout_gpu.cu: the doc-word map of the tile layout built on the device.
+// keys[i] = (tail[w] ? ndt : tile(d(i)))·V + w, vals[i] = i for every token i
+int launch_layout_keys(const uint32_t *doc_ptr32, const int32_t *words, const uint8_t *tail, const uint32_t *tile_doc,
+                       int ndt, int32_t V, int64_t D, uint32_t *keys, uint32_t *vals, int num_sms, void *stream);
+// stable LSD radix sort of (keys, vals) by the low `bits` key bits (8 per
+// pass); the result is in (keys_tmp, vals_tmp) when *result_in_tmp, else in
+// (keys, vals); temp: radix_sort_temp_words(n) words
+size_t radix_sort_temp_words(uint64_t n);
+int radix_sort_pairs(uint32_t *keys, uint32_t *vals, uint32_t *keys_tmp, uint32_t *vals_tmp, uint64_t n, int bits,
+                     uint32_t *temp, void *stream, bool *result_in_tmp);
+// doc_map[vals[p]] = p
+int launch_invert(const uint32_t *vals, uint32_t *doc_map, uint64_t n, int num_sms, void *stream);
 
 // ---------------------------------------------------------------------------
 // The exchange of Eq. 4 (L935-937), comm.cpp.  All calls return an lda_status

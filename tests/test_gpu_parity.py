@@ -326,3 +326,19 @@ def test_invalid_word_ids_rejected_on_device(tile_tokens):
         assert e.value.code == L.LDA_EINVAL, e.value
     g = U.gpu_model(400, 300, 16, 0.5, 0.01, doc_ptr, words, 1, tile_tokens=tile_tokens)
     U.check_invariants_gpu(g, doc_ptr, words)
+
+
+@pytest.mark.parametrize("n,bits", [(1, 1), (4095, 7), (4097, 23), (300_000, 17), (1_000_003, 23), (70_000, 32)])
+def test_device_radix_sort_stable(n, bits):
+    """The device radix sort the load uses for the doc-word map: equal to a
+    stable sort (numpy mergesort) on the low `bits` key bits, values carried."""
+    import paper_conf_hpdc_xie0lt19_b200 as L
+    rng = np.random.default_rng(n + bits)
+    # Zipf-like keys: long runs of equal keys test the stability
+    keys = (rng.zipf(1.3, n) % (1 << min(bits, 31))).astype(np.uint32)
+    if bits == 32:
+        keys = rng.integers(0, 1 << 32, n, dtype=np.uint64).astype(np.uint32)
+    vals = np.arange(n, dtype=np.uint32)
+    ok, ov = L.lda_debug_radix_sort(keys, vals, bits)
+    order = np.argsort(keys, kind="stable")
+    assert np.array_equal(ok, keys[order]) and np.array_equal(ov, vals[order])
