@@ -93,6 +93,8 @@ typedef struct lda_stats {
                                14·T_g + 4·Σ_t nnz_d(t) + 4·V·K */
     int64_t n_stream_chunks;/* M: chunks streamed per sweep (option stream_chunks;
                                1 = the corpus stays resident, WorkSchedule1) */
+    int64_t n_sparse_words; /* sampler 3 (K > 4096): words whose tables are
+                               built from sparse rows (option "sparse_words") */
 } lda_stats;
 
 /* Create a context.  D = global number of documents, V = vocabulary size,
@@ -157,6 +159,19 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   stay resident.  Needs sampler 2 or 3 (exclude_self = 0).
  *                   Same draws as M = 1.  With M > 1 ms_sample holds the
  *                   whole chunk loop (recount and θ inside it).
+ *   "sparse_words"  sampler 3 at K > 4096 with K % 4 == 0 (f2; SparseLDA's
+ *                   split p*(k) = β/(n_k+Vβ) + n_wk/(n_k+Vβ), ref [32], L999):
+ *                   words with at most this many tokens in the corpus get no
+ *                   O(K) p* row in their table; the table kernel writes their
+ *                   nonzero topics instead and the sampler rebuilds the row in
+ *                   shared memory from the smoothing row β/(n_k+Vβ), shared by
+ *                   all words, patched at those topics.  -1: K/4; 0
+ *                   (default): off -- measured slower on B200 at NYTimes
+ *                   shape, K = 8192 (19.90 vs 19.45 ms per sweep: the table
+ *                   kernel is latency-bound, not write-bound, and the bulk
+ *                   copy of a dense row costs the sampler's warps nothing
+ *                   while the patching does).  Same draws (the tables are
+ *                   bit-identical).
  *   "comm_pipeline" world > 1 with the recount kernel (fused_recount = 0):
  *                   recount n_wk in this many word ranges (default 4) and
  *                   start the exchange (Eq. 4) of each range's rows as soon

@@ -50,7 +50,7 @@ class lda_stats(ctypes.Structure):
                 ("ms_table", ctypes.c_double), ("ms_allreduce_exposed", ctypes.c_double),
                 ("tile_tokens", ctypes.c_int64), ("n_tiles", ctypes.c_int32), ("sampler", ctypes.c_int32),
                 ("bytes_alg", ctypes.c_double), ("bytes_sample", ctypes.c_double),
-                ("n_stream_chunks", ctypes.c_int64)]
+                ("n_stream_chunks", ctypes.c_int64), ("n_sparse_words", ctypes.c_int64)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}

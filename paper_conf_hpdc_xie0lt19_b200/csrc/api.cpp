@@ -57,6 +57,7 @@ struct lda_ctx {
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int64_t comm_pipeline = 4;  // world > 1: word ranges whose rows are exchanged as soon as recounted (f1)
+    int64_t sparse_words = 0;  // f2: words with <= this many tokens get sparse rows (-1: K/4; 0 off: measured slower)
     int threads = 0;
     // distribution: the exchange of Eq. 4 (NCCL or the in-process peer group)
     int32_t rank = 0, world = 1;
@@ -94,6 +95,7 @@ struct lda_ctx {
     int64_t loglik_every = 0;
     std::vector<int64_t> ll_sweep;
     std::vector<double> ll_value, ll_pending;
+    std::vector<int64_t> gcount;  // V: global tokens per word (load)
 };
 
 // Handle of an in-process peer group (shared by its ranks' contexts).
@@ -165,6 +167,42 @@ int dalloc(lda_ctx *ctx, T **p, size_t n) {
         int r_ = dalloc(ctx, &(ptr), (n));       \
         if (r_ != LDA_OK) return r_;             \
     } while (0)
+
+// f2: sparse word rows for the large-K sampler's compact tables (kernels.cu
+// SparseRows): a word with at most `sparse_words` tokens in the whole corpus
+// (so at most that many nonzero n_wk) gets min(count, K) entries.
+int setup_sparse_rows(lda_ctx *ctx) {
+    lda::DevState &S = ctx->S;
+    const int32_t V = ctx->V, K = ctx->K;
+    const int64_t thr = ctx->sparse_words < 0 ? K / 4 : ctx->sparse_words;
+    S.sp_words = 0;
+    S.sp_cap = 0;
+    if (!(S.sweep_tile_cta && S.tile_cta_gnk) || (K & 3) || thr <= 0 ||
+        ctx->gcount.size() != static_cast<size_t>(V))
+        return LDA_OK;
+    std::vector<uint32_t> off(static_cast<size_t>(V) + 1);
+    uint64_t tot = 0;
+    int64_t nsp = 0;
+    for (int32_t w = 0; w < V; ++w) {
+        off[w] = static_cast<uint32_t>(tot);
+        const int64_t c = ctx->gcount[w];
+        if (c > 0 && c <= thr) {
+            tot += static_cast<uint64_t>(std::min<int64_t>(c, K));
+            ++nsp;
+        }
+        if (tot >= 0xFFFFFFF0ull) return LDA_OK;  // beyond 32-bit offsets: dense tables only
+    }
+    off[V] = static_cast<uint32_t>(tot);
+    if (nsp == 0) return LDA_OK;
+    DA(S.sp_off, static_cast<size_t>(V) + 1);
+    DA(S.sp_nnz, static_cast<size_t>(V));
+    DA(S.sp_ent, 2 * static_cast<size_t>(tot));
+    DA(S.s32, static_cast<size_t>((K + 3) & ~3));
+    CU(cudaMemcpy(S.sp_off, off.data(), sizeof(uint32_t) * off.size(), cudaMemcpyHostToDevice));
+    S.sp_words = nsp;
+    S.sp_cap = static_cast<int64_t>(tot);
+    return LDA_OK;
+}
 
 int ensure_events(lda_ctx *ctx, size_t n) {
     while (ctx->ev.size() < n) {
@@ -392,6 +430,10 @@ int load_chunked(lda_ctx *ctx, const int64_t *doc_ptr, const int32_t *words, int
     S.seed = seed;
     S.ntiles = 0;
     for (auto &c : ctx->chunks) S.ntiles += c->H.ntiles;
+    {
+        const int rs = setup_sparse_rows(ctx);
+        if (rs != LDA_OK) return rs;
+    }
     int launches = 0;
     int r = chunked_rebuild(ctx, true, &launches);
     if (r != LDA_OK) return r;
@@ -408,6 +450,7 @@ int load_chunked(lda_ctx *ctx, const int64_t *doc_ptr, const int32_t *words, int
     ctx->stats.n_tiles = S.ntiles;
     ctx->stats.sampler = S.sweep_tile ? 2 : 3;
     ctx->stats.n_stream_chunks = M;
+    ctx->stats.n_sparse_words = S.sp_words;
     ctx->stats.sum_nnz_doc = ctx->cur_nnz;
     return LDA_OK;
 }
@@ -578,6 +621,9 @@ int lda_set_option(lda_ctx *ctx, const char *key, int64_t value) {
     } else if (k == "comm_pipeline") {
         if (value < 1 || value > 64) return fail(ctx, LDA_EINVAL, "comm_pipeline must be in [1, 64]");
         ctx->comm_pipeline = value;
+    } else if (k == "sparse_words") {
+        if (value < -1) return fail(ctx, LDA_EINVAL, "sparse_words must be -1 (auto), 0 (off) or > 0");
+        ctx->sparse_words = value;
     } else if (k == "loglik_every") {
         if (value < 0 || value > (int64_t(1) << 31)) return fail(ctx, LDA_EINVAL, "loglik_every must be >= 0");
         ctx->loglik_every = value;
@@ -756,6 +802,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         int64_t run = 0;
         lda_canonical_bases(V, ctx->world, ctx->rank, all.data(), cbase.data(), &run);
         ctx->T_global = run;
+        ctx->gcount.assign(V, 0);
+        for (int32_t g = 0; g < ctx->world; ++g)
+            for (int32_t w = 0; w < V; ++w) ctx->gcount[w] += all[static_cast<size_t>(g) * V + w];
     }
 
     lda::HostLayout &H = ctx->H;
@@ -991,6 +1040,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         int64_t run = 0;
         lda_canonical_bases(V, 1, 0, H.word_count.data(), cbase.data(), &run);
         ctx->T_global = run;
+        ctx->gcount = H.word_count;
     }
     if (copy_err != cudaSuccess) {
         cudaGetLastError();
@@ -1139,6 +1189,10 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         lda::tmark("device layout (keys, radix sort, doc_map)");
     }
     if (tile_layout) KL(lda::launch_tok_row(S, ctx->stream));
+    {
+        const int rs = setup_sparse_rows(ctx);
+        if (rs != LDA_OK) return rs;
+    }
     // a1: random init (t = 0), then the count rebuild.
     CU(cudaStreamSynchronize(ctx->stream));
     lda::tmark("H2D copies");
@@ -1164,6 +1218,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     ctx->stats.tile_tokens = ctx->tile_tokens_used;
     ctx->stats.n_tiles = S.ntiles;
     ctx->stats.sampler = S.sweep_tile ? 2 : (S.sweep_tile_cta ? 3 : 0);
+    ctx->stats.n_sparse_words = S.sp_words;
     ctx->stats.n_stream_chunks = 1;
     ctx->stats.sum_nnz_doc = ctx->cur_nnz;
     return LDA_OK;

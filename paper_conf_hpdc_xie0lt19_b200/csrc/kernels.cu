@@ -486,6 +486,46 @@ __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restric
     return fmaf(count_f32(e), tab32(p32, e), acc);
 }
 
+// Packed fp32 pairs (Blackwell FFMA2 / FADD2 / FMUL2: two IEEE fp32
+// operations per instruction, each rounded as its scalar form -- the two
+// FFMA chains of a block sum below stay bit-identical).
+typedef unsigned long long f32x2;
+__device__ __forceinline__ f32x2 f2_pack(float a, float b) {
+    f32x2 r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ f32x2 f2_add(f32x2 a, f32x2 b) {
+    f32x2 r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ f32x2 f2_mul(f32x2 a, f32x2 b) {
+    f32x2 r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ f32x2 f2_fma(f32x2 a, f32x2 b, f32x2 c) {
+    f32x2 r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
+__device__ __forceinline__ float f2_hsum(f32x2 a) {
+    float x, y;
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(x), "=f"(y) : "l"(a));
+    return x + y;
+}
+// the counts of entries e0, e1 as an fp32 pair: (2^23 + c) - 2^23, exact
+__device__ __forceinline__ f32x2 count_f32x2(uint32_t e0, uint32_t e1) {
+    return f2_add(f2_pack(__uint_as_float(__byte_perm(e0, 0x4B00u, 0x5410)),
+                          __uint_as_float(__byte_perm(e1, 0x4B00u, 0x5410))),
+                  f2_pack(-8388608.0f, -8388608.0f));
+}
+// the masses c·p32(t) of entries e0, e1, added to the pair acc
+__device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const float *__restrict__ p32, f32x2 acc) {
+    return f2_fma(count_f32x2(e0, e1), f2_pack(tab32(p32, e0), tab32(p32, e1)), acc);
+}
+
 // ---------------------------------------------------------------------------
 // a3 + a4, tile sampler (sampler 2, the default).
 //
@@ -518,6 +558,9 @@ __device__ __forceinline__ float entry_mass32(uint32_t e, const float *__restric
 // ---------------------------------------------------------------------------
 #ifndef LDA_TRING
 #define LDA_TRING 3
+#endif
+#ifndef LDA_F32X2
+#define LDA_F32X2 1  // the walk's block sums with packed fp32 pairs (FFMA2)
 #endif
 #ifndef LDA_TILE_WPC
 #define LDA_TILE_WPC 8
@@ -570,6 +613,11 @@ struct TileArgs {
     uint32_t wt_bytes;
     int nbuf;                  // sweep_tile_cta_kernel: table buffers per CTA
     int recount;               // 1: the ϕ update fused here; 0: recount_kernel after the sweep
+    // f2 sparse word rows (sweep_tile_cta_kernel, compact tables): see SparseRows
+    const uint32_t *sp_off;    // V+1, null = off
+    const uint32_t *sp_nnz;
+    const uint32_t *sp_ent;
+    const float *s32;
     uint32_t t;
     uint32_t key0[10], key1[10];
 };
@@ -694,14 +742,30 @@ __host__ __device__ constexpr size_t tab_bytes_compact(int K) {
     return static_cast<size_t>(tab_g2(K)) * 8 + static_cast<size_t>(4) * ((K + 3) & ~3);
 }
 
+// f2 (SparseLDA's split of p* = β·inv(k) + n_wk·inv(k), ref [32], L999):
+// sparse word rows.  A word with sp_off[w+1] > sp_off[w] ("rare": few tokens
+// against K) gets no p32 row in its table -- only Pg -- but the list of its
+// nonzero topics (topic, p32(topic)) in sp_ent[2·sp_off[w] ..], ascending,
+// count in sp_nnz[w]; the sampler rebuilds its p32 row in shared memory from
+// the smoothing row s32[k] = fl32(β·inv(k)) (shared by all words, written
+// here by block 0) plus those entries -- bit-identical to the dense row.
+struct SparseRows {
+    const uint32_t *off;  // V+1 (null: off)
+    uint32_t *nnz;        // V
+    uint32_t *ent;        // 2 words per entry: topic, p32 bits
+    float *s32;           // K4: fl32(β·inv(k)), zero padding
+};
+
 template <bool VEC, bool COMPACT>
 __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double *__restrict__ denom, int V, int K,
-                                  double alpha, double beta, char *__restrict__ tab) {
+                                  double alpha, double beta, char *__restrict__ tab, SparseRows sp) {
     extern __shared__ double inv64[];
     const int lane = threadIdx.x & 31;
     for (int k = threadIdx.x; k < K; k += blockDim.x) inv64[k] = 1.0 / denom[k];
     __syncthreads();
     const int K4 = (K + 3) & ~3;
+    if (COMPACT && sp.off && blockIdx.x == 0)
+        for (int k = threadIdx.x; k < K4; k += blockDim.x) sp.s32[k] = k < K ? d2f_trunc((0.0 + beta) * inv64[k]) : 0.0f;
     const size_t wt = COMPACT ? tab_bytes_compact(K) : tab_bytes(K);
     const int nwarp = gridDim.x * (blockDim.x >> 5);
     for (int w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < V; w += nwarp) {
@@ -709,21 +773,55 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
         double *Pc = reinterpret_cast<double *>(tab + wt * w);
         float *p32 = reinterpret_cast<float *>(Pc + (COMPACT ? tab_g2(K) : tab_nc2(K)));
         float *L32 = p32 + K4;
+        // f2: a sparse word's nonzero topics go to its list instead of a p32 row
+        uint32_t *ent = nullptr;
+        uint32_t nz = 0;
+        if (COMPACT && sp.off) {
+            const uint32_t o0 = __ldg(sp.off + w), o1 = __ldg(sp.off + w + 1);
+            if (o1 > o0) ent = sp.ent + 2 * static_cast<size_t>(o0);
+        }
         double carry = 0.0;
-        for (int k0 = 0, c = 0; k0 < K; k0 += 128, ++c) {
+        // one 128-topic chunk (lane l: topics k0 + 4l .. 4l+3; VEC: their counts n)
+        auto chunk = [&](const int k0, const int c, const int4 n) {
             const int k = k0 + 4 * lane;
             double a4[4] = {0.0, 0.0, 0.0, 0.0};
             if (VEC) {
-                if (k < K) {
-                    const int4 n = __ldg(reinterpret_cast<const int4 *>(nwk_row + k));
-                    const double p0 = (i2d_pos(n.x) + beta) * inv64[k], p1 = (i2d_pos(n.y) + beta) * inv64[k + 1];
-                    const double p2 = (i2d_pos(n.z) + beta) * inv64[k + 2], p3 = (i2d_pos(n.w) + beta) * inv64[k + 3];
-                    *reinterpret_cast<float4 *>(p32 + k) =
-                        make_float4(d2f_trunc(p0), d2f_trunc(p1), d2f_trunc(p2), d2f_trunc(p3));
-                    a4[0] = alpha * p0;
-                    a4[1] = alpha * p1;
-                    a4[2] = alpha * p2;
-                    a4[3] = alpha * p3;
+                if (k < K || (COMPACT && ent)) {
+                    float f4[4] = {0.0f, 0.0f, 0.0f, 0.0f};
+                    if (k < K) {
+                        const double p0 = (i2d_pos(n.x) + beta) * inv64[k], p1 = (i2d_pos(n.y) + beta) * inv64[k + 1];
+                        const double p2 = (i2d_pos(n.z) + beta) * inv64[k + 2],
+                                     p3 = (i2d_pos(n.w) + beta) * inv64[k + 3];
+                        f4[0] = d2f_trunc(p0);
+                        f4[1] = d2f_trunc(p1);
+                        f4[2] = d2f_trunc(p2);
+                        f4[3] = d2f_trunc(p3);
+                        if (!(COMPACT && ent)) *reinterpret_cast<float4 *>(p32 + k) = make_float4(f4[0], f4[1], f4[2], f4[3]);
+                        a4[0] = alpha * p0;
+                        a4[1] = alpha * p1;
+                        a4[2] = alpha * p2;
+                        a4[3] = alpha * p3;
+                    }
+                    if (COMPACT && ent) {
+                        // the nonzero topics of this 128-topic chunk, in topic order
+                        const int cnt = (n.x != 0) + (n.y != 0) + (n.z != 0) + (n.w != 0);
+                        int incl = cnt;
+#pragma unroll
+                        for (int o = 1; o < 32; o <<= 1) {
+                            const int y = __shfl_up_sync(kFull, incl, o);
+                            if (lane >= o) incl += y;
+                        }
+                        uint32_t j = nz + static_cast<uint32_t>(incl - cnt);
+                        const int nn[4] = {n.x, n.y, n.z, n.w};
+#pragma unroll
+                        for (int e = 0; e < 4; ++e)
+                            if (nn[e] != 0) {
+                                ent[2 * j] = static_cast<uint32_t>(k + e);
+                                ent[2 * j + 1] = __float_as_uint(f4[e]);
+                                ++j;
+                            }
+                        nz += static_cast<uint32_t>(__shfl_sync(kFull, incl, 31));
+                    }
                 }
             } else {
 #pragma unroll
@@ -760,6 +858,23 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
                 if (lane == 0) Pc[c] = carry;
             }
             carry += __shfl_sync(kFull, incl, 31);
+        };
+        if (VEC) {
+            // the counts of 4 chunks in flight at a time (the chunks' fp64
+            // scans are a serial chain: without this the loads wait in it)
+            for (int k00 = 0; k00 < K; k00 += 512) {
+                int4 nn[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const int k = k00 + 128 * u + 4 * lane;
+                    nn[u] = k < K ? __ldg(reinterpret_cast<const int4 *>(nwk_row + k)) : make_int4(0, 0, 0, 0);
+                }
+#pragma unroll
+                for (int u = 0; u < 4; ++u)
+                    if (k00 + 128 * u < K) chunk(k00 + 128 * u, k00 / 128 + u, nn[u]);
+            }
+        } else {
+            for (int k0 = 0, c = 0; k0 < K; k0 += 128, ++c) chunk(k0, c, make_int4(0, 0, 0, 0));
         }
         // zero the padding so that the table bytes are deterministic
         if (COMPACT) {
@@ -771,7 +886,11 @@ __global__ void word_table_kernel(const int32_t *__restrict__ nwk, const double 
             if (lane == 1 && tab_nc2(K) > (K + 127) / 128 + 1) Pc[tab_nc2(K) - 1] = 0.0;
             for (int k = K + lane; k < 128 * ((K + 127) / 128); k += 32) L32[l32_idx(k)] = 0.0f;
         }
-        for (int k = K + lane; k < K4; k += 32) p32[k] = 0.0f;
+        if (COMPACT && ent) {
+            if (lane == 0) sp.nnz[w] = nz;
+        } else {
+            for (int k = K + lane; k < K4; k += 32) p32[k] = 0.0f;
+        }
     }
 }
 
@@ -896,6 +1015,15 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
 #pragma unroll
         for (int s2 = 0; s2 < R; ++s2) {
             const uint32_t w0 = hdr[s2] ? 0u : ring[s2].w[0];  // header word
+#if LDA_F32X2
+            // the two chains (even / odd entries) as one packed pair
+            f32x2 sp = f2_mul(count_f32x2(w0, ring[s2].w[1]),
+                              f2_pack(tab32(p32, w0), tab32(p32, ring[s2].w[1])));
+            sp = mass_f32x2(ring[s2].w[2], ring[s2].w[3], p32, sp);
+            sp = mass_f32x2(ring[s2].w[4], ring[s2].w[5], p32, sp);
+            sp = mass_f32x2(ring[s2].w[6], ring[s2].w[7], p32, sp);
+            bs[s2] = f2_hsum(sp);
+#else
             float s0 = count_f32(w0) * tab32(p32, w0);
             float s1 = count_f32(ring[s2].w[1]) * tab32(p32, ring[s2].w[1]);
             s0 = entry_mass32(ring[s2].w[2], p32, s0);
@@ -905,6 +1033,7 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
             s0 = entry_mass32(ring[s2].w[6], p32, s0);
             s1 = entry_mass32(ring[s2].w[7], p32, s1);
             bs[s2] = s0 + s1;
+#endif
         }
 #pragma unroll
         for (int s2 = 0; s2 < R; ++s2) {
@@ -1300,7 +1429,7 @@ __host__ __device__ constexpr size_t tile_cta_warp_bytes(int lmax) {
 __host__ __device__ constexpr size_t tile_cta_bytes(int K, int lmax, int nwarps, bool gnk, int nb) {
     return (gnk ? 0 : static_cast<size_t>(4) * ((K + 3) & ~3)) +
            static_cast<size_t>(nb) * (gnk ? tab_bytes_compact(K) : tab_bytes(K)) +
-           nwarps * tile_cta_warp_bytes(lmax) + 128;
+           nwarps * tile_cta_warp_bytes(lmax) + 256;
 }
 
 __device__ __forceinline__ void mbar_arrive(uint64_t *bar) {
@@ -1330,7 +1459,11 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     TileItem *items = reinterpret_cast<TileItem *>(ctrl + 32);  // [4]
     uint32_t *slot = reinterpret_cast<uint32_t *>(ctrl + 96);   // [4]
     uint32_t *left = slot + 4;                                  // [4]
+    int *bsw = reinterpret_cast<int *>(ctrl + 128);             // [4] f2: the sparse word whose p32 row the
+                                                                //     buffer holds (-1: a dense table / none)
     const double gS = 9.5 * 5.9604644775390625e-08 * a.slack;
+    const int K4c = (K + 3) & ~3;
+    const uint32_t pg_bytes = static_cast<uint32_t>(8 * tab_g2(K));
 
     // buffer b <- the CTA's next work item (its table by bulk copy); the end
     // of the queue is an item with n = 0.  items[b] / slot[b] / left[b] are
@@ -1339,26 +1472,82 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
     // compute-sanitizer's racecheck does not model mbarrier ordering and
     // reports this handoff as a hazard (memcheck is clean).  The loader runs
     // only after every warp has left the buffer (left[b] reached 0).
+    // Run by a whole warp.  A sparse word (f2) is built in place by the warp:
+    // its Pg copied, the p32 row = the smoothing row s32 (copied in full when
+    // the buffer held a dense table, else restored at the previous sparse
+    // word's topics) patched at the word's nonzero topics; plain smem stores,
+    // published by the warp's arrive.  Dense tables: one bulk copy.
     auto load = [&](int b) {
-        const uint32_t ci = atomicAdd(a.counter, 1u);
+        uint32_t ci = 0;
+        if (lane == 0) ci = atomicAdd(a.counter, 1u);
+        ci = __shfl_sync(kFull, ci, 0);
         TileItem it = {0u, 0u, 0u, 0u};
         if (ci < a.n_items) it = a.items[ci];
-        items[b] = it;
-        slot[b] = 0u;
-        left[b] = static_cast<uint32_t>(nwarps);
-        if (it.n) {
-            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-            mbar_arrive_expect_tx(bar + b, a.wt_bytes);
-            bulk_g2s(tabs + b * wt, a.wtab + static_cast<size_t>(it.word) * a.wt_bytes, a.wt_bytes, bar + b);
+        uint32_t o0 = 0, o1 = 0;
+        if (GNK && a.sp_off && it.n) {
+            o0 = __ldg(a.sp_off + it.word);
+            o1 = __ldg(a.sp_off + it.word + 1);
+        }
+        const int prev = bsw[b];
+        __syncwarp();
+        if (lane == 0) {
+            items[b] = it;
+            slot[b] = 0u;
+            left[b] = static_cast<uint32_t>(nwarps);
+            bsw[b] = o1 > o0 ? static_cast<int>(it.word) : -1;
+        }
+        if (o1 > o0) {
+            char *tb = tabs + b * wt;
+            float *p32s = reinterpret_cast<float *>(tb + pg_bytes);
+            if (prev < 0) {
+                for (int i = lane; i < K4c / 4; i += 32)
+                    reinterpret_cast<float4 *>(p32s)[i] = __ldg(reinterpret_cast<const float4 *>(a.s32) + i);
+            } else {
+                const uint32_t *pe = a.sp_ent + 2 * static_cast<size_t>(__ldg(a.sp_off + prev));
+                const uint32_t pn = __ldg(a.sp_nnz + prev);
+                for (uint32_t j = lane; j < pn; j += 32) {
+                    const uint32_t t = __ldg(pe + 2 * j);
+                    p32s[t] = __ldg(a.s32 + t);
+                }
+            }
+            const double2 *src = reinterpret_cast<const double2 *>(a.wtab + static_cast<size_t>(it.word) * a.wt_bytes);
+            for (uint32_t i = lane; i < pg_bytes / 16; i += 32) reinterpret_cast<double2 *>(tb)[i] = __ldg(src + i);
+            __syncwarp();
+            const uint2 *e2 = reinterpret_cast<const uint2 *>(a.sp_ent) + o0;
+            const uint32_t n = __ldg(a.sp_nnz + it.word);
+            for (uint32_t j = lane; j < n; j += 32) {
+                const uint2 e = __ldg(e2 + j);
+                p32s[e.x] = __uint_as_float(e.y);
+            }
+            __syncwarp();
+            __threadfence_block();
+            if (lane == 0) mbar_arrive(bar + b);
         } else {
-            mbar_arrive(bar + b);
+            // the buffer's previous contents were written by this warp's or
+            // other warps' generic stores (a sparse word) or read by them
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp();
+            if (lane == 0) {
+                if (it.n) {
+                    mbar_arrive_expect_tx(bar + b, a.wt_bytes);
+                    bulk_g2s(tabs + b * wt, a.wtab + static_cast<size_t>(it.word) * a.wt_bytes, a.wt_bytes, bar + b);
+                } else {
+                    mbar_arrive(bar + b);
+                }
+            }
         }
     };
     if (!GNK)
         for (int k = threadIdx.x; k < K; k += blockDim.x) nkh[k] = 0;
     if (threadIdx.x == 0) {
-        for (int b = 0; b < NB; ++b) mbar_init(bar + b, 1);
+        for (int b = 0; b < NB; ++b) {
+            mbar_init(bar + b, 1);
+            bsw[b] = -1;
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 0) {
+        __syncwarp();
         for (int b = 0; b < NB; ++b) load(b);
     }
     __syncthreads();
@@ -1413,7 +1602,7 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
         uint32_t was = 0;
         if (lane == 0) was = atomicSub(left + b, 1u);
         was = __shfl_sync(kFull, was, 0);
-        if (was == 1u && lane == 0) {
+        if (was == 1u) {
             __threadfence_block();
             load(b);
         }
@@ -2069,20 +2258,21 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
             return e;
         const int wtb = static_cast<int>(std::min<int64_t>((static_cast<int64_t>(s.V) + 7) / 8, 8 * s.num_sms));
         const bool compact = s.sweep_tile_cta && s.tile_cta_gnk;
+        SparseRows sp{compact ? s.sp_off : nullptr, s.sp_nnz, s.sp_ent, s.s32};
         if (!(parts & 1)) {
             // the tables of this sweep are built (out-of-HBM chunks after the first)
         } else if ((s.K & 3) == 0 && compact)
             word_table_kernel<true, true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
-                                                                     s.wtab);
+                                                                     s.wtab, sp);
         else if (compact)
             word_table_kernel<false, true><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
-                                                                      s.wtab);
+                                                                      s.wtab, sp);
         else if ((s.K & 3) == 0)
             word_table_kernel<true, false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
-                                                                      s.wtab);
+                                                                      s.wtab, sp);
         else
             word_table_kernel<false, false><<<wtb, 256, 8 * s.K, st>>>(s.nwk, s.denom, s.V, s.K, s.alpha, s.beta,
-                                                                       s.wtab);
+                                                                       s.wtab, sp);
         if (parts & 1) ++*launches;
         if (table_done_event && (e = cudaEventRecord(static_cast<cudaEvent_t>(table_done_event), st)) != cudaSuccess)
             return e;
@@ -2109,6 +2299,10 @@ int launch_sweep(const DevState &s, uint32_t t, void *stream, int *launches, voi
         ta.wt_bytes = static_cast<uint32_t>(s.wt_bytes);
         ta.nbuf = s.tile_nbuf;
         ta.recount = s.tile_fused ? 1 : 0;
+        ta.sp_off = sp.off;
+        ta.sp_nnz = s.sp_nnz;
+        ta.sp_ent = s.sp_ent;
+        ta.s32 = s.s32;
         ta.t = t;
         uint32_t k0 = static_cast<uint32_t>(s.seed), k1 = static_cast<uint32_t>(s.seed >> 32);
         for (int r = 0; r < 10; ++r) {

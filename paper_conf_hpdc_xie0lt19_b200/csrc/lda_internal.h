@@ -187,6 +187,13 @@ struct DevState {
     int tile_grid = 0, tile_block = 0, tile_lmax = 160;
     char *wtab = nullptr;           // tile sampler: per-word tables (p32, dense prefix), rebuilt every sweep
     size_t wt_bytes = 0;
+    // f2, sampler 3 with compact tables: sparse word rows (kernels.cu SparseRows)
+    uint32_t *sp_off = nullptr;     // V+1: word w's entries [sp_off[w], sp_off[w+1]) (empty: a dense table)
+    uint32_t *sp_nnz = nullptr;     // V: its nonzero topics this sweep
+    uint32_t *sp_ent = nullptr;     // 2 words per entry (topic, fp32 p* bits)
+    float *s32 = nullptr;           // K4: the smoothing row fl32(β / (n_k + Vβ))
+    int64_t sp_words = 0;           // words with sparse rows
+    int64_t sp_cap = 0;             // entries allocated
     double certify_slack = 1.0;     // test option: scales the tile sampler's certification bounds
     double *denom = nullptr;        // K: n_k + Vβ of the frozen counts
     // scratch

@@ -342,3 +342,39 @@ def test_device_radix_sort_stable(n, bits):
     ok, ov = L.lda_debug_radix_sort(keys, vals, bits)
     order = np.argsort(keys, kind="stable")
     assert np.array_equal(ok, keys[order]) and np.array_equal(ov, vals[order])
+
+
+@pytest.mark.parametrize("opts", [dict(), dict(tile_tokens=20_000), dict(fused_recount=1, tile_tokens=50_000)])
+def test_k8192_sparse_word_rows_bit_identical(opts):
+    """f2 (SparseLDA's split p* = β/(n_k+Vβ) + n_wk/(n_k+Vβ), ref [32], L999):
+    the large-K sampler rebuilds a rare word's p32 row in shared memory from
+    the shared smoothing row patched at the word's nonzero topics, instead of
+    copying an O(K) row the table kernel wrote.  The tables are bit-identical,
+    so the draws must be too -- for every threshold (none, the default K/4,
+    every word), over several sweeps (buffers switch between dense and sparse
+    words and are patched / restored) -- and the chain matches the oracle."""
+    cfg = synth.scaled(synth.CONFIGS["nytimes_k8192"], 0.003)
+    doc_ptr, words = synth.to_numpy(*synth.generate_config(cfg, "cpu"))[:2]
+    K = cfg.K
+    runs = {thr: U.gpu_model(cfg.D, cfg.V, K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed, sparse_words=thr,
+                             **opts) for thr in (0, -1, 1 << 40)}
+    assert runs[0].stats()["n_sparse_words"] == 0
+    nsp = runs[-1].stats()["n_sparse_words"]
+    wc = np.bincount(words, minlength=cfg.V)
+    assert nsp == int(((wc > 0) & (wc <= K // 4)).sum()) and nsp > 0
+    assert runs[1 << 40].stats()["n_sparse_words"] == int((wc > 0).sum())
+    o = U.oracle_for(cfg.D, cfg.V, K, cfg.alpha, cfg.beta, doc_ptr, words, cfg.seed)
+    for _ in range(3):
+        margins = o.iterate(1, margins=True)
+        for g in runs.values():
+            g.iterate(1)
+        z0 = runs[0].z()
+        for thr, g in runs.items():
+            assert np.array_equal(g.z(), z0), thr
+            assert np.array_equal(g.nwk(), runs[0].nwk()), thr
+        bad = np.nonzero(z0 != o.z)[0]
+        assert (margins[bad] < U.MARGIN_EXCUSE).all()
+        if len(bad):
+            for g in runs.values():
+                g.set_z(o.z)
+    U.check_counts_equal(runs[-1], o)

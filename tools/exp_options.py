@@ -58,7 +58,7 @@ def main():
         nnz = float(np.mean(log["sum_nnz_tok"])) / cfg.T
         bs = np.mean([C.bytes_sample(cfg.T, cfg.V, cfg.K, int(x)) for x in log["sum_nnz_tok"]])
         out = {"set": s, "Gtok_s": round(cfg.T / ms / 1e6, 3), "ms": round(ms, 3),
-               "sample": round(st["ms_sample"] / n, 3), "theta": round(st["ms_theta"] / n, 3),
+               "sample": round(st["ms_sample"] / n, 3), "table": round(st["ms_table"] / n, 3), "theta": round(st["ms_theta"] / n, 3),
                "recount": round(st["ms_recount"] / n, 3), "nnz": round(nnz, 2),
                "sample_GBs": round(bs / (st["ms_sample"] / n / 1e3) / 1e9, 1), "load_s": round(tl, 1),
                "n_exact_per_sweep": st["n_exact_redraws"] / n, "ll": round(m.loglik(), 5)}
