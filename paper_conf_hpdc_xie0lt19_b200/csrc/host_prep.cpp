@@ -147,7 +147,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
                          int64_t chunk_tokens, int64_t recount_tokens, int nthreads,
                          int sampler, int64_t tail_per_tile, HostLayout &L,
                          const std::function<void(uint64_t, uint64_t, uint64_t, uint64_t)> &on_final,
-                         const int64_t *word_counts, bool host_tok_row, bool device_scatter) {
+                         const int64_t *word_counts, bool host_tok_row, bool device_scatter,
+                         const std::function<void()> &on_keys) {
     const int64_t T = doc_ptr[D];
     L.D = D;
     L.T = T;
@@ -275,6 +276,8 @@ std::string build_layout(const int64_t *doc_ptr, const int32_t *words, int64_t D
     if (dev_scatter) {
         L.tile_doc.assign(tile_doc.begin(), tile_doc.end());
         L.tail.assign(tail.begin(), tail.end());
+        // the device sort can start now (doc_ptr32, tile_doc and tail are final)
+        if (on_keys) on_keys();
     }
     HostBuf<uint32_t> ctmp;  // canonical rank of token i (document order)
     if (!tile_layout && !ctmp.allocate(T)) return "host allocation of the token tables failed";

@@ -1,0 +1,12 @@
+# load path with the overlapped device layout: timing + the GPU suite
+OUT=gpurun_out; mkdir -p $OUT
+LDA_TIMING=1 python tools/load_only.py --config pubmed --reps 3 > $OUT/r02aa_load.log 2>&1
+grep -v "layout:" $OUT/r02aa_load.log | tail -30
+timeout 1500 python -m pytest tests -m gpu -q -x -p no:cacheprovider > $OUT/r02aa_pytest.log 2>&1; echo "pytest exit $?" >> $OUT/r02aa_pytest.log
+tail -3 $OUT/r02aa_pytest.log
+for i in 1 2; do
+timeout 900 python bench.py --steps 20 --warmup 3 --no-cpu-baseline > $OUT/r02aa_bench$i.json 2> $OUT/r02aa_bench$i.err
+python -c "
+import json
+d=json.loads(open('$OUT/r02aa_bench$i.json').read().strip().splitlines()[-1]); print(d['value']/1e9, d['roofline']['frac'], d['e2e']['value']/1e9, d['e2e']['breakdown'])"
+done
