@@ -867,7 +867,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     bool words_pinned = false;
     int64_t words_left = 0;  // words upload jobs not finished (device layout)
     bool alloc_done = false;
-    double copy_ms_total = 0.0, memcpy_ms_total = 0.0, alloc_ms = 0.0, last_copy_end = 0.0, layout_end = 0.0;
+    double copy_ms_total = 0.0, memcpy_ms_total = 0.0, alloc_ms = 0.0, alloc_arena_ms = 0.0, last_copy_end = 0.0,
+           layout_end = 0.0;
     // page-locked staging ring: the copiers memcpy a finished piece of a token
     // table into a slot (in parallel, from several threads) and DMA it from
     // there -- the driver's own pageable path serialises the copies at ~10 GB/s
@@ -898,8 +899,13 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                     off += (std::max<size_t>(pa.second, 1) + 511) & ~size_t(511);
                 }
             }
-            if (err == cudaSuccess && cudaHostAlloc(reinterpret_cast<void **>(&stage), kSlots * kSlotBytes,
-                                                    cudaHostAllocDefault) != cudaSuccess) {
+            // (no staging ring when every copy is a straight DMA: the device
+            // layout with page-locked words copies nothing else)
+            const bool need_stage = !(dev_scatter && words_pinned);
+            alloc_arena_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - c0).count();
+            if (err == cudaSuccess && need_stage &&
+                cudaHostAlloc(reinterpret_cast<void **>(&stage), kSlots * kSlotBytes, cudaHostAllocDefault) !=
+                    cudaSuccess) {
                 cudaGetLastError();
                 stage = nullptr;  // fall back to pageable copies
             }
@@ -981,6 +987,16 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                                                     std::chrono::steady_clock::now() - load_t0).count());
     };
     pre.push_back({reinterpret_cast<void **>(&S.rows), sizeof(uint32_t) * 8 * r32});
+    // the device layout's scratch (see sorter_main), in the same allocation:
+    // cudaMalloc / cudaFree on the sorter thread while the copiers and the
+    // host pass run measured 1-150 ms and 1-820 ms
+    uint32_t *sort_scratch = nullptr;
+    const bool vtmp_rows = 8 * r32 >= static_cast<uint64_t>(Tg);
+    const size_t sort_words = tile_layout && Tg > 0
+                                  ? (vtmp_rows ? 0 : static_cast<size_t>(Tg)) + lda::radix_sort_temp_words(Tg) +
+                                        2 * static_cast<size_t>(Dg + 1) + (static_cast<size_t>(V) + 3) / 4 + 64
+                                  : 0;
+    if (sort_words) pre.push_back({reinterpret_cast<void **>(&sort_scratch), sizeof(uint32_t) * sort_words});
     // the tile layout's doc-word map is built on the device (layout_gpu.cu):
     // the copiers upload the words into S.tok_row (rebuilt from doc_map
     // afterwards) while the host computes the counts
@@ -1013,8 +1029,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             sort_start_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - load_t0).count();
         }
         cudaError_t ce = cudaSetDevice(ctx->device);
-        cudaStream_t ss = nullptr;
-        if (ce == cudaSuccess) ce = cudaStreamCreateWithFlags(&ss, cudaStreamNonBlocking);
+        cudaStream_t ss = ctx->comm_stream;  // idle during the load
         // doc_map = the stable sort of the tokens by (tile, word)
         const uint64_t n = static_cast<uint64_t>(Tg);
         const int ndt = static_cast<int>(H.tile_doc.size()) - 1;
@@ -1025,51 +1040,40 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         }
         int bits = 1;
         while (bits < 32 && (uint64_t(1) << bits) < maxkey) ++bits;
+        // The sort's four T-word buffers are the load's own: the keys over the
+        // words (S.tok_row), the keys' second buffer S.doc_map, the values in
+        // the z buffers (S.tok_z, S.z_doc: >= 4·T contiguous bytes of the
+        // arena) and the values' second buffer in the θ row storage when it
+        // holds >= T words (zeroed after the load; else in sort_scratch).  The
+        // final values land in the z buffers or the θ rows, never in doc_map,
+        // which the inversion then writes.
         const size_t tw = lda::radix_sort_temp_words(n);
-        const size_t words_total =
-            4 * n + tw + H.tile_doc.size() + (static_cast<size_t>(V) + 3) / 4 + 2 * (Dg + 1) + 64;
-        uint32_t *tmp = nullptr;
+        uint32_t *tmp = sort_scratch;
         auto now_ms = [&] {
             return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - load_t0).count();
         };
-        if (ce == cudaSuccess) ce = cudaMalloc(&tmp, sizeof(uint32_t) * words_total);
         sort_malloc_ms = now_ms();
-        if (ce != cudaSuccess) {
-            sort_err = ce;
-            sort_where = "layout sort scratch";
-            cudaGetLastError();
-            if (ss) cudaStreamDestroy(ss);
-            return;
-        }
-        // the keys overwrite the words in place (S.tok_row); rowof[i] = the θ
-        // row of token i's document, gathered into tok_row by the inversion
-        uint32_t *keys = S.tok_row, *vals = tmp, *ktmp = tmp + n, *vtmp = tmp + 2 * n, *rowof = tmp + 3 * n;
-        uint32_t *rtmp = tmp + 4 * n;
+        uint32_t *keys = S.tok_row, *ktmp = S.doc_map, *vals = reinterpret_cast<uint32_t *>(S.tok_z);
+        uint32_t *vtmp = vtmp_rows ? S.rows : tmp;
+        uint32_t *rtmp = tmp + (vtmp_rows ? 0 : n);
         uint32_t *d_tile_doc = rtmp + tw;
         uint32_t *d_doc_ptr = d_tile_doc + H.tile_doc.size();
-        uint32_t *d_row_off = d_doc_ptr + Dg + 1;
-        uint8_t *d_tail = reinterpret_cast<uint8_t *>(d_row_off + Dg + 1);
+        uint8_t *d_tail = reinterpret_cast<uint8_t *>(d_doc_ptr + Dg + 1);
         bool in_tmp = false;
         int r = 0;
         ce = cudaMemcpyAsync(d_tile_doc, H.tile_doc.data(), sizeof(uint32_t) * H.tile_doc.size(),
                              cudaMemcpyHostToDevice, ss);
         if (ce == cudaSuccess)
             ce = cudaMemcpyAsync(d_doc_ptr, H.doc_ptr32.data(), sizeof(uint32_t) * (Dg + 1), cudaMemcpyHostToDevice, ss);
-        if (ce == cudaSuccess && Dg > 0)
-            ce = cudaMemcpyAsync(d_row_off, H.row_off32.data(), sizeof(uint32_t) * Dg, cudaMemcpyHostToDevice, ss);
         if (ce == cudaSuccess) ce = cudaMemcpyAsync(d_tail, H.tail.data(), H.tail.size(), cudaMemcpyHostToDevice, ss);
         if (ce == cudaSuccess)
             r = lda::launch_layout_keys(d_doc_ptr, reinterpret_cast<const int32_t *>(S.tok_row), d_tail, d_tile_doc,
-                                        ndt, V, Dg, keys, vals, S.num_sms, ss, d_row_off, rowof);
+                                        ndt, V, Dg, keys, vals, S.num_sms, ss);
         if (ce == cudaSuccess && r == 0) r = lda::radix_sort_pairs(keys, vals, ktmp, vtmp, n, bits, rtmp, ss, &in_tmp);
-        // doc_map, and tok_row (the sorted keys are no longer needed)
-        if (ce == cudaSuccess && r == 0)
-            r = lda::launch_invert(in_tmp ? vtmp : vals, S.doc_map, n, S.num_sms, ss, rowof, S.tok_row);
+        if (ce == cudaSuccess && r == 0) r = lda::launch_invert(in_tmp ? vtmp : vals, S.doc_map, n, S.num_sms, ss);
         if (ce == cudaSuccess && r != 0) ce = static_cast<cudaError_t>(r);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(ss);
         sort_kernels_ms = now_ms();
-        cudaFree(tmp);
-        cudaStreamDestroy(ss);
         if (ce != cudaSuccess) {
             sort_err = ce;
             sort_where = "device layout";
@@ -1121,9 +1125,9 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     if (stage) cudaFreeHost(stage);
     if (std::getenv("LDA_TIMING"))
         std::fprintf(stderr,
-                     "[lda]   copiers: device allocation %.1f ms, H2D %.1f ms (of which host memcpy %.1f; summed "
-                     "over %d threads); layout end at %.1f ms, last copy end at %.1f ms (from the load start)\n",
-                     alloc_ms, copy_ms_total, memcpy_ms_total, kCopiers, layout_end, last_copy_end);
+                     "[lda]   copiers: device allocation %.1f ms (arena %.1f), H2D %.1f ms (of which host memcpy %.1f; "
+                     "summed over %d threads); layout end at %.1f ms, last copy end at %.1f ms (from the load start)\n",
+                     alloc_ms, alloc_arena_ms, copy_ms_total, memcpy_ms_total, kCopiers, layout_end, last_copy_end);
     ctx->allocs.insert(ctx->allocs.end(), pre_done.begin(), pre_done.end());
     // a layout error (invalid word id, or a range) takes precedence over an allocation error
     if (!e.empty()) {
@@ -1261,7 +1265,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
                          sort_start_ms, sort_malloc_ms, sort_kernels_ms, sort_end_ms);
         lda::tmark("device layout done");
     }
-    if (tile_layout && !(dev_scatter && Tg > 0)) KL(lda::launch_tok_row(S, ctx->stream));  // else: the sorter did
+    if (tile_layout) KL(lda::launch_tok_row(S, ctx->stream));
     {
         const int rs = setup_sparse_rows(ctx);
         if (rs != LDA_OK) return rs;

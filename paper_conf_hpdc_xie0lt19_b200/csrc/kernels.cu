@@ -1621,11 +1621,15 @@ __global__ void __launch_bounds__(512, 1) sweep_tile_cta_kernel(TileArgs a) {
 // ---------------------------------------------------------------------------
 // a0 on the device: the θ row of every token's document at its word-major
 // position (warp per document: coalesced doc_map reads, scattered stores).
+// One warp per document and no grid-stride loop: the blocks in flight are
+// consecutive documents, so the scattered stores stay inside one tile's part
+// of the word-major stream (L2).
 __global__ void tok_row_kernel(const uint32_t *__restrict__ doc_ptr32, const uint32_t *__restrict__ row_off32,
                                const uint32_t *__restrict__ doc_map, uint32_t *__restrict__ tok_row, int64_t D) {
     const int lane = threadIdx.x & 31;
-    const int64_t nw = static_cast<int64_t>(gridDim.x) * (blockDim.x >> 5);
-    for (int64_t d = static_cast<int64_t>(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); d < D; d += nw) {
+    {
+        const int64_t d = static_cast<int64_t>(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5);
+        if (d >= D) return;
         const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1], row = row_off32[d];
         for (uint32_t i = s + lane; i < e; i += 32) tok_row[doc_map[i]] = row;
     }
@@ -2181,8 +2185,8 @@ int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0, 
 
 int launch_tok_row(const DevState &s, void *stream) {
     if (s.D > 0)
-        tok_row_kernel<<<s.num_sms * 8, 256, 0, static_cast<cudaStream_t>(stream)>>>(s.doc_ptr32, s.row_off32,
-                                                                                    s.doc_map, s.tok_row, s.D);
+        tok_row_kernel<<<static_cast<unsigned>((s.D + 7) / 8), 256, 0, static_cast<cudaStream_t>(stream)>>>(
+            s.doc_ptr32, s.row_off32, s.doc_map, s.tok_row, s.D);
     return cudaGetLastError();
 }
 

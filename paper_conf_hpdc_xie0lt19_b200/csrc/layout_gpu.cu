@@ -28,6 +28,7 @@ constexpr int kRsBlock = 8 * kRsWarpItems;       // 4096 elements per block
 constexpr int kRadix = 256;
 constexpr int kScanChunk = 4096;
 constexpr unsigned kAll = 0xffffffffu;
+static_assert(kRsThreads == kRadix, "rs_scatter_kernel: one thread per digit");
 
 // keys may alias words (each thread reads words[i] before writing keys[i]);
 // rowof (optional): the θ row of token i's document, in document order
@@ -145,56 +146,95 @@ __global__ void scan_chunks_kernel(uint32_t *__restrict__ a, uint64_t L, const u
 // stable scatter of one digit pass: warp w of block b owns elements
 // [b·4096 + 512w, +512) and places them, in index order, after every element
 // with a smaller digit and after the same digit's elements of earlier warps
-// and blocks (hist: the scanned digit-major block histograms)
+// and blocks (hist: the scanned digit-major block histograms).  A lane holds
+// its 16 elements in registers (all loads issued up front), ranks them within
+// the warp with match_any once, and the block reorders its 4096 elements by
+// digit in shared memory first, so that consecutive threads store
+// consecutive addresses of a digit's run (coalesced) instead of 32 lanes
+// storing into 32 different runs.
 __global__ void __launch_bounds__(kRsThreads) rs_scatter_kernel(const uint32_t *__restrict__ kin,
                                                                 const uint32_t *__restrict__ vin,
                                                                 uint32_t *__restrict__ kout,
                                                                 uint32_t *__restrict__ vout, uint64_t n, int shift,
                                                                 uint32_t mask, uint32_t nblocks,
                                                                 const uint32_t *__restrict__ hist) {
-    __shared__ uint32_t wcnt[8][kRadix];
+    constexpr int kIt = kRsWarpItems / 32;  // 16 elements per lane
+    __shared__ uint32_t wcnt[8][kRadix];    // per-warp digit counts, then the warp's start in the block
+    __shared__ uint32_t lstart[kRadix];     // block-local start of each digit's run
+    __shared__ uint32_t gbase[kRadix];      // the block's global start of each digit's run
+    __shared__ uint32_t wsum[8];
+    __shared__ uint32_t sk[kRsBlock], sv[kRsBlock];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (int d = lane; d < kRadix; d += 32) wcnt[warp][d] = 0u;
     __syncwarp();
-    const uint64_t w0 = static_cast<uint64_t>(blockIdx.x) * kRsBlock + static_cast<uint64_t>(warp) * kRsWarpItems;
+    const uint64_t b0 = static_cast<uint64_t>(blockIdx.x) * kRsBlock;
+    const uint64_t w0 = b0 + static_cast<uint64_t>(warp) * kRsWarpItems;
     const unsigned lt = (1u << lane) - 1u;
-    // pass A: the warp's digit counts
-    for (int r = 0; r < kRsWarpItems; r += 32) {
-        const uint64_t i = w0 + r + lane;
-        const uint32_t d = i < n ? (kin[i] >> shift) & mask : kRadix + lane;
+    uint32_t k[kIt], v[kIt], off[kIt];
+#pragma unroll
+    for (int r = 0; r < kIt; ++r) {
+        const uint64_t i = w0 + 32 * r + lane;
+        k[r] = i < n ? kin[i] : 0u;
+        v[r] = i < n ? vin[i] : 0u;
+    }
+    // the warp's digit counts; off = the element's rank among the warp's
+    // elements of its digit
+#pragma unroll
+    for (int r = 0; r < kIt; ++r) {
+        const uint64_t i = w0 + 32 * r + lane;
+        const uint32_t d = i < n ? (k[r] >> shift) & mask : kRadix + lane;
         const unsigned peers = __match_any_sync(kAll, d);
+        off[r] = 0u;
+        if (i < n) off[r] = wcnt[warp][d] + __popc(peers & lt);
+        __syncwarp();
         if (i < n && (peers & lt) == 0u) wcnt[warp][d] += __popc(peers);
         __syncwarp();
     }
     __syncthreads();
-    // each warp's start for every digit
-    for (int d = threadIdx.x; d < kRadix; d += blockDim.x) {
-        uint32_t base = hist[static_cast<uint64_t>(d) * nblocks + blockIdx.x];
+    // per digit (thread d): the warps' starts inside the digit's block run,
+    // the run's length, then an exclusive scan of the lengths over digits
+    uint32_t len = 0;
+    {
+        const int d = threadIdx.x;  // kRsThreads == kRadix
         for (int w = 0; w < 8; ++w) {
             const uint32_t c = wcnt[w][d];
-            wcnt[w][d] = base;
-            base += c;
+            wcnt[w][d] = len;
+            len += c;
+        }
+        gbase[d] = hist[static_cast<uint64_t>(d) * nblocks + blockIdx.x];
+        uint32_t x = len;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(kAll, x, o);
+            if (lane >= o) x += y;
+        }
+        if (lane == 31) wsum[warp] = x;
+        __syncthreads();
+        uint32_t pre = 0;
+        for (int w = 0; w < warp; ++w) pre += wsum[w];
+        lstart[d] = pre + x - len;
+    }
+    __syncthreads();
+    // block-local placement in digit order
+#pragma unroll
+    for (int r = 0; r < kIt; ++r) {
+        const uint64_t i = w0 + 32 * r + lane;
+        if (i < n) {
+            const uint32_t d = (k[r] >> shift) & mask;
+            const uint32_t lp = lstart[d] + wcnt[warp][d] + off[r];
+            sk[lp] = k[r];
+            sv[lp] = v[r];
         }
     }
     __syncthreads();
-    // pass B: place the warp's elements in order
-    for (int r = 0; r < kRsWarpItems; r += 32) {
-        const uint64_t i = w0 + r + lane;
-        uint32_t k = 0, v = 0, d = kRadix + lane;
-        if (i < n) {
-            k = kin[i];
-            v = vin[i];
-            d = (k >> shift) & mask;
-        }
-        const unsigned peers = __match_any_sync(kAll, d);
-        if (i < n) {
-            const uint32_t pos = wcnt[warp][d] + __popc(peers & lt);
-            kout[pos] = k;
-            vout[pos] = v;
-        }
-        __syncwarp();
-        if (i < n && (peers & lt) == 0u) wcnt[warp][d] += __popc(peers);
-        __syncwarp();
+    // coalesced stores: element t of the block's digit-ordered run
+    const uint32_t nb = static_cast<uint32_t>(n - b0 < static_cast<uint64_t>(kRsBlock) ? n - b0 : kRsBlock);
+    for (uint32_t t = threadIdx.x; t < nb; t += kRsThreads) {
+        const uint32_t kk = sk[t];
+        const uint32_t d = (kk >> shift) & mask;
+        const uint32_t pos = gbase[d] + (t - lstart[d]);
+        kout[pos] = kk;
+        vout[pos] = sv[t];
     }
 }
 
