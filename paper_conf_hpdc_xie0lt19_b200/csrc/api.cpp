@@ -1070,7 +1070,7 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
             r = lda::launch_layout_keys(d_doc_ptr, reinterpret_cast<const int32_t *>(S.tok_row), d_tail, d_tile_doc,
                                         ndt, V, Dg, keys, vals, S.num_sms, ss);
         if (ce == cudaSuccess && r == 0) r = lda::radix_sort_pairs(keys, vals, ktmp, vtmp, n, bits, rtmp, ss, &in_tmp);
-        if (ce == cudaSuccess && r == 0) r = lda::launch_invert(in_tmp ? vtmp : vals, S.doc_map, n, S.num_sms, ss);
+        if (ce == cudaSuccess && r == 0) r = lda::launch_invert(in_tmp ? vtmp : vals, S.doc_map, n, ss);
         if (ce == cudaSuccess && r != 0) ce = static_cast<cudaError_t>(r);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(ss);
         sort_kernels_ms = now_ms();

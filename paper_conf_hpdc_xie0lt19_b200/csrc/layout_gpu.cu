@@ -30,12 +30,10 @@ constexpr int kScanChunk = 4096;
 constexpr unsigned kAll = 0xffffffffu;
 static_assert(kRsThreads == kRadix, "rs_scatter_kernel: one thread per digit");
 
-// keys may alias words (each thread reads words[i] before writing keys[i]);
-// rowof (optional): the θ row of token i's document, in document order
+// keys may alias words (each thread reads words[i] before writing keys[i])
 __global__ void layout_keys_kernel(const uint32_t *__restrict__ doc_ptr32, const int32_t *words,
                                    const uint8_t *__restrict__ tail, const uint32_t *__restrict__ tile_doc, int ndt,
-                                   uint32_t V, int64_t D, uint32_t *keys, uint32_t *__restrict__ vals,
-                                   const uint32_t *__restrict__ row_off32, uint32_t *__restrict__ rowof) {
+                                   uint32_t V, int64_t D, uint32_t *keys, uint32_t *__restrict__ vals) {
     const int lane = threadIdx.x & 31;
     const int64_t nw = static_cast<int64_t>(gridDim.x) * (blockDim.x >> 5);
     for (int64_t d = static_cast<int64_t>(blockIdx.x) * (blockDim.x >> 5) + (threadIdx.x >> 5); d < D; d += nw) {
@@ -48,12 +46,10 @@ __global__ void layout_keys_kernel(const uint32_t *__restrict__ doc_ptr32, const
         }
         const uint32_t tbase = static_cast<uint32_t>(lo) * V, tailbase = static_cast<uint32_t>(ndt) * V;
         const uint32_t s = doc_ptr32[d], e = doc_ptr32[d + 1];
-        const uint32_t row = rowof ? row_off32[d] : 0u;
         for (uint32_t i = s + lane; i < e; i += 32) {
             const uint32_t w = static_cast<uint32_t>(words[i]);
             keys[i] = (tail[w] ? tailbase : tbase) + w;
             vals[i] = i;
-            if (rowof) rowof[i] = row;
         }
     }
 }
@@ -238,19 +234,14 @@ __global__ void __launch_bounds__(kRsThreads) rs_scatter_kernel(const uint32_t *
     }
 }
 
-// doc_map[vals[p]] = p, and (rowof) tok_row[p] = rowof[vals[p]].  One
-// thread per position and no grid-stride loop: blocks start in position
-// order, so the scattered stores of the blocks in flight stay inside one
-// document tile's part of doc_map (L2-resident; a grid-stride loop lets the
-// blocks drift apart and the stores miss L2: 24.6 ms -> see DESIGN §6.4)
-__global__ void invert_kernel(const uint32_t *__restrict__ vals, uint32_t *__restrict__ doc_map, uint64_t n,
-                              const uint32_t *__restrict__ rowof, uint32_t *__restrict__ tok_row) {
+// doc_map[vals[p]] = p.  One thread per position and no grid-stride loop:
+// blocks start in position order, so the scattered stores of the blocks in
+// flight stay inside one document tile's part of doc_map (L2-resident; a
+// grid-stride loop lets the blocks drift apart and the stores miss L2:
+// 24.6 -> 9.7 ms at PubMed shape)
+__global__ void invert_kernel(const uint32_t *__restrict__ vals, uint32_t *__restrict__ doc_map, uint64_t n) {
     const uint64_t p = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-    if (p < n) {
-        const uint32_t i = vals[p];
-        doc_map[i] = static_cast<uint32_t>(p);
-        if (rowof) tok_row[p] = rowof[i];
-    }
+    if (p < n) doc_map[vals[p]] = static_cast<uint32_t>(p);
 }
 
 }  // namespace
@@ -287,20 +278,17 @@ int radix_sort_pairs(uint32_t *keys, uint32_t *vals, uint32_t *keys_tmp, uint32_
 }
 
 int launch_layout_keys(const uint32_t *doc_ptr32, const int32_t *words, const uint8_t *tail, const uint32_t *tile_doc,
-                       int ndt, int32_t V, int64_t D, uint32_t *keys, uint32_t *vals, int num_sms, void *stream,
-                       const uint32_t *row_off32, uint32_t *rowof) {
+                       int ndt, int32_t V, int64_t D, uint32_t *keys, uint32_t *vals, int num_sms, void *stream) {
     if (D > 0)
         layout_keys_kernel<<<num_sms * 8, 256, 0, static_cast<cudaStream_t>(stream)>>>(
-            doc_ptr32, words, tail, tile_doc, ndt, static_cast<uint32_t>(V), D, keys, vals, row_off32, rowof);
+            doc_ptr32, words, tail, tile_doc, ndt, static_cast<uint32_t>(V), D, keys, vals);
     return cudaGetLastError();
 }
 
-int launch_invert(const uint32_t *vals, uint32_t *doc_map, uint64_t n, int num_sms, void *stream,
-                  const uint32_t *rowof, uint32_t *tok_row) {
-    (void)num_sms;
+int launch_invert(const uint32_t *vals, uint32_t *doc_map, uint64_t n, void *stream) {
     if (n > 0)
         invert_kernel<<<static_cast<unsigned>((n + 255) / 256), 256, 0, static_cast<cudaStream_t>(stream)>>>(
-            vals, doc_map, n, rowof, tok_row);
+            vals, doc_map, n);
     return cudaGetLastError();
 }
 

@@ -233,19 +233,17 @@ int launch_loglik(const DevState &s, bool word_part, void *stream, int *launches
 
 // layout_gpu.cu: the doc-word map of the tile layout built on the device.
 // keys[i] = (tail[w] ? ndt : tile(d(i)))·V + w, vals[i] = i for every token i
-// keys may alias words; rowof (optional, T entries): rowof[i] = row_off32[d(i)]
+// (keys may alias words)
 int launch_layout_keys(const uint32_t *doc_ptr32, const int32_t *words, const uint8_t *tail, const uint32_t *tile_doc,
-                       int ndt, int32_t V, int64_t D, uint32_t *keys, uint32_t *vals, int num_sms, void *stream,
-                       const uint32_t *row_off32 = nullptr, uint32_t *rowof = nullptr);
+                       int ndt, int32_t V, int64_t D, uint32_t *keys, uint32_t *vals, int num_sms, void *stream);
 // stable LSD radix sort of (keys, vals) by the low `bits` key bits (8 per
 // pass); the result is in (keys_tmp, vals_tmp) when *result_in_tmp, else in
 // (keys, vals); temp: radix_sort_temp_words(n) words
 size_t radix_sort_temp_words(uint64_t n);
 int radix_sort_pairs(uint32_t *keys, uint32_t *vals, uint32_t *keys_tmp, uint32_t *vals_tmp, uint64_t n, int bits,
                      uint32_t *temp, void *stream, bool *result_in_tmp);
-// doc_map[vals[p]] = p; with rowof also tok_row[p] = rowof[vals[p]]
-int launch_invert(const uint32_t *vals, uint32_t *doc_map, uint64_t n, int num_sms, void *stream,
-                  const uint32_t *rowof = nullptr, uint32_t *tok_row = nullptr);
+// doc_map[vals[p]] = p
+int launch_invert(const uint32_t *vals, uint32_t *doc_map, uint64_t n, void *stream);
 
 // ---------------------------------------------------------------------------
 // The exchange of Eq. 4 (L935-937), comm.cpp.  All calls return an lda_status

@@ -15,7 +15,9 @@ from paper_conf_hpdc_xie0lt19_b200 import synth  # noqa: E402
 doc_ptr, words = synth.to_numpy(*synth.generate(300, 400, 20_000, 0.7, 16, 7, "cpu"))[:2]
 for K, opts in [(64, dict(sampler=2, tile_tokens=5000)), (64, dict(sampler=3, tile_tokens=5000)),
                 (64, dict(sampler=2, fused_recount=1, tile_tokens=5000)), (37, dict(sampler=2)),
-                (5000, dict(sampler=3, tile_tokens=3000)), (64, dict(sampler=0)),
+                (5000, dict(sampler=3, tile_tokens=3000)),
+                (5000, dict(sampler=3, tile_tokens=3000, sparse_words=-1)),   # f2 sparse word rows
+                (5000, dict(sampler=3, sparse_words=1 << 30)), (64, dict(sampler=0)),
                 (64, dict(exclude_self=1)), (20000, {}), (64, dict(stream_chunks=3, tile_tokens=5000)),
                 (64, dict(sampler=2, certify_slack=1 << 20))]:
     m = L.LDA(300, 400, K, 50.0 / K, 0.01, loglik_every=2, **opts).load(doc_ptr, words, 3)
