@@ -50,9 +50,11 @@ def test_options_validation():
         L.lda_set_option(ctx, "tile_tokens", 0)
         L.lda_set_option(ctx, "tile_tokens", -1)
         L.lda_set_option(ctx, "loglik_every", 5)
+        for v in (-1, 0, 4096):
+            L.lda_set_option(ctx, "sparse_words", v)   # f2: -1 = K/4, 0 = off, n = threshold
         for key, val in [("exclude_self", 2), ("chunk_tokens", 1), ("nonsense", 1), ("device", -1),
                          ("sampler", 1), ("tile_tokens", -2), ("loglik_every", -1), ("theta_mode", 1),
-                         ("filter32", 1)]:
+                         ("filter32", 1), ("sparse_words", -2)]:
             with pytest.raises(L.LDAError) as e:
                 L.lda_set_option(ctx, key, val)
             assert e.value.code == L.LDA_EINVAL
