@@ -562,6 +562,9 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_F32X2
 #define LDA_F32X2 1  // the walk's block sums with packed fp32 pairs (FFMA2)
 #endif
+#ifndef LDA_DENSE4
+#define LDA_DENSE4 1  // the dense in-chunk search 4-ary (4 dependent loads instead of 7)
+#endif
 #ifndef LDA_TILE_WPC
 #define LDA_TILE_WPC 8
 #endif
@@ -1054,6 +1057,28 @@ __device__ __forceinline__ void tile_walk(const TileArgs &a, uint32_t lsum, cons
     if (!hooked) at_step2();
 }
 
+// The last c in [0, n) with P[c] <= y, for non-decreasing P with P[0] <= y
+// (the dense bucket's fp64 chunk / group bases).  4-ary while n > 3: three
+// independent probes per level, so about half the dependent shared loads of
+// a binary search (the draw is latency-bound); the same c as a binary search.
+__device__ __forceinline__ int last_le(const double *P, int n, double y) {
+    int c = 0;
+#if LDA_DENSE4
+    while (n > 3) {
+        const int q = n >> 2;
+        const int cnt = (P[c + q] <= y) + (P[c + 2 * q] <= y) + (P[c + 3 * q] <= y);
+        c += cnt * q;
+        n = cnt == 3 ? n - 3 * q : q;
+    }
+#endif
+    while (n > 1) {
+        const int h = n >> 1;
+        if (P[c + h] <= y) c += h;
+        n -= h;
+    }
+    return c;
+}
+
 // Draw of one token of a tile-sampler batch (lane per token, `take` lanes):
 // Every search runs on the approximate (monotone) prefixes with plain
 // comparisons; the draw is then certified by the margins of the two prefixes
@@ -1138,12 +1163,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             // fp32 from p32 (p32 2u, α u, <= 32 FMA roundings: 35u)
             const double y = U * Q64 - (1.0 - U) * S;
             const double ey = (1.0 - U) * gS * S + eps;
-            int g = 0;
-            for (int n = NC; n > 1;) {  // last group g with Pg[g] <= y
-                const int h = n >> 1;
-                if (Pc[g + h] <= y) g += h;
-                n -= h;
-            }
+            const int g = last_le(Pc, NC, y);  // last group g with Pg[g] <= y
             const double r = y - Pc[g];
             const float r32 = static_cast<float>(r);
             const float eR = static_cast<float>((ey + u * fabs(r)) * 1.0001 + 1e-30);
@@ -1177,7 +1197,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             const double y = U * Q64 - (1.0 - U) * S;
             const double ey = (1.0 - U) * gS * S + eps;
             int c = 0;
-            for (int n = NC; n > 1;) {  // last chunk c with Pc[c] <= y
+            for (int n = NC; n > 1;) {  // last chunk c with Pc[c] <= y (NC small: binary)
                 const int h = n >> 1;
                 if (Pc[c + h] <= y) c += h;
                 n -= h;
@@ -1187,6 +1207,20 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             const float eR = static_cast<float>((ey + u * fabs(r)) * 1.0001 + 1e-30);
             const int kb = 128 * c, kn = min(K, kb + 128) - kb;
             int k = 0;  // first k in the chunk with L32 > r (kn - 1 if none)
+#if LDA_DENSE4
+            if (kn == 128) {
+                // 4-ary: three independent probes per level (4 dependent
+                // shared loads instead of 7).  Same k when L32 is monotone;
+                // any other k fails the bracket certification below.
+#pragma unroll
+                for (int g = 32; g >= 2; g >>= 2) {
+                    const float a0 = L32[l32_idx(kb + k + g - 1)], a1 = L32[l32_idx(kb + k + 2 * g - 1)];
+                    const float a2 = L32[l32_idx(kb + k + 3 * g - 1)];
+                    k += g * ((a0 <= r32) + (a1 <= r32) + (a2 <= r32));
+                }
+                if (L32[l32_idx(kb + k)] <= r32) k += 1;
+            } else
+#endif
             for (int n = kn; n > 1;) {
                 const int h = n >> 1;
                 if (L32[l32_idx(kb + k + h - 1)] <= r32) k += h;
