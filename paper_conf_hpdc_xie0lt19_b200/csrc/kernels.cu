@@ -562,6 +562,9 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_F32X2
 #define LDA_F32X2 1  // the walk's block sums with packed fp32 pairs (FFMA2)
 #endif
+#ifndef LDA_LCACHE
+#define LDA_LCACHE 1  // the draw keeps the prefixes after the first 3 θ-row lines from the S pass
+#endif
 #ifndef LDA_DENSE4
 #define LDA_DENSE4 1  // the dense in-chunk search 4-ary (4 dependent loads instead of 7)
 #endif
@@ -1096,7 +1099,19 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
     x0 = 0;
     if (take) {
         double S = 0.0;
+#if LDA_LCACHE
+        // the prefixes after lines 0..2, kept for the sparse search below
+        // (the same doubles it would recompute, in the same order)
+        double P0 = 0.0, P1 = 0.0, P2 = 0.0;
+        for (uint32_t i = 0; i < nl; ++i) {
+            S += f2d_pos(line_sum(blk, c0 + i));
+            if (i == 0) P0 = S;
+            if (i == 1) P1 = S;
+            if (i == 2) P2 = S;
+        }
+#else
         for (uint32_t i = 0; i < nl; ++i) S += f2d_pos(line_sum(blk, c0 + i));
+#endif
         x0 = philox_x0_sched(cb + crank, a.t, a.key0, a.key1);
         const double U = (__hiloint2double(0x43300000, static_cast<int>(x0)) - 4503599627370496.0) *
                          2.3283064365386962890625e-10;  // x0·2^-32, exact
@@ -1112,11 +1127,32 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             // sparse bucket: the line, then the block, whose end prefix first exceeds x
             double C = 0.0, Cn = 0.0;
             uint32_t i = 0;
+#if LDA_LCACHE
+            if (P0 > x || nl <= 1) {
+                Cn = P0;
+            } else if (P1 > x || nl <= 2) {
+                i = 1;
+                C = P0;
+                Cn = P1;
+            } else if (P2 > x || nl <= 3) {
+                i = 2;
+                C = P1;
+                Cn = P2;
+            } else {
+                C = P2;
+                for (i = 3;; ++i) {
+                    Cn = C + f2d_pos(line_sum(blk, c0 + i));
+                    if (Cn > x || i + 1 >= nl) break;
+                    C = Cn;
+                }
+            }
+#else
             for (;; ++i) {
                 Cn = C + f2d_pos(line_sum(blk, c0 + i));
                 if (Cn > x || i + 1 >= nl) break;
                 C = Cn;
             }
+#endif
             const float *bk = blk + 4 * (c0 + i);
             uint32_t b = 0;
             for (; b < 3; ++b) {
