@@ -565,6 +565,9 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_LCACHE
 #define LDA_LCACHE 1  // the draw keeps the prefixes after the first 3 θ-row lines from the S pass
 #endif
+#ifndef LDA_BSEL
+#define LDA_BSEL 1  // the draw's block search branch-free
+#endif
 #ifndef LDA_DENSE4
 #define LDA_DENSE4 1  // the dense in-chunk search 4-ary (4 dependent loads instead of 7)
 #endif
@@ -1155,6 +1158,19 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
 #endif
             const float *bk = blk + 4 * (c0 + i);
             uint32_t b = 0;
+#if LDA_BSEL
+            {
+                // the block: branch-free over the line's first three block-end
+                // prefixes (the same doubles as the sequential scan)
+                const float4 bq = *reinterpret_cast<const float4 *>(bk);
+                const double C1 = C + f2d_pos(bq.x), C2 = C1 + f2d_pos(bq.y), C3 = C2 + f2d_pos(bq.z);
+                const bool g1 = C1 > x, g2 = C2 > x, g3 = C3 > x;
+                b = g1 ? 0u : g2 ? 1u : g3 ? 2u : 3u;
+                const double Cp = g1 ? C : g2 ? C1 : g3 ? C2 : C3;
+                Cn = g1 ? C1 : g2 ? C2 : g3 ? C3 : Cn;
+                C = Cp;
+            }
+#else
             for (; b < 3; ++b) {
                 const double Cb = C + f2d_pos(bk[b]);
                 if (Cb > x) {
@@ -1163,6 +1179,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
                 }
                 C = Cb;
             }
+#endif
             // certify: C <= x < Cn with margins (C = 0 needs none)
             flag = (x - C <= gS * C + eX && C > 0.0) || (Cn - x <= gS * Cn + eX);
             b += 4 * i;
