@@ -565,6 +565,9 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_LCACHE
 #define LDA_LCACHE 1  // the draw keeps the prefixes after the first 3 θ-row lines from the S pass
 #endif
+#ifndef LDA_LSEL
+#define LDA_LSEL 1  // the draw's line selection (first three lines) branch-free
+#endif
 #ifndef LDA_BSEL
 #define LDA_BSEL 1  // the draw's block search branch-free
 #endif
@@ -1131,6 +1134,22 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             double C = 0.0, Cn = 0.0;
             uint32_t i = 0;
 #if LDA_LCACHE
+#if LDA_LSEL
+            {
+                // branch-free over the first three lines (the common case)
+                const bool s0 = P0 > x || nl <= 1, s1 = P1 > x || nl <= 2, s2 = P2 > x || nl <= 3;
+                i = s0 ? 0u : s1 ? 1u : s2 ? 2u : 3u;
+                C = s0 ? 0.0 : s1 ? P0 : s2 ? P1 : P2;
+                Cn = s0 ? P0 : s1 ? P1 : P2;
+            }
+            if (i == 3) {
+                for (;; ++i) {
+                    Cn = C + f2d_pos(line_sum(blk, c0 + i));
+                    if (Cn > x || i + 1 >= nl) break;
+                    C = Cn;
+                }
+            }
+#else
             if (P0 > x || nl <= 1) {
                 Cn = P0;
             } else if (P1 > x || nl <= 2) {
@@ -1149,6 +1168,7 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
                     C = Cn;
                 }
             }
+#endif
 #else
             for (;; ++i) {
                 Cn = C + f2d_pos(line_sum(blk, c0 + i));
