@@ -565,6 +565,9 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_LCACHE
 #define LDA_LCACHE 1  // the draw keeps the prefixes after the first 3 θ-row lines from the S pass
 #endif
+#ifndef LDA_NC8
+#define LDA_NC8 1  // the dense chunk search specialised for 8 chunks (K = 1024)
+#endif
 #ifndef LDA_LSEL
 #define LDA_LSEL 1  // the draw's line selection (first three lines) branch-free
 #endif
@@ -1270,6 +1273,12 @@ __device__ __forceinline__ void tile_draw(const TileArgs &a, bool take, uint32_t
             const double y = U * Q64 - (1.0 - U) * S;
             const double ey = (1.0 - U) * gS * S + eps;
             int c = 0;
+#if LDA_NC8
+            if (NC == 8) {  // K = 1024: two rounds of independent probes instead of three dependent ones
+                c = 2 * ((Pc[2] <= y) + (Pc[4] <= y) + (Pc[6] <= y));
+                c += Pc[c + 1] <= y;
+            } else
+#endif
             for (int n = NC; n > 1;) {  // last chunk c with Pc[c] <= y (NC small: binary)
                 const int h = n >> 1;
                 if (Pc[c + h] <= y) c += h;
