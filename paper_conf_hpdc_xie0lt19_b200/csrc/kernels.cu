@@ -565,6 +565,9 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_LCACHE
 #define LDA_LCACHE 1  // the draw keeps the prefixes after the first 3 θ-row lines from the S pass
 #endif
+#ifndef LDA_BALLOT_SCAN
+#define LDA_BALLOT_SCAN 1  // the batch head's line-count prefix by ballots (K < 2016)
+#endif
 #ifndef LDA_NC8
 #define LDA_NC8 1  // the dense chunk search specialised for 8 chunks (K = 1024)
 #endif
@@ -974,10 +977,22 @@ __device__ __forceinline__ TileHead tile_head(const TileArgs &a, uint32_t row, u
     h.nl = valid ? (nnz + 32u) >> 5 : 0u;  // 128-byte lines holding words 0..nnz
     const uint32_t nlw = h.dup ? 0u : h.nl;
     uint32_t incl = nlw;
+#if LDA_BALLOT_SCAN
+    if (a.K <= 2015) {
+        // nlw < 64: the inclusive prefix by bit planes (six independent
+        // ballots instead of five dependent shuffle rounds)
+        const unsigned le = 0xFFFFFFFFu >> (31 - lane);
+        incl = 0u;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
+        for (int bp = 0; bp < 6; ++bp) incl += static_cast<uint32_t>(__popc(__ballot_sync(kFull, (nlw >> bp) & 1u) & le)) << bp;
+    } else
+#endif
+    {
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += y;
+        }
     }
     h.take = valid && (incl <= static_cast<uint32_t>(LM) || lane == 0);
     h.nb = __popc(__ballot_sync(kFull, h.take));
