@@ -7,10 +7,15 @@ TAG=${1:-r02}
 OUT=gpurun_out; mkdir -p $OUT
 timeout 2400 python -m pytest tests -m gpu -q -rA -p no:cacheprovider > $OUT/${TAG}_pytest.log 2>&1; echo "pytest exit $?" >> $OUT/${TAG}_pytest.log
 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/${TAG}_smoke.log 2>&1
+# the bench lines first (their e2e loads measured 0.25 s standalone but up
+# to 0.40 s right after the ncu captures on the same box); roofline.traffic
+# comes from the committed profiles/traffic.json (the previous capture)
+for c in pubmed nytimes nytimes_k128 nytimes_k8192 pubmed_x5; do
+  timeout 900 python bench.py --config $c --steps 20 --warmup 3 > $OUT/bench_${TAG}_$c.json 2> $OUT/bench_${TAG}_$c.err
+done
 bash tools/ncu_configs.sh $TAG pubmed nytimes nytimes_k128 nytimes_k8192 pubmed_x5
 cp profiles/traffic.json $OUT/traffic_${TAG}.json
 for c in pubmed nytimes nytimes_k128 nytimes_k8192 pubmed_x5; do
-  timeout 900 python bench.py --config $c --steps 20 --warmup 3 > $OUT/bench_${TAG}_$c.json 2> $OUT/bench_${TAG}_$c.err
   k=$( [ $c = nytimes_k8192 ] && echo sweep_tile_cta || echo sweep_tile )
   python tools/profile_md.py $OUT/prof_${TAG}_$c.ncu-rep $k "sampling kernel, $c, $TAG" > $OUT/${TAG}_${c}_profile.md 2>&1
 done
