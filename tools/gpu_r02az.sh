@@ -1,0 +1,8 @@
+OUT=gpurun_out; mkdir -p $OUT
+for c in pubmed nytimes nytimes_k128 nytimes_k8192 pubmed_x5; do
+  timeout 900 python bench.py --config $c --steps 20 --warmup 3 > $OUT/bench_r02i_$c.json 2> $OUT/bench_r02i_$c.err
+  python -c "
+import json
+d=json.loads(open('$OUT/bench_r02i_$c.json').read().strip().splitlines()[-1]); r=d['roofline']
+print('$c', round(d['value']/1e9,3), round(d['ms_per_step'],2), round(r['frac'],3), round(r['sweep_frac'],3), r['dram_frac'] and round(r['dram_frac'],3), round(d['e2e']['value']/1e9,3), d['e2e']['breakdown'], d['clocks'])" 2>&1 | tail -1
+done
