@@ -261,6 +261,15 @@ int lda_layout_selfcheck(int64_t D, int32_t V, int32_t K, const int64_t *doc_ptr
 int lda_debug_radix_sort(const uint32_t *keys, const uint32_t *vals, int64_t n, int32_t bits, uint32_t *out_keys,
                          uint32_t *out_vals);
 
+/* Diagnostic (tests): the NCCL backend of the exchange end to end with one
+ * rank on `device` (this environment has one GPU; NCCL refuses two ranks on
+ * one device): dlopen of libnccl.so.2 and its symbols, ncclGetUniqueId,
+ * ncclCommInitRank, the three collectives the library issues (in place, on
+ * a stream) and ncclCommDestroy; with one rank each collective is the
+ * identity, which is checked.  Returns 0, LDA_ENCCL or LDA_ECUDA, with a
+ * message in msg (msg_cap bytes). */
+int lda_debug_nccl_selftest(int32_t device, char *msg, int32_t msg_cap);
+
 /* Load this rank's documents [doc_begin, doc_end) of the global corpus,
  * randomly initialise every token's topic (L377-379; Philox at t = 0, X10)
  * and build n_wk, n_k and θ (allreduced across ranks when world > 1).

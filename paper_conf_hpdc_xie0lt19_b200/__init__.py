@@ -25,7 +25,7 @@ STATUS = {0: "LDA_OK", -1: "LDA_EINVAL", -2: "LDA_ERANGE", -3: "LDA_ENOMEM", -4:
 # every symbol include/lda.h declares
 ABI_SYMBOLS = ("lda_create", "lda_set_option", "lda_init_dist", "lda_nccl_unique_id", "lda_peer_group_create",
                "lda_init_peer", "lda_peer_group_destroy", "lda_partition_docs",
-               "lda_canonical_bases", "lda_layout_selfcheck", "lda_debug_radix_sort",
+               "lda_canonical_bases", "lda_layout_selfcheck", "lda_debug_radix_sort", "lda_debug_nccl_selftest",
                "lda_load_corpus", "lda_iterate", "lda_loglik", "lda_get_counts", "lda_get_stats",
                "lda_get_sweep_log", "lda_get_loglik_log", "lda_get_stream", "lda_set_z", "lda_destroy",
                "lda_last_error", "lda_version")
@@ -83,6 +83,7 @@ def lib():
                                       _i32], ctypes.c_int),
             "lda_load_corpus": ([_vp, _i64, _i64, _vp, _vp, _u64], ctypes.c_int),
             "lda_debug_radix_sort": ([_vp, _vp, _i64, _i32, _vp, _vp], ctypes.c_int),
+            "lda_debug_nccl_selftest": ([_i32, ctypes.c_char_p, _i32], ctypes.c_int),
             "lda_iterate": ([_vp, _i32], ctypes.c_int),
             "lda_loglik": ([_vp, ctypes.POINTER(_f64)], ctypes.c_int),
             "lda_get_counts": ([_vp, _vp, _vp, _vp, _vp, _vp, _i64, _vp, _vp], ctypes.c_int),
@@ -171,6 +172,15 @@ def lda_debug_radix_sort(keys, vals, bits):
     ok, ov = np.empty_like(k), np.empty_like(v)
     _check(lib().lda_debug_radix_sort(_p(k), _p(v), len(k), int(bits), _p(ok), _p(ov)))
     return ok, ov
+
+
+def lda_debug_nccl_selftest(device=0) -> str:
+    """The NCCL backend end to end with one rank (diagnostic); returns its message."""
+    buf = ctypes.create_string_buffer(512)
+    r = lib().lda_debug_nccl_selftest(int(device), buf, 512)
+    if r != LDA_OK:
+        raise LDAError(r, buf.value.decode())
+    return buf.value.decode()
 
 
 def lda_canonical_bases(word_counts, rank):

@@ -357,3 +357,62 @@ int make_peer_comm(const std::shared_ptr<PeerGroup> &g, int rank, int device, st
 }
 
 }  // namespace lda
+
+// Diagnostic (include/lda.h): the NCCL backend end to end with one rank on
+// `device` -- dlopen + symbols, ncclGetUniqueId, ncclCommInitRank, the three
+// collectives the library issues (in place, on a stream), ncclCommDestroy.
+// With one rank every collective is the identity, which is checked.
+extern "C" int lda_debug_nccl_selftest(int32_t device, char *msg, int32_t msg_cap) {
+    std::string err;
+    auto out = [&](int code, const std::string &m) {
+        if (msg && msg_cap > 0) {
+            std::strncpy(msg, m.c_str(), static_cast<size_t>(msg_cap) - 1);
+            msg[msg_cap - 1] = '\0';
+        }
+        return code;
+    };
+    unsigned char uid[128];
+    int r = lda::nccl_unique_id(uid, err);
+    if (r != LDA_OK) return out(r, err);
+    std::unique_ptr<lda::Comm> comm;
+    r = lda::make_nccl_comm(0, 1, uid, device, comm, err);
+    if (r != LDA_OK) return out(r, err);
+    const size_t n = 1000;
+    int32_t *di = nullptr;
+    double *dd = nullptr;
+    int64_t *dg = nullptr;
+    cudaStream_t s = nullptr;
+    cudaError_t ce = cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    if (ce == cudaSuccess) ce = cudaMalloc(&di, n * sizeof(int32_t));
+    if (ce == cudaSuccess) ce = cudaMalloc(&dd, n * sizeof(double));
+    if (ce == cudaSuccess) ce = cudaMalloc(&dg, 2 * n * sizeof(int64_t));
+    std::vector<int32_t> hi(n), hi2(n);
+    std::vector<double> hd(n), hd2(n);
+    std::vector<int64_t> hg(n), hg2(n);
+    for (size_t i = 0; i < n; ++i) {
+        hi[i] = static_cast<int32_t>(i * 7919 % 1000003) - 5;
+        hd[i] = 0.5 * static_cast<double>(i) - 3.25;
+        hg[i] = static_cast<int64_t>(i) * 1000000007LL;
+    }
+    if (ce == cudaSuccess) ce = cudaMemcpy(di, hi.data(), n * sizeof(int32_t), cudaMemcpyHostToDevice);
+    if (ce == cudaSuccess) ce = cudaMemcpy(dd, hd.data(), n * sizeof(double), cudaMemcpyHostToDevice);
+    if (ce == cudaSuccess) ce = cudaMemcpy(dg, hg.data(), n * sizeof(int64_t), cudaMemcpyHostToDevice);
+    if (ce == cudaSuccess && r == LDA_OK) r = comm->allreduce_i32(di, n, s, err);
+    if (ce == cudaSuccess && r == LDA_OK) r = comm->allreduce_f64(dd, n, s, err);
+    if (ce == cudaSuccess && r == LDA_OK) r = comm->allgather_i64(dg, dg + n, n, s, err);
+    if (ce == cudaSuccess && r == LDA_OK) ce = cudaStreamSynchronize(s);
+    if (ce == cudaSuccess && r == LDA_OK) ce = cudaMemcpy(hi2.data(), di, n * sizeof(int32_t), cudaMemcpyDeviceToHost);
+    if (ce == cudaSuccess && r == LDA_OK) ce = cudaMemcpy(hd2.data(), dd, n * sizeof(double), cudaMemcpyDeviceToHost);
+    if (ce == cudaSuccess && r == LDA_OK)
+        ce = cudaMemcpy(hg2.data(), dg + n, n * sizeof(int64_t), cudaMemcpyDeviceToHost);
+    if (di) cudaFree(di);
+    if (dd) cudaFree(dd);
+    if (dg) cudaFree(dg);
+    if (s) cudaStreamDestroy(s);
+    const std::string name = comm->name();
+    comm.reset();
+    if (ce != cudaSuccess) return out(LDA_ECUDA, cudaGetErrorString(ce));
+    if (r != LDA_OK) return out(r, err);
+    if (hi2 != hi || hd2 != hd || hg2 != hg) return out(LDA_ENCCL, "one-rank collectives changed the data");
+    return out(LDA_OK, name + ": one-rank allreduce(int32), allreduce(fp64), allgather(int64) ok");
+}

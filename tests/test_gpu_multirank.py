@@ -146,3 +146,15 @@ def test_world2_tiny_matches_oracle_and_set_z():
         bad = np.nonzero(zg != zs[s])[0]
         assert (margins[s - 1][bad] < U.MARGIN_EXCUSE).all()
         assert len(bad) <= U.MAX_EXCUSED_FRAC * c.T + 1
+
+
+def test_nccl_backend_one_rank():
+    """The NCCL data plane (one process per GPU) on this one-GPU box: NCCL
+    refuses two ranks on one device, so the backend runs end to end with one
+    rank -- dlopen of the process's libnccl.so.2, unique id, communicator,
+    the in-place int32 / fp64 allreduces and the int64 all-gather the library
+    issues, teardown -- and each collective must be the identity."""
+    import torch  # noqa: F401  (loads torch's NCCL first, as in bench.py)
+    import paper_conf_hpdc_xie0lt19_b200 as L
+    msg = L.lda_debug_nccl_selftest(0)
+    assert msg.startswith("nccl:"), msg
