@@ -559,6 +559,12 @@ __device__ __forceinline__ f32x2 mass_f32x2(uint32_t e0, uint32_t e1, const floa
 #ifndef LDA_TRING
 #define LDA_TRING 3
 #endif
+#ifndef LDA_CTA_NBUF_MAX
+#define LDA_CTA_NBUF_MAX 3   // large-K CTA sampler: table buffers per CTA (at most; 3: 16 warps, +2.5 % over 4 at K = 8192)
+#endif
+#ifndef LDA_CTA_MIN_WARPS
+#define LDA_CTA_MIN_WARPS 12  // ...as long as at least this many warps fit beside them
+#endif
 #ifndef LDA_TRING_GNK
 #define LDA_TRING_GNK 3  // the large-K CTA sampler's ring (4: +0.5 % at K = 8192 alone, -0.2 % with the early line-table reads)
 #endif
@@ -2190,8 +2196,8 @@ int configure_kernels(DevState &s) {
         };
         s.tile_nbuf = 2;
         if (s.tile_cta_gnk)
-            for (int nb = 4; nb > 2; --nb)
-                if (fit(nb) >= 12) {
+            for (int nb = LDA_CTA_NBUF_MAX; nb > 2; --nb)
+                if (fit(nb) >= LDA_CTA_MIN_WARPS) {
                     s.tile_nbuf = nb;
                     break;
                 }
