@@ -353,7 +353,7 @@ int load_chunked(lda_ctx *ctx, const int64_t *doc_ptr, const int32_t *words, int
                                          : std::max<int64_t>(int64_t(1) << 20,
                                                              static_cast<int64_t>(c->T * (target / (32.0 * r32))));
         }
-        std::string e = lda::build_layout(dp.data(), words + t0, c->D, V, K, cb.data(), tile * kscale,
+        std::string e = lda::build_layout(dp.data(), words + t0, c->D, V, K, cb.data(), tile,
                                           ctx->chunk_tokens, ctx->recount_tokens, ctx->threads, 2,
                                           ctx->tail_per_tile * kscale, c->H, {}, wc.data(), /*host_tok_row=*/true);
         if (!e.empty()) return fail(ctx, LDA_ERANGE, e);
@@ -1097,11 +1097,13 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
         }
         cv.notify_all();
     };
-    // the large-K sampler copies a table of 8·K bytes per work item: its items
-    // grow with K (tiles and the tail threshold scaled by K/1024; measured at
-    // K = 8192 on the NYTimes shape: 1.94 -> 2.4 G tokens/s)
+    // the large-K sampler copies a table of 4·K bytes per work item: words
+    // with few tokens per tile go to the tail tile at a threshold scaled by
+    // K/1024 (round 1, per-item tables: tiles scaled too, 1.94 -> 2.4 G
+    // tokens/s at K = 8192); with CTA-shared tables the tiles themselves are
+    // not scaled (5.31 -> 5.73 G tokens/s at NYTimes shape, K = 8192)
     const int64_t kscale = S.sweep_tile_cta ? std::max<int64_t>(1, K / 1024) : 1;
-    std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), tile_tokens * kscale,
+    std::string e = lda::build_layout(doc_ptr, words, Dg, V, K, cbase.data(), tile_tokens,
                                       ctx->chunk_tokens, ctx->recount_tokens, ctx->threads,
                                       tile_layout ? 2 : 0,
                                       ctx->tail_per_tile * kscale, H,
