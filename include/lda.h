@@ -139,9 +139,9 @@ int lda_create(int64_t D, int32_t V, int32_t K, double alpha, double beta, lda_c
  *                   only within fp64 rounding of it).
  *   "tail_per_tile" samplers 2, 3: words with fewer than this many tokens
  *                   per document tile on average are sampled as one
- *                   corpus-wide item each (default 64; 0 = off).  Sampler 3
- *                   scales it and tile_tokens by K/1024 (its per-item table
- *                   copy grows with K).
+ *                   corpus-wide item each (default 48; 0 = off).  Sampler 3
+ *                   scales it by K/1024 (its per-item table copy grows
+ *                   with K).
  *   "fused_recount" samplers 2, 3: 0 (default) = n_wk / n_k rebuilt after
  *                   the sampler by the segmented recount kernel (per-word
  *                   shared histograms over the word's runs, no global atomics

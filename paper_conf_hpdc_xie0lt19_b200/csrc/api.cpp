@@ -53,7 +53,7 @@ struct lda_ctx {
     int64_t recount_tokens = 65536;
     int64_t tile_tokens = -1;  // auto: tiles whose θ rows fill about half the L2
     int sampler = -1;  // auto
-    int64_t tail_per_tile = 64;
+    int64_t tail_per_tile = 48;  // measured: +1.9 % at PubMed shape over 64, neutral at NYTimes shape
     int64_t certify_slack = 1;
     int fused_recount = 0;  // segmented recount after the sampler (measured faster)
     int64_t comm_pipeline = 4;  // world > 1: word ranges whose rows are exchanged as soon as recounted (f1)
