@@ -1226,8 +1226,8 @@ int lda_load_corpus(lda_ctx *ctx, int64_t doc_begin, int64_t doc_end, const int6
     S.n_titems = static_cast<int64_t>(H.titems.size());
     S.n_zero_words = static_cast<int64_t>(H.zero_words.size());
     if (S.recount_gmem) {
-        DA(S.recount_scratch, static_cast<size_t>(S.num_sms) * 4 * 2 * K);
-        CU(cudaMemsetAsync(S.recount_scratch, 0, sizeof(int) * S.num_sms * 4 * 2 * static_cast<size_t>(K),
+        DA(S.recount_scratch, static_cast<size_t>(S.num_sms) * S.recount_bps * 2 * K);
+        CU(cudaMemsetAsync(S.recount_scratch, 0, sizeof(int) * S.num_sms * S.recount_bps * 2 * static_cast<size_t>(K),
                            ctx->stream));
     }
     if (S.theta_gmem) {

@@ -2323,7 +2323,7 @@ int launch_recount(const DevState &s, void *stream, int *launches, int64_t rc0, 
     }
     if (rc1 <= rc0) return cudaGetLastError();
     if ((e = cudaMemsetAsync(s.counter + 1, 0, sizeof(uint32_t), st)) != cudaSuccess) return e;
-    const int grid = static_cast<int>(std::min<int64_t>(rc1 - rc0, static_cast<int64_t>(s.num_sms) * 4));
+    const int grid = static_cast<int>(std::min<int64_t>(rc1 - rc0, static_cast<int64_t>(s.num_sms) * s.recount_bps));
     if (s.recount_gmem)
         recount_kernel<true><<<grid, 256, 0, st>>>(s.rchunks + rc0, rc1 - rc0, s.segs, s.K, s.tok_z, s.nwk, nk,
                                                   s.counter + 1, s.recount_scratch);

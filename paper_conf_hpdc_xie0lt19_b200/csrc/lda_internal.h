@@ -209,7 +209,8 @@ struct DevState {
     int sweep_grid = 0, sweep_block = 0;
     int theta_grid = 0, theta_block = 0;
     bool recount_gmem = false, theta_gmem = false;  // K > 16384: K-length histograms in global scratch
-    int *recount_scratch = nullptr;                 // recount_gmem: num_sms*4 CTAs x 2K
+    int recount_bps = 8;                            // recount CTAs per SM (8: 2.06 -> 1.11 ms at PubMed shape vs 4)
+    int *recount_scratch = nullptr;                 // recount_gmem: num_sms*recount_bps CTAs x 2K
     uint32_t *theta_scratch = nullptr;              // theta_gmem: theta_grid*8 warps x (K + K/32)
     size_t sweep_smem = 0, theta_smem = 0;
     int ll_blocks = 0;
